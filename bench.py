@@ -1,0 +1,391 @@
+#!/usr/bin/env python
+"""bench.py -- Gaussian pair-interactions/s of the fused kernel summation on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--cfg 3] [--impl ours|reference]
+
+One STEP is one pass of the whole hot path
+over one batch of synthetic input: ks_set_sources (a1: centre, norms,
+prescale, layout) + ks_eval (a2-a7: the fused kernel with its in-kernel
+cross-CTA fix-up).  With N > 1 GPUs (torchrun, one rank per GPU) the step
+also contains the NCCL broadcast of alpha/W and the all-gather of V (row e),
+and the targets are sharded (fixed total N: "strong" scaling).
+
+Workload (default): BASELINE.json configs[2] -- the headline metric's config:
+N = M = 65,536, K = 32, h = 1, R = 1, Gaussian mixture (16 centres,
+sigma = 0.1), W ~ U[0,1] (workloads/, seeded).  Inputs are resident in HBM
+before the timed region; L2 (126 MB) is flushed with a 256 MiB write before
+every step (outside the per-step CUDA events).
+
+Printed: one JSON line (rank 0) with value = pairs/s for the whole job,
+the device-timed ms/step (max over ranks), the roofline of the dominant
+(fused) kernel from CUDA events on its launching stream, e2e through the
+C-ABI host entry points (pinned host buffers, copies inside the timed
+region), the FP64 oracle as cpu_baseline on a bounded sample (rank 0), the
+SM clocks sampled during the timed region, and the count of our kernel
+launches in the timed region.
+
+--impl reference: the oracle itself (oracle/, plain FP64 CPU loop) timed on
+this host's cores, each step a bounded target sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import workloads  # noqa: E402
+
+METRIC = "Gaussian pair-interactions/sec (N=65,536, K=32) at 1/2/4/8 B200 + % roofline"
+UNIT = "pairs/s"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=10)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--cfg", type=int, default=3, help="BASELINE config id (1-based, SURVEY SS8(a))")
+    p.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
+    p.add_argument("--no-flush", action="store_true")
+    return p.parse_args()
+
+
+def workload_desc(c: workloads.Config) -> str:
+    dist = (f"Gaussian mixture (16 centres ~U[0,1]^K, sigma={c.sigma})" if c.dist == "gm"
+            else "uniform [0,1]^K")
+    return (f"cfg{c.cfg}: M=N={c.N:,} sources=targets count, K={c.K}, h={c.h}, R={c.R}, {dist}, "
+            f"W~U[0,1], seeds 2016{c.cfg}+(0,1,2,3)")
+
+
+def per_pair_ops(K: int, R: int):
+    """Algorithmic per-pair work charged to the pipe the FP32 design uses
+    (SS7): K FFMA (dot) + 1 FADD (norm init) + R FFMA (weight) on the
+    FP32 pipe, 1 MUFU ex2."""
+    return K + 1 + R, 1
+
+
+# ---------------------------------------------------------------- clocks (NVML, sampled during the timed region)
+class ClockSampler:
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+        0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+        0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
+    }
+
+    def __init__(self, dev_index: int, period: float = 0.05):
+        self.samples, self.reasons, self.ok = [], 0, False
+        self.period = period
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(dev_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover - no NVML
+            self.err = str(e)
+            self.max_mhz = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                self.reasons |= int(self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h))
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *exc):
+        self._stop.set()
+        if self.ok:
+            self.t.join()
+
+    def summary(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": [], "samples": 0}
+        names = [n for bit, n in self.REASONS.items() if self.reasons & bit and n != "gpu_idle"]
+        return {"sm_mhz": float(statistics.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": names, "samples": len(self.samples),
+                "sm_mhz_min": float(min(self.samples))}
+
+
+# ---------------------------------------------------------------- CPU baseline (the oracle)
+def cpu_baseline(a, W, b, h, cpu_seconds, seed=20163):
+    """Oracle (oracle/, as it stands) on all M sources x a bounded seeded target
+    sample; returns (dict, J, V_ref)."""
+    import oracle
+    oracle.build()
+    threads = len(os.sched_getaffinity(0))
+    oracle.set_num_threads(threads)
+    M, N = a.shape[0], b.shape[0]
+    J0 = workloads.sample_targets(N, 4 * threads, seed)
+    t0 = time.perf_counter()
+    oracle.oracle_eval(a, W, b, float(h), J=J0)
+    dt = max(time.perf_counter() - t0, 1e-4)
+    per_target = dt / len(J0)
+    n = int(max(16, min(N, cpu_seconds / per_target)))
+    J = workloads.sample_targets(N, n, seed + 1)
+    t0 = time.perf_counter()
+    Vr = oracle.oracle_eval(a, W, b, float(h), J=J)
+    dt = time.perf_counter() - t0
+    pairs = M * len(J)
+    return ({"value": pairs / dt, "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
+             "sample": f"all {M:,} sources x {len(J):,} seeded targets (of {N:,}); {dt:.1f} s; "
+                       f"FP64 direct-difference double loop, OpenMP over targets"},
+            J, Vr)
+
+
+# ---------------------------------------------------------------- reference arm
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    oracle.build()
+    c = workloads.CONFIGS[args.cfg]
+    a, W, b, h = workloads.make(c)
+    threads = len(os.sched_getaffinity(0))
+    oracle.set_num_threads(threads)
+    # size one step at ~3 s of CPU work
+    J0 = workloads.sample_targets(c.N, 4 * threads, 1)
+    t0 = time.perf_counter()
+    oracle.oracle_eval(a, W, b, float(h), J=J0)
+    per_t = max(time.perf_counter() - t0, 1e-4) / len(J0)
+    n = int(max(8, min(c.N, 3.0 / per_t)))
+    times = []
+    for s in range(args.warmup + args.steps):
+        J = workloads.sample_targets(c.N, n, 100 + s)[:n]
+        t0 = time.perf_counter()
+        oracle.oracle_eval(a, W, b, float(h), J=J)
+        if s >= args.warmup:
+            times.append((time.perf_counter() - t0, len(J)))
+    tot = sum(t for t, _ in times)
+    pairs = sum(c.M * m for _, m in times)
+    value = pairs / tot
+    out = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / len(times),
+           "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+           "data": "synthetic",
+           "config": {"workload": workload_desc(c), "step": f"all {c.M:,} sources x {n} sampled targets"},
+           "cpu_baseline": {"value": value, "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
+                            "sample": f"per step: all {c.M:,} sources x {n} seeded targets"},
+           "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+# ---------------------------------------------------------------- our arm
+def l2_flush(buf):
+    buf.add_(1.0)  # 256 MiB read+write > 126 MB L2
+
+
+def load_traffic(cfg):
+    """DRAM bytes per launch of the fused kernel from the committed ncu capture, if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        d = json.load(open(p))
+        e = d.get(f"cfg{cfg}", {})
+        return e.get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icppw_wangkbgj16_b200 as ks
+    from paper_conf_icppw_wangkbgj16_b200.dist import shard_bounds
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    c = workloads.CONFIGS[args.cfg]
+    a, W, b, h = workloads.make(c)
+    M, N, K, R = c.M, c.N, c.K, c.R
+    lo, hi = shard_bounds(N, world, rank)
+
+    plan = ks.KernelSum(K, float(h))
+    ta = torch.from_numpy(a).to(dev) if rank == 0 or world == 1 else torch.empty((M, K), device=dev)
+    tw = torch.from_numpy(W).to(dev) if rank == 0 or world == 1 else torch.empty((M, R), device=dev)
+    tb = torch.from_numpy(b[lo:hi].copy()).to(dev)
+    Vloc = torch.empty((max(hi - lo, 0), R), device=dev)
+    S = -(-N // world)
+    S = -(-S // 128) * 128
+    Vpad = torch.zeros((S, R), device=dev)
+    Vall = torch.empty((S * world, R), device=dev) if world > 1 else None
+    flush = None if args.no_flush else torch.empty(64 * 1024 * 1024, dtype=torch.float32, device=dev)
+    ks.ks_reserve(plan.ctx, max(hi - lo, 1))
+
+    def step():
+        if world > 1:
+            dist.broadcast(ta, src=0)
+            dist.broadcast(tw, src=0)
+        plan.set_sources(ta, tw)
+        if hi > lo:
+            plan.eval(tb, out=Vloc)
+        if world > 1:
+            Vpad[: hi - lo].copy_(Vloc)
+            dist.all_gather_into_tensor(Vall, Vpad)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    # ---- timed region
+    n_ev = args.steps
+    ev0 = [torch.cuda.Event(enable_timing=True) for _ in range(n_ev)]
+    ev1 = [torch.cuda.Event(enable_timing=True) for _ in range(n_ev)]
+    info0 = plan.info()
+    ks.ks_timing_read(plan.ctx, reset=True)
+    ks.ks_timing_enable(plan.ctx, True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for i in range(n_ev):
+            if flush is not None:
+                l2_flush(flush)
+            ev0[i].record()
+            step()
+            ev1[i].record()
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ks.ks_timing_enable(plan.ctx, False)
+    kern_ms, kern_n = ks.ks_timing_read(plan.ctx, reset=True)
+    info1 = plan.info()
+    ms_steps = [s.elapsed_time(e) for s, e in zip(ev0, ev1)]
+    ms_local = sum(ms_steps) / n_ev
+    t = torch.tensor([ms_local], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_per_step = float(t.item())
+    launches = int(info1["launches"] - info0["launches"])
+    if world > 1:
+        lt = torch.tensor([launches], dtype=torch.int64, device=dev)
+        dist.all_reduce(lt)
+        launches = int(lt.item())
+    pairs_per_step = M * N
+    value = pairs_per_step / (ms_per_step / 1e3)
+
+    # ---- roofline of the dominant (fused) kernel, from its own CUDA events
+    kms = kern_ms / max(kern_n, 1)
+    pairs_launch = M * (hi - lo)
+    fp32_ops, mufu = per_pair_ops(K, R)
+    achieved = pairs_launch * fp32_ops / (kms / 1e3) / 1e12      # T FP32-pipe lane-ops / s
+    sms = info1["num_sms"]
+    clk_sum = clk.summary()
+    max_mhz = clk_sum["sm_max_mhz"] or 1965
+    peak = 128 * sms * max_mhz * 1e6 / 1e12
+    roof = {"bound": "alu", "kernel": "ks_fused_fp32_kernel", "achieved": achieved, "peak": peak,
+            "unit": "Top/s FP32-pipe lane ops (K+2 per pair: K FFMA dot, 1 FADD norm, 1 FFMA weight)",
+            "frac": achieved / peak, "traffic": load_traffic(args.cfg),
+            "peak_derivation": f"128 FP32 lanes/clk/SM x {sms} SMs x {max_mhz} MHz (sm_max); MUFU ex2 "
+                               f"16/clk/SM is not binding at K={K}",
+            "kernel_ms": kms, "kernel_share_of_step": kms / ms_per_step if ms_per_step else None,
+            "pairs_per_launch": pairs_launch}
+    if clk_sum["sm_mhz"]:
+        roof["frac_at_measured_clock"] = achieved / (128 * sms * clk_sum["sm_mhz"] * 1e6 / 1e12)
+
+    # ---- e2e through the C-ABI host entry points (pinned buffers, copies timed)
+    ha = torch.from_numpy(a).pin_memory()
+    hw = torch.from_numpy(W).pin_memory()
+    hb = torch.from_numpy(b[lo:hi].copy()).pin_memory()
+    hv = torch.empty((max(hi - lo, 1), R), dtype=torch.float32).pin_memory()
+    an, wn, bn, vn = ha.numpy(), hw.numpy(), hb.numpy(), hv.numpy()
+    e2e_plan = ks.KernelSum(K, float(h))
+
+    def e2e_step():
+        if world > 1:
+            dist.broadcast(ta, src=0)
+            dist.broadcast(tw, src=0)
+        e2e_plan.set_sources_host(an, wn)
+        if hi > lo:
+            e2e_plan.eval_host(bn, out=vn[: hi - lo])
+
+    for _ in range(max(1, args.warmup)):
+        e2e_step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    e_ms = []
+    for _ in range(args.steps):
+        if flush is not None:
+            l2_flush(flush)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        e2e_step()
+        torch.cuda.synchronize()
+        e_ms.append(1e3 * (time.perf_counter() - t0))
+    t = torch.tensor([sum(e_ms) / len(e_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    e2e_ms = float(t.item())
+    e2e = {"value": pairs_per_step / (e2e_ms / 1e3), "unit": UNIT,
+           "h2d_bytes_per_step": int(4 * (M * K + M * R + (hi - lo) * K)),
+           "d2h_bytes_per_step": int(4 * (hi - lo) * R), "ms_per_step": e2e_ms,
+           "api": "ks_set_sources_host + ks_eval_host (pinned host buffers)"}
+    e2e_plan.close()
+
+    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+           "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+           "config": {"workload": workload_desc(c),
+                      "l2": "flushed before every step (256 MiB write, outside the step events)",
+                      "parallelism": f"target-sharded x{world}" + (" (NCCL broadcast alpha,W + all-gather V)"
+                                                                    if world > 1 else ""),
+                      "step": "ks_set_sources (a1) + ks_eval (a2-a7)" + (" + collectives" if world > 1 else ""),
+                      "path": info1["path"], "k_pad": info1["k_pad"], "ctas": info1["num_ctas"],
+                      "stages": info1["stages"]},
+           "roofline": roof, "e2e": e2e, "clocks": clk_sum, "gpu_launches": launches,
+           "gpu": torch.cuda.get_device_name(dev)}
+
+    # ---- CPU baseline (oracle) on rank 0 at N=1 only; also a parity spot-check of the timed V
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cb, J, Vr = cpu_baseline(a, W, b, h, args.cpu_seconds)
+        out["cpu_baseline"] = cb
+        Vg = Vloc.cpu().numpy().astype(np.float64)[J]
+        out["parity_sampled"] = {"e_norm": float(np.max(np.abs(Vg - Vr)) / np.abs(W).sum()),
+                                 "targets": int(len(J)), "bar": 1e-5}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    plan.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,162 @@
+/*
+ * ks.h -- C ABI of libks.so: fused Gaussian kernel summation on NVIDIA B200
+ * (sm_100a).
+ *
+ * The library evaluates, for sources alpha_i in R^K with weights W_i in R^R
+ * and targets beta_j in R^K,
+ *
+ *     V[j][r] = sum_{i<M} exp( -||alpha_i - beta_j||^2 / (2 h^2) ) * W[i][r]
+ *
+ * i.e. Eq.1 + Eq.2 of Wang et al., "Optimizing GPGPU Kernel Summation for
+ * Performance and Energy Efficiency", ICPP Workshops 2016 (PAPER.md P:L24-38,
+ * SS I), with the squared distance taken through the norm identity Eq.3
+ * and the -2 alpha^T beta contraction, the norm add, the exp and
+ * the weighted reduction fused in one kernel so the M x N kernel matrix never
+ * reaches memory (SS III-C, Alg.2).  Readings of the paper
+ * (which set carries W, the 2h^2 bandwidth, M != N, R columns) are listed
+ * in DESIGN.md SS3.
+ *
+ * Conventions (all entry points):
+ *   - extern "C", no C++ exceptions cross the boundary, no torch types.
+ *   - Arrays are FP32, row-major, one point's K coordinates contiguous
+ *     (A row-major / B column-major in the paper's GEMM view).
+ *   - Pointers taken by ks_set_sources / ks_eval are CUDA DEVICE pointers on
+ *     the context's device; the *_host variants take HOST pointers.
+ *   - Every call returns a ks_status.  On failure nothing is enqueued, the
+ *     context is unchanged, and ks_last_error() holds a thread-local detail
+ *     string.  There is no CPU fallback: without a usable sm_100 device,
+ *     ks_create fails with KS_ECUDA / KS_EUNSUPPORTED.
+ *   - Threading: a context is used by one host thread at a time.  Distinct
+ *     contexts are independent.
+ */
+#ifndef KS_H_
+#define KS_H_
+
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define KS_API __attribute__((visibility("default")))
+#else
+#define KS_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct ks_ctx ks_ctx;
+
+typedef enum {
+  KS_OK = 0,
+  KS_EINVAL = 1,        /* bad argument (size, NULL, h, K, R)                */
+  KS_ESTATE = 2,        /* ks_eval before ks_set_sources                     */
+  KS_ENOMEM = 3,        /* device allocation failed                          */
+  KS_ECUDA = 4,         /* CUDA runtime / launch error (see ks_last_error)   */
+  KS_EUNSUPPORTED = 5   /* no kernel for this (K, R, precision) or no sm_100 */
+} ks_status;
+
+typedef enum {
+  KS_PREC_AUTO = 0,     /* FP32 path if K <= 32 and R == 1, else 3XTF32      */
+  KS_PREC_FP32 = 1,     /* FP32 FFMA contraction (K <= 32, R == 1)           */
+  KS_PREC_3XTF32 = 2,   /* tcgen05 tensor cores, hi/lo split (3 products)    */
+  KS_PREC_TF32 = 3      /* tcgen05 tensor cores, single TF32 product         */
+} ks_precision;
+
+typedef enum { KS_PATH_NONE = 0, KS_PATH_FP32 = 1, KS_PATH_TC = 2 } ks_path;
+
+/* Launch/plan description of the last configured path (for reports). */
+typedef struct {
+  int path;             /* ks_path chosen for the current sources            */
+  int precision;        /* effective ks_precision (never AUTO)               */
+  int k_pad;            /* K padded to the kernel's dimension granularity    */
+  int tile_t;           /* targets per CTA tile                              */
+  int tile_s;           /* sources per pipeline stage                        */
+  int num_ctas;         /* persistent CTAs of the last ks_eval launch        */
+  int stages;           /* TMA pipeline depth                                */
+  int num_sms;          /* SMs of the device                                 */
+  int64_t m;            /* sources currently set                             */
+  int64_t m_pad;        /* padded source count                               */
+  int r;                /* weight columns                                    */
+  int64_t launches;     /* cumulative kernels launched by this context       */
+  int64_t fused_launches; /* cumulative launches of the fused kernel         */
+  double c_log2;        /* c = log2(e) / (2 h^2), the ex2 prescale           */
+} ks_info;
+
+/* Create a context for dimension K (1 <= K <= 4096) and bandwidth h (finite,
+ * > 0, with log2(e)/(2h^2) finite in FP32), bound to the current CUDA device.
+ * The default stream is the legacy default stream (0).
+ * Errors: KS_EINVAL (K, h, out == NULL), KS_ECUDA / KS_EUNSUPPORTED (no
+ * device, or device is not compute capability 10.0), KS_ENOMEM. */
+KS_API ks_status ks_create(int K, float h, ks_ctx **out);
+
+/* Destroy a context and free every library-owned buffer.  Synchronises the
+ * context's stream first.  NULL is a no-op returning KS_OK. */
+KS_API ks_status ks_destroy(ks_ctx *ctx);
+
+/* Select the arithmetic (default KS_PREC_AUTO).  Takes effect at the next
+ * ks_set_sources.  KS_EINVAL for an unknown value. */
+KS_API ks_status ks_set_precision(ks_ctx *ctx, ks_precision p);
+
+/* Set the CUDA stream (a cudaStream_t, passed as void*) every later call is
+ * ordered on.  NULL means the legacy default stream. */
+KS_API ks_status ks_set_stream(ks_ctx *ctx, void *cuda_stream);
+
+/* Source preparation (Alg.1 l.3 vec_alpha; Eq.3):
+ * copies alpha [M][K] and W [M][R] (DEVICE pointers, FP32, row-major) into
+ * library-owned buffers: centred on the source mean, squared norms with FP64
+ * accumulation, prescaled / split for the selected path, padded.
+ * Stream-ordered: the caller keeps alpha and W alive and unmodified until the
+ * stream passes this call.  Replaces any previous sources.
+ * Errors: KS_EINVAL (M < 0, R < 1, R > 256, NULL with M > 0),
+ * KS_EUNSUPPORTED (explicit FP32 precision with K > 32 or R > 1),
+ * KS_ENOMEM, KS_ECUDA.  M == 0 is valid (every V becomes 0). */
+KS_API ks_status ks_set_sources(ks_ctx *ctx, const float *alpha, const float *W,
+                         int64_t M, int R);
+
+/* Evaluate V [N][R] (DEVICE pointer, FP32, row-major) for targets beta [N][K]
+ * (DEVICE pointer): one fused kernel launch (Alg.2) plus, when
+ * the persistent schedule splits a target tile, an in-kernel deterministic
+ * fix-up (no separate launch, no atomics on V).  Asynchronous on the
+ * context's stream; V is OVERWRITTEN (not accumulated).  beta and V must not
+ * overlap.  N == 0 is a no-op.  Library scratch grows on demand (a
+ * synchronising allocation the first time a larger N is seen).
+ * Errors: KS_ESTATE (no sources), KS_EINVAL (N < 0, NULL with N > 0),
+ * KS_ENOMEM, KS_ECUDA. */
+KS_API ks_status ks_eval(ks_ctx *ctx, const float *beta, int64_t N, float *V);
+
+/* Same as ks_set_sources / ks_eval but alpha, W, beta, V are HOST pointers.
+ * The library stages them through its own device buffers (host->device copy,
+ * compute, device->host copy) and returns after V is in host memory.
+ * Pinned host memory gives the fastest copies; pageable memory works. */
+KS_API ks_status ks_set_sources_host(ks_ctx *ctx, const float *alpha, const float *W,
+                              int64_t M, int R);
+KS_API ks_status ks_eval_host(ks_ctx *ctx, const float *beta, int64_t N, float *V);
+
+/* Pre-size the scratch for targets up to N_max so later ks_eval calls never
+ * allocate (useful before CUDA-graph capture).  KS_EINVAL if N_max < 0. */
+KS_API ks_status ks_reserve(ks_ctx *ctx, int64_t N_max);
+
+/* Report the configured path (see ks_info).  KS_EINVAL on NULL. */
+KS_API ks_status ks_get_info(const ks_ctx *ctx, ks_info *out);
+
+/* Kernel timing for the roofline report: when enabled, every fused-kernel
+ * launch is bracketed by CUDA events on the launching stream.
+ * ks_timing_read synchronises the stream and returns the summed device time
+ * (ms) and number of timed launches since the last reset. */
+KS_API ks_status ks_timing_enable(ks_ctx *ctx, int on);
+KS_API ks_status ks_timing_read(ks_ctx *ctx, double *total_ms, int64_t *launches, int reset);
+
+/* Human-readable status name; never NULL. */
+KS_API const char *ks_status_str(ks_status s);
+
+/* Thread-local detail of the last failing call on this thread ("" if none). */
+KS_API const char *ks_last_error(void);
+
+/* Library version string. */
+KS_API const char *ks_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* KS_H_ */

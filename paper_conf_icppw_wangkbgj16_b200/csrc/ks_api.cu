@@ -1,0 +1,490 @@
+// ks_api.cu -- the C ABI of libks.so (include/ks.h): context, validation,
+// library-owned buffers, path dispatch, stream-K launch configuration.
+//
+// Boundary passages: Eq.2 defines the inputs (sources
+// alpha_i, weights W_i, targets beta_j, bandwidth h) and the output V; Alg.1
+// lists A (M x K), B (K x N), W and V; A row-major / B
+// column-major means one point's K coordinates are contiguous, which
+// is the [points][K] layout taken here.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cfloat>
+#include <cstdarg>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/ks.h"
+#include "ks_internal.h"
+
+namespace {
+
+thread_local std::string g_err;
+
+ks_status fail(ks_status s, const char* fmt, ...) __attribute__((format(printf, 2, 3)));
+ks_status fail(ks_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return s;
+}
+
+ks_status cuda_fail(cudaError_t e, const char* what) {
+  return fail(e == cudaErrorMemoryAllocation ? KS_ENOMEM : KS_ECUDA, "%s: %s (%s)", what, cudaGetErrorName(e),
+              cudaGetErrorString(e));
+}
+
+#define KS_CUDA(call, what)                      \
+  do {                                           \
+    cudaError_t e_ = (call);                     \
+    if (e_ != cudaSuccess) return cuda_fail(e_, what); \
+  } while (0)
+
+typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                    const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+PFN_encodeTiled get_encode() {
+  static PFN_encodeTiled fn = nullptr;
+  if (!fn) {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_encodeTiled>(p);
+  }
+  return fn;
+}
+
+int64_t round_up(int64_t x, int64_t m) { return (x + m - 1) / m * m; }
+
+// Device buffer that grows on demand.  Growth synchronises the stream first
+// (the old buffer may still be read by queued kernels).
+template <typename T>
+struct DBuf {
+  T* p = nullptr;
+  size_t cap = 0;  // elements
+  cudaError_t reserve(size_t n, cudaStream_t st, bool zero) {
+    if (n <= cap) return cudaSuccess;
+    cudaError_t e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return e;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    e = cudaMalloc(&p, n * sizeof(T));
+    if (e != cudaSuccess) {
+      p = nullptr;
+      return e;
+    }
+    cap = n;
+    if (zero) {
+      e = cudaMemsetAsync(p, 0, n * sizeof(T), st);
+      if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+  }
+};
+
+}  // namespace
+
+struct ks_ctx {
+  int device = 0;
+  int num_sms = 0;
+  int K = 0;
+  float h = 0.f;
+  double c = 0.0;  // log2(e) / (2 h^2)
+  ks_precision prec_req = KS_PREC_AUTO;
+  cudaStream_t stream = nullptr;
+
+  // current sources
+  bool have_src = false;
+  int path = KS_PATH_NONE;
+  int prec_eff = KS_PREC_AUTO;
+  int k_pad = 0;
+  int64_t M = 0, m_pad = 0;
+  int R = 1;
+  DBuf<float> src;        // FP32 path: [k_pad + 2][m_pad]
+  DBuf<float> mu;         // [k_pad]
+  DBuf<double> mean_part; // [nparts][K]
+  CUtensorMap tmap_src;
+
+  // eval scratch
+  DBuf<float> partial;
+  DBuf<int> counters;
+  DBuf<unsigned long long> dbg_times;
+  int last_grid = 0;
+
+  // host staging (ks_*_host)
+  DBuf<float> h_alpha, h_W, h_beta, h_V;
+
+  // accounting / timing
+  int64_t launches = 0, fused_launches = 0;
+  bool timing = false;
+  std::vector<cudaEvent_t> ev;  // pairs (start, stop)
+  size_t ev_used = 0;           // pairs in use
+};
+
+namespace {
+
+ks_status check_ctx(const ks_ctx* ctx) {
+  if (!ctx) return fail(KS_EINVAL, "ctx is NULL");
+  return KS_OK;
+}
+
+ks_status set_device(const ks_ctx* ctx) {
+  int cur = -1;
+  KS_CUDA(cudaGetDevice(&cur), "cudaGetDevice");
+  if (cur != ctx->device) KS_CUDA(cudaSetDevice(ctx->device), "cudaSetDevice");
+  return KS_OK;
+}
+
+int fp32_k_pad(int K) { return K <= 4 ? 4 : K <= 8 ? 8 : K <= 16 ? 16 : 32; }
+
+ks_status timed_begin(ks_ctx* ctx, cudaEvent_t* stop_out) {
+  *stop_out = nullptr;
+  if (!ctx->timing) return KS_OK;
+  if (2 * ctx->ev_used + 2 > ctx->ev.size()) {
+    cudaEvent_t a, b;
+    KS_CUDA(cudaEventCreate(&a), "cudaEventCreate");
+    KS_CUDA(cudaEventCreate(&b), "cudaEventCreate");
+    ctx->ev.push_back(a);
+    ctx->ev.push_back(b);
+  }
+  cudaEvent_t start = ctx->ev[2 * ctx->ev_used];
+  *stop_out = ctx->ev[2 * ctx->ev_used + 1];
+  KS_CUDA(cudaEventRecord(start, ctx->stream), "cudaEventRecord");
+  return KS_OK;
+}
+
+ks_status timed_end(ks_ctx* ctx, cudaEvent_t stop) {
+  if (!stop) return KS_OK;
+  KS_CUDA(cudaEventRecord(stop, ctx->stream), "cudaEventRecord");
+  ctx->ev_used++;
+  return KS_OK;
+}
+
+ks_status prepare_fp32(ks_ctx* ctx, const float* alpha, const float* W, int64_t M) {
+  const int K = ctx->K;
+  const int k_pad = fp32_k_pad(K);
+  const int64_t m_pad = round_up(M > 0 ? M : 1, ks::kTileS);
+  cudaStream_t st = ctx->stream;
+  const size_t need = (size_t)(k_pad + 2) * (size_t)m_pad;
+  KS_CUDA(ctx->src.reserve(need, st, false), "allocate source buffer");
+  KS_CUDA(ctx->mu.reserve(k_pad, st, false), "allocate mean buffer");
+  int nparts = (int)((M + 511) / 512);
+  if (nparts < 1) nparts = 1;
+  if (nparts > 1024) nparts = 1024;
+  KS_CUDA(ctx->mean_part.reserve((size_t)nparts * K, st, false), "allocate mean partials");
+  KS_CUDA(ks::launch_source_mean(alpha, M, K, k_pad, ctx->mean_part.p, nparts, ctx->mu.p, st), "source mean");
+  ctx->launches += (M > 0) ? 2 : 1;
+  KS_CUDA(ks::launch_prep_fp32(alpha, W, M, m_pad, K, k_pad, ctx->mu.p, ctx->c, ctx->src.p, st), "source prep");
+  ctx->launches += 1;
+
+  PFN_encodeTiled enc = get_encode();
+  if (!enc) return fail(KS_ECUDA, "cuTensorMapEncodeTiled unavailable from the driver");
+  cuuint64_t dims[2] = {(cuuint64_t)m_pad, (cuuint64_t)(k_pad + 2)};
+  cuuint64_t strides[1] = {(cuuint64_t)m_pad * sizeof(float)};
+  cuuint32_t box[2] = {(cuuint32_t)ks::kTileS, (cuuint32_t)(k_pad + 2)};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(&ctx->tmap_src, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, ctx->src.p, dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(KS_ECUDA, "cuTensorMapEncodeTiled failed (CUresult %d)", (int)r);
+
+  ctx->k_pad = k_pad;
+  ctx->m_pad = m_pad;
+  return KS_OK;
+}
+
+ks_status eval_fp32(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
+  cudaStream_t st = ctx->stream;
+  ks::StreamK sk;
+  sk.n_t = (N + ks::kTileT - 1) / ks::kTileT;
+  sk.n_s = (int32_t)(ctx->m_pad / ks::kTileS);
+  sk.units = sk.n_t * (int64_t)sk.n_s;
+  int64_t g = (int64_t)ctx->num_sms * ks::fused_fp32_ctas_per_sm(ctx->k_pad);
+  if (g > sk.units) g = sk.units;  // every CTA owns >= 1 unit (fix-up relies on it)
+  sk.grid = (int32_t)g;
+  KS_CUDA(ctx->partial.reserve((size_t)sk.grid * 2 * ks::kTileT, st, false), "allocate partials");
+  KS_CUDA(ctx->counters.reserve((size_t)sk.n_t, st, true), "allocate tile counters");
+
+  ks::Fp32Args a;
+  a.beta = beta;
+  a.N = N;
+  a.K = ctx->K;
+  a.mu = ctx->mu.p;
+  a.c = ctx->c;
+  a.V = V;
+  a.partial = ctx->partial.p;
+  a.counters = ctx->counters.p;
+  a.sk = sk;
+  a.cta_times = nullptr;
+  // debug knob: KS_CTA_TIMES=<file> appends per-CTA start/end globaltimer (ns) of each launch
+  const char* dbg = getenv("KS_CTA_TIMES");
+  if (dbg && *dbg) {
+    KS_CUDA(ctx->dbg_times.reserve((size_t)sk.grid * 2, st, true), "allocate debug timers");
+    a.cta_times = ctx->dbg_times.p;
+  }
+  cudaEvent_t stop;
+  ks_status s = timed_begin(ctx, &stop);
+  if (s != KS_OK) return s;
+  KS_CUDA(ks::launch_fused_fp32(&ctx->tmap_src, ctx->k_pad, a, st), "fused FP32 kernel launch");
+  ctx->launches++;
+  ctx->fused_launches++;
+  ctx->last_grid = sk.grid;
+  ks_status ts = timed_end(ctx, stop);
+  if (a.cta_times) {
+    std::vector<unsigned long long> h((size_t)sk.grid * 2);
+    KS_CUDA(cudaMemcpyAsync(h.data(), a.cta_times, h.size() * 8, cudaMemcpyDeviceToHost, st), "copy debug timers");
+    KS_CUDA(cudaStreamSynchronize(st), "synchronize");
+    FILE* f = fopen(dbg, "a");
+    if (f) {
+      for (int i = 0; i < sk.grid; ++i) fprintf(f, "%d %llu %llu\n", i, h[2 * i], h[2 * i + 1]);
+      fprintf(f, "--\n");
+      fclose(f);
+    }
+  }
+  return ts;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* ks_version(void) { return "ks-b200 0.1 (sm_100a)"; }
+
+const char* ks_status_str(ks_status s) {
+  switch (s) {
+    case KS_OK: return "KS_OK";
+    case KS_EINVAL: return "KS_EINVAL";
+    case KS_ESTATE: return "KS_ESTATE";
+    case KS_ENOMEM: return "KS_ENOMEM";
+    case KS_ECUDA: return "KS_ECUDA";
+    case KS_EUNSUPPORTED: return "KS_EUNSUPPORTED";
+  }
+  return "KS_UNKNOWN";
+}
+
+const char* ks_last_error(void) { return g_err.c_str(); }
+
+ks_status ks_create(int K, float h, ks_ctx** out) {
+  if (!out) return fail(KS_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (K < 1 || K > 4096) return fail(KS_EINVAL, "K=%d outside [1, 4096]", K);
+  if (!std::isfinite(h) || !(h > 0.f)) return fail(KS_EINVAL, "h=%g must be finite and > 0", (double)h);
+  const double hd = (double)h;
+  const double c = 1.4426950408889634 / (2.0 * hd * hd);
+  if (!(c * 2.0 <= (double)FLT_MAX) || !(c >= (double)FLT_MIN))
+    return fail(KS_EINVAL, "h=%g gives c=log2(e)/(2h^2)=%g outside FP32 range", (double)h, c);
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice (no CUDA device?)");
+  cudaDeviceProp prop;
+  e = cudaGetDeviceProperties(&prop, dev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceProperties");
+  if (!(prop.major == 10 && prop.minor == 0))
+    return fail(KS_EUNSUPPORTED, "device %d is sm_%d%d; libks.so is built for sm_100a (B200) only", dev, prop.major,
+                prop.minor);
+  ks_ctx* ctx = new (std::nothrow) ks_ctx();
+  if (!ctx) return fail(KS_ENOMEM, "host allocation of the context failed");
+  ctx->device = dev;
+  ctx->num_sms = prop.multiProcessorCount;
+  ctx->K = K;
+  ctx->h = h;
+  ctx->c = c;
+  *out = ctx;
+  g_err.clear();
+  return KS_OK;
+}
+
+ks_status ks_destroy(ks_ctx* ctx) {
+  if (!ctx) return KS_OK;
+  set_device(ctx);
+  cudaStreamSynchronize(ctx->stream);
+  ctx->src.release();
+  ctx->mu.release();
+  ctx->mean_part.release();
+  ctx->partial.release();
+  ctx->counters.release();
+  ctx->dbg_times.release();
+  ctx->h_alpha.release();
+  ctx->h_W.release();
+  ctx->h_beta.release();
+  ctx->h_V.release();
+  for (cudaEvent_t ev : ctx->ev) cudaEventDestroy(ev);
+  delete ctx;
+  return KS_OK;
+}
+
+ks_status ks_set_precision(ks_ctx* ctx, ks_precision p) {
+  if (check_ctx(ctx)) return KS_EINVAL;
+  if (p != KS_PREC_AUTO && p != KS_PREC_FP32 && p != KS_PREC_3XTF32 && p != KS_PREC_TF32)
+    return fail(KS_EINVAL, "unknown precision %d", (int)p);
+  ctx->prec_req = p;
+  return KS_OK;
+}
+
+ks_status ks_set_stream(ks_ctx* ctx, void* cuda_stream) {
+  if (check_ctx(ctx)) return KS_EINVAL;
+  ctx->stream = reinterpret_cast<cudaStream_t>(cuda_stream);
+  return KS_OK;
+}
+
+ks_status ks_set_sources(ks_ctx* ctx, const float* alpha, const float* W, int64_t M, int R) {
+  if (check_ctx(ctx)) return KS_EINVAL;
+  if (M < 0) return fail(KS_EINVAL, "M=%lld < 0", (long long)M);
+  if (R < 1 || R > 256) return fail(KS_EINVAL, "R=%d outside [1, 256]", R);
+  if (M > 0 && (!alpha || !W)) return fail(KS_EINVAL, "alpha/W is NULL with M=%lld", (long long)M);
+  if (M > ((int64_t)1 << 31) - 256) return fail(KS_EINVAL, "M=%lld too large", (long long)M);
+  int prec = ctx->prec_req;
+  int path;
+  if (prec == KS_PREC_AUTO) {
+    path = (ctx->K <= 32 && R == 1) ? KS_PATH_FP32 : KS_PATH_TC;
+    prec = (path == KS_PATH_FP32) ? KS_PREC_FP32 : KS_PREC_3XTF32;
+  } else if (prec == KS_PREC_FP32) {
+    if (ctx->K > 32 || R != 1)
+      return fail(KS_EUNSUPPORTED, "FP32 path needs K <= 32 and R == 1 (K=%d, R=%d)", ctx->K, R);
+    path = KS_PATH_FP32;
+  } else {
+    path = KS_PATH_TC;
+  }
+  if (path == KS_PATH_TC)
+    return fail(KS_EUNSUPPORTED, "tensor-core path (K=%d, R=%d, precision %d) not built yet", ctx->K, R, prec);
+  ks_status s = set_device(ctx);
+  if (s != KS_OK) return s;
+  ctx->have_src = false;
+  s = prepare_fp32(ctx, alpha, W, M);
+  if (s != KS_OK) return s;
+  ctx->path = path;
+  ctx->prec_eff = prec;
+  ctx->M = M;
+  ctx->R = R;
+  ctx->have_src = true;
+  return KS_OK;
+}
+
+ks_status ks_eval(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
+  if (check_ctx(ctx)) return KS_EINVAL;
+  if (N < 0) return fail(KS_EINVAL, "N=%lld < 0", (long long)N);
+  if (!ctx->have_src) return fail(KS_ESTATE, "ks_eval before ks_set_sources");
+  if (N == 0) return KS_OK;
+  if (!beta || !V) return fail(KS_EINVAL, "beta/V is NULL with N=%lld", (long long)N);
+  if (N > ((int64_t)1 << 31) - 256) return fail(KS_EINVAL, "N=%lld too large", (long long)N);
+  ks_status s = set_device(ctx);
+  if (s != KS_OK) return s;
+  if (ctx->M == 0) {
+    KS_CUDA(cudaMemsetAsync(V, 0, (size_t)N * ctx->R * sizeof(float), ctx->stream), "zero V");
+    return KS_OK;
+  }
+  return eval_fp32(ctx, beta, N, V);
+}
+
+ks_status ks_reserve(ks_ctx* ctx, int64_t N_max) {
+  if (check_ctx(ctx)) return KS_EINVAL;
+  if (N_max < 0) return fail(KS_EINVAL, "N_max < 0");
+  ks_status s = set_device(ctx);
+  if (s != KS_OK) return s;
+  const int64_t n_t = (N_max + ks::kTileT - 1) / ks::kTileT;
+  const int64_t g = (int64_t)ctx->num_sms * 8;  // >= any persistent grid
+  KS_CUDA(ctx->partial.reserve((size_t)g * 2 * ks::kTileT, ctx->stream, false), "allocate partials");
+  KS_CUDA(ctx->counters.reserve((size_t)(n_t > 0 ? n_t : 1), ctx->stream, true), "allocate tile counters");
+  return KS_OK;
+}
+
+ks_status ks_set_sources_host(ks_ctx* ctx, const float* alpha, const float* W, int64_t M, int R) {
+  if (check_ctx(ctx)) return KS_EINVAL;
+  if (M < 0) return fail(KS_EINVAL, "M=%lld < 0", (long long)M);
+  if (R < 1 || R > 256) return fail(KS_EINVAL, "R=%d outside [1, 256]", R);
+  if (M > 0 && (!alpha || !W)) return fail(KS_EINVAL, "alpha/W is NULL with M=%lld", (long long)M);
+  ks_status s = set_device(ctx);
+  if (s != KS_OK) return s;
+  const size_t na = (size_t)M * ctx->K, nw = (size_t)M * R;
+  KS_CUDA(ctx->h_alpha.reserve(na ? na : 1, ctx->stream, false), "allocate alpha staging");
+  KS_CUDA(ctx->h_W.reserve(nw ? nw : 1, ctx->stream, false), "allocate W staging");
+  if (M > 0) {
+    KS_CUDA(cudaMemcpyAsync(ctx->h_alpha.p, alpha, na * 4, cudaMemcpyHostToDevice, ctx->stream), "copy alpha H2D");
+    KS_CUDA(cudaMemcpyAsync(ctx->h_W.p, W, nw * 4, cudaMemcpyHostToDevice, ctx->stream), "copy W H2D");
+  }
+  s = ks_set_sources(ctx, ctx->h_alpha.p, ctx->h_W.p, M, R);
+  if (s != KS_OK) return s;
+  KS_CUDA(cudaStreamSynchronize(ctx->stream), "synchronize");
+  return KS_OK;
+}
+
+ks_status ks_eval_host(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
+  if (check_ctx(ctx)) return KS_EINVAL;
+  if (N < 0) return fail(KS_EINVAL, "N=%lld < 0", (long long)N);
+  if (!ctx->have_src) return fail(KS_ESTATE, "ks_eval before ks_set_sources");
+  if (N == 0) return KS_OK;
+  if (!beta || !V) return fail(KS_EINVAL, "beta/V is NULL with N=%lld", (long long)N);
+  ks_status s = set_device(ctx);
+  if (s != KS_OK) return s;
+  const size_t nb = (size_t)N * ctx->K, nv = (size_t)N * ctx->R;
+  KS_CUDA(ctx->h_beta.reserve(nb, ctx->stream, false), "allocate beta staging");
+  KS_CUDA(ctx->h_V.reserve(nv, ctx->stream, false), "allocate V staging");
+  KS_CUDA(cudaMemcpyAsync(ctx->h_beta.p, beta, nb * 4, cudaMemcpyHostToDevice, ctx->stream), "copy beta H2D");
+  s = ks_eval(ctx, ctx->h_beta.p, N, ctx->h_V.p);
+  if (s != KS_OK) return s;
+  KS_CUDA(cudaMemcpyAsync(V, ctx->h_V.p, nv * 4, cudaMemcpyDeviceToHost, ctx->stream), "copy V D2H");
+  KS_CUDA(cudaStreamSynchronize(ctx->stream), "synchronize");
+  return KS_OK;
+}
+
+ks_status ks_get_info(const ks_ctx* ctx, ks_info* out) {
+  if (!ctx || !out) return fail(KS_EINVAL, "ctx/out is NULL");
+  memset(out, 0, sizeof *out);
+  out->path = ctx->have_src ? ctx->path : KS_PATH_NONE;
+  out->precision = ctx->have_src ? ctx->prec_eff : ctx->prec_req;
+  out->k_pad = ctx->k_pad;
+  out->tile_t = ks::kTileT;
+  out->tile_s = ks::kTileS;
+  out->num_ctas = ctx->last_grid;
+  out->stages = ctx->k_pad ? ks::fused_fp32_stages(ctx->k_pad) : 0;
+  out->num_sms = ctx->num_sms;
+  out->m = ctx->M;
+  out->m_pad = ctx->m_pad;
+  out->r = ctx->R;
+  out->launches = ctx->launches;
+  out->fused_launches = ctx->fused_launches;
+  out->c_log2 = ctx->c;
+  return KS_OK;
+}
+
+ks_status ks_timing_enable(ks_ctx* ctx, int on) {
+  if (check_ctx(ctx)) return KS_EINVAL;
+  ctx->timing = on != 0;
+  return KS_OK;
+}
+
+ks_status ks_timing_read(ks_ctx* ctx, double* total_ms, int64_t* launches, int reset) {
+  if (check_ctx(ctx)) return KS_EINVAL;
+  if (!total_ms || !launches) return fail(KS_EINVAL, "total_ms/launches is NULL");
+  ks_status s = set_device(ctx);
+  if (s != KS_OK) return s;
+  KS_CUDA(cudaStreamSynchronize(ctx->stream), "synchronize");
+  double tot = 0.0;
+  for (size_t i = 0; i < ctx->ev_used; ++i) {
+    float ms = 0.f;
+    KS_CUDA(cudaEventElapsedTime(&ms, ctx->ev[2 * i], ctx->ev[2 * i + 1]), "cudaEventElapsedTime");
+    tot += ms;
+  }
+  *total_ms = tot;
+  *launches = (int64_t)ctx->ev_used;
+  if (reset) ctx->ev_used = 0;
+  return KS_OK;
+}
+
+}  // extern "C"

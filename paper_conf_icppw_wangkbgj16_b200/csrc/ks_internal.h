@@ -1,0 +1,55 @@
+// ks_internal.h -- host-side declarations shared by the C-ABI layer and the
+// kernel translation units (not part of the public ABI).
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cstdint>
+
+namespace ks {
+
+constexpr int kTileT = 256;   // targets per CTA tile (FP32 path)
+constexpr int kTileS = 128;   // sources per pipeline stage (FP32 path)
+constexpr int kFp32Threads = 512;  // 16 warps, one CTA per SM
+
+// Stream-K partition of the (target tile x source tile) unit space over G
+// persistent CTAs: CTA b owns units [b*U/G, (b+1)*U/G).
+struct StreamK {
+  int64_t units;       // U = n_t * n_s
+  int64_t n_t;         // target tiles
+  int32_t n_s;         // source tiles
+  int32_t grid;        // G
+};
+
+// ---------------------------------------------------------------- prep (a1)
+// mu[d] (FP32, d < k_pad; zero for d >= K) = mean_i alpha[i][d], FP64 accumulation, fixed order.
+cudaError_t launch_source_mean(const float* alpha, int64_t M, int K, int k_pad, double* part, int nparts,
+                               float* mu, cudaStream_t st);
+
+// FP32 path source layout, dimension-major [k_pad + 2][m_pad]:
+//   rows d < k_pad : a[d][i]  = RN(2c * (alpha[i][d] - mu[d]))
+//   row k_pad      : na[i]    = RN(-c * ||alpha_i - mu||^2)   (FP64 accumulation)
+//   row k_pad + 1  : W[i]     (0 for padding)
+cudaError_t launch_prep_fp32(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
+                             const float* mu, double c, float* src, cudaStream_t st);
+
+// ---------------------------------------------------------------- FP32 fused kernel (a2-a7)
+struct Fp32Args {
+  const float* beta;   // [N][K] raw targets
+  int64_t N;
+  int K;
+  const float* mu;     // [k_pad]
+  double c;            // log2(e) / (2 h^2)
+  float* V;            // [N]
+  float* partial;      // [grid][2][kTileT]
+  int* counters;       // [n_t], zero on entry, left zero on exit
+  StreamK sk;
+  unsigned long long* cta_times;  // debug: [grid][2] globaltimer at CTA start / end, or nullptr
+};
+
+// Returns the number of stages used; launches one kernel.
+cudaError_t launch_fused_fp32(const CUtensorMap* tmap_src, int k_pad, const Fp32Args& a, cudaStream_t st);
+int fused_fp32_ctas_per_sm(int k_pad);
+int fused_fp32_stages(int k_pad);
+
+}  // namespace ks
