@@ -38,6 +38,8 @@
 #include "ks_internal.h"
 #include "ks_ptx.cuh"
 
+#include <cstdlib>
+
 
 namespace ks {
 
@@ -153,7 +155,52 @@ __device__ __forceinline__ void init_half(const float* __restrict__ sp, const fl
     for (int p = 0; p < 4; ++p) acc[j][p] = fadd2(f2_bcast(nbv[j]), na[p]);
 }
 
+// Full 8x8 micro-tile in one k loop (4 LDS.128 per 32 FFMA2: half the
+// shared-memory traffic per FMA of the split form) with the epilogue at the
+// end of the tile.
 template <int KP>
+__device__ __forceinline__ void full_tile(const float* __restrict__ sp, const float* __restrict__ tgt,
+                                          const float* __restrict__ nbs, int tx, int ty, float (&bsA)[4],
+                                          float (&bsB)[4]) {
+  f2_t acc[8][4];
+  {
+    const ulonglong2 n01 = lds_pairs(sp + KP * kTileS + 4 * tx);
+    const ulonglong2 n23 = lds_pairs(sp + KP * kTileS + 64 + 4 * tx);
+    const float4 nbA = lds128(nbs + 4 * ty);
+    const float4 nbB = lds128(nbs + kTileT / 2 + 4 * ty);
+    const f2_t na[4] = {n01.x, n01.y, n23.x, n23.y};
+    const float nb[8] = {nbA.x, nbA.y, nbA.z, nbA.w, nbB.x, nbB.y, nbB.z, nbB.w};
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+#pragma unroll
+      for (int p = 0; p < 4; ++p) acc[j][p] = fadd2(f2_bcast(nb[j]), na[p]);
+  }
+#pragma unroll
+  for (int k = 0; k < KP; ++k) {
+    const ulonglong2 a01 = lds_pairs(sp + k * kTileS + 4 * tx);
+    const ulonglong2 a23 = lds_pairs(sp + k * kTileS + 64 + 4 * tx);
+    const float4 bA = lds128(tgt + k * kTileT + 4 * ty);
+    const float4 bB = lds128(tgt + k * kTileT + kTileT / 2 + 4 * ty);
+    const f2_t av[4] = {a01.x, a01.y, a23.x, a23.y};
+    const float bv[8] = {bA.x, bA.y, bA.z, bA.w, bB.x, bB.y, bB.z, bB.w};
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+#pragma unroll
+      for (int p = 0; p < 4; ++p) acc[j][p] = ffma2(f2_bcast(bv[j]), av[p], acc[j][p]);
+  }
+  const ulonglong2 w01 = lds_pairs(sp + (KP + 1) * kTileS + 4 * tx);
+  const ulonglong2 w23 = lds_pairs(sp + (KP + 1) * kTileS + 64 + 4 * tx);
+  const f2_t w2[4] = {w01.x, w01.y, w23.x, w23.y};
+#pragma unroll
+  for (int j = 0; j < 4; ++j)
+#pragma unroll
+    for (int p = 0; p < 4; ++p) {
+      epi_pair(acc[j][p], w2[p], bsA[j]);
+      epi_pair(acc[4 + j][p], w2[p], bsB[j]);
+    }
+}
+
+template <int KP, bool SPLIT>
 __global__ void __launch_bounds__(kFp32Threads, 1)
     ks_fused_fp32_kernel(const __grid_constant__ CUtensorMap tmap_src, const Fp32Args args) {
   using C = Fp32Cfg<KP>;
@@ -253,6 +300,9 @@ __global__ void __launch_bounds__(kFp32Threads, 1)
       mbar_wait(&full[s], ph);
       const float* sp = smem + s * C::kStageFloats;
 
+      if constexpr (!SPLIT) {
+        full_tile<KP>(sp, tgt, nbs, tx, ty, bsA, bsB);
+      } else {
       // targets A: contraction; epilogue of the previous tile's half B
       init_half<KP>(sp, nbs + 4 * ty, tx, accA);
       half_tile<KP>(sp, tgt + 4 * ty, tx, accA, accB, w2, bsB);
@@ -265,6 +315,7 @@ __global__ void __launch_bounds__(kFp32Threads, 1)
       __syncwarp();
       init_half<KP>(sp, nbs + kTileT / 2 + 4 * ty, tx, accB);
       half_tile<KP>(sp, tgt + kTileT / 2 + 4 * ty, tx, accB, accA, w2, bsA);
+      }
 
       // release the stage; the last warp to release it refills it (unit q + S)
       __syncwarp();
@@ -291,8 +342,10 @@ __global__ void __launch_bounds__(kFp32Threads, 1)
       }
     }
     // drain: epilogue of the last tile's half B
+    if constexpr (SPLIT) {
 #pragma unroll
-    for (int qq = 0; qq < 16; ++qq) epi_pair(accB[qq >> 2][qq & 3], w2[qq & 3], bsB[qq >> 2]);
+      for (int qq = 0; qq < 16; ++qq) epi_pair(accB[qq >> 2][qq & 3], w2[qq & 3], bsB[qq >> 2]);
+    }
     double vacc[8];
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
@@ -366,18 +419,37 @@ __global__ void __launch_bounds__(kFp32Threads, 1)
   }
 }
 
+// Tile-body variant.  Measured on B200 (SS7): at K = 32 the split
+// halves with the interleaved epilogue are faster (76% vs 74% of the FP32
+// roofline); at K <= 16 the full 8x8 tile (half the LDS per FMA) wins.
+// KS_FP32_SPLIT=0/1 overrides (measurement knob).
 template <int KP>
-static cudaError_t launch_kp(const CUtensorMap* tmap, const Fp32Args& a, cudaStream_t st) {
+static bool fp32_split() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("KS_FP32_SPLIT");
+    v = (e && (e[0] == '0' || e[0] == '1')) ? (e[0] - '0') : (KP >= 32 ? 1 : 0);
+  }
+  return v == 1;
+}
+
+template <int KP, bool SPLIT>
+static cudaError_t launch_kps(const CUtensorMap* tmap, const Fp32Args& a, cudaStream_t st) {
   using C = Fp32Cfg<KP>;
   static bool attr_done = false;
   if (!attr_done) {
-    cudaError_t e = cudaFuncSetAttribute(ks_fused_fp32_kernel<KP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)C::kSmemBytes);
+    cudaError_t e = cudaFuncSetAttribute(ks_fused_fp32_kernel<KP, SPLIT>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::kSmemBytes);
     if (e != cudaSuccess) return e;
     attr_done = true;
   }
-  ks_fused_fp32_kernel<KP><<<a.sk.grid, C::kThreads, C::kSmemBytes, st>>>(*tmap, a);
+  ks_fused_fp32_kernel<KP, SPLIT><<<a.sk.grid, C::kThreads, C::kSmemBytes, st>>>(*tmap, a);
   return cudaGetLastError();
+}
+
+template <int KP>
+static cudaError_t launch_kp(const CUtensorMap* tmap, const Fp32Args& a, cudaStream_t st) {
+  return fp32_split<KP>() ? launch_kps<KP, true>(tmap, a, st) : launch_kps<KP, false>(tmap, a, st);
 }
 
 cudaError_t launch_fused_fp32(const CUtensorMap* tmap_src, int k_pad, const Fp32Args& a, cudaStream_t st) {
@@ -394,9 +466,10 @@ template <int KP>
 static int ctas_per_sm_kp() {
   using C = Fp32Cfg<KP>;
   int n = 0;
-  cudaFuncSetAttribute(ks_fused_fp32_kernel<KP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::kSmemBytes);
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, ks_fused_fp32_kernel<KP>, C::kThreads, C::kSmemBytes) !=
-      cudaSuccess)
+  cudaFuncSetAttribute(ks_fused_fp32_kernel<KP, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       (int)C::kSmemBytes);
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, ks_fused_fp32_kernel<KP, false>, C::kThreads,
+                                                    C::kSmemBytes) != cudaSuccess)
     n = 1;
   return n < 1 ? 1 : n;
 }
