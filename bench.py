@@ -51,7 +51,7 @@ UNIT = "pairs/s"
 def parse():
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
-    p.add_argument("--steps", type=int, default=10)
+    p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--cfg", type=int, default=3, help="BASELINE config id (1-based, SURVEY SS8(a))")
     p.add_argument("--impl", choices=["ours", "reference"], default="ours")
@@ -83,7 +83,7 @@ class ClockSampler:
         0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
     }
 
-    def __init__(self, dev_index: int, period: float = 0.05):
+    def __init__(self, dev_index: int, period: float = 0.005):
         self.samples, self.reasons, self.ok = [], 0, False
         self.period = period
         self._stop = threading.Event()
@@ -136,7 +136,8 @@ def cpu_baseline(a, W, b, h, cpu_seconds, seed=20163):
     threads = len(os.sched_getaffinity(0))
     oracle.set_num_threads(threads)
     M, N = a.shape[0], b.shape[0]
-    J0 = workloads.sample_targets(N, 4 * threads, seed)
+    oracle.oracle_eval(a, W, b, float(h), J=workloads.sample_targets(N, threads, seed - 1))  # spin up threads
+    J0 = workloads.sample_targets(N, 8 * threads, seed)
     t0 = time.perf_counter()
     oracle.oracle_eval(a, W, b, float(h), J=J0)
     dt = max(time.perf_counter() - t0, 1e-4)
