@@ -10,6 +10,7 @@
 #include <cuda_runtime.h>
 
 #include <cfloat>
+#include <algorithm>
 #include <cstdarg>
 #include <cmath>
 #include <cstdio>
@@ -117,6 +118,11 @@ struct ks_ctx {
   int64_t M = 0, m_pad = 0;
   int R = 1;
   DBuf<float> src;        // FP32 path: [k_pad + 2][m_pad]
+  // TC path (tcgen05): TF32 hi/lo operand splits, norms, W^T splits
+  DBuf<float> src_hi, src_lo, na, wt_hi, wt_lo;
+  DBuf<float> tgt_hi, tgt_lo, nb;
+  int r_pad = 16;
+  CUtensorMap tmB_hi, tmB_lo;
   DBuf<float> mu;         // [k_pad]
   DBuf<double> mean_part; // [nparts][K]
   CUtensorMap tmap_src;
@@ -260,6 +266,153 @@ ks_status eval_fp32(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   return ts;
 }
 
+
+ks_status encode_2d_sw64(CUtensorMap* map, const float* base, int64_t inner, int64_t rows, int box_rows) {
+  PFN_encodeTiled enc = get_encode();
+  if (!enc) return fail(KS_ECUDA, "cuTensorMapEncodeTiled unavailable from the driver");
+  cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)inner * sizeof(float)};
+  cuuint32_t box[2] = {(cuuint32_t)ks::kTcKC, (cuuint32_t)box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(KS_ECUDA, "cuTensorMapEncodeTiled (2D SW64) failed (CUresult %d)", (int)r);
+  return KS_OK;
+}
+
+// W^T [r_pad][m_pad] viewed as {16 sources, r, m_pad/16 chunks}: one box =
+// 8 chunks x r_c rows x 16 floats = the K-major SWIZZLE_64B B operand of V-MMA.
+ks_status encode_wt(CUtensorMap* map, const float* base, int64_t m_pad, int r_pad, int r_c) {
+  PFN_encodeTiled enc = get_encode();
+  if (!enc) return fail(KS_ECUDA, "cuTensorMapEncodeTiled unavailable from the driver");
+  cuuint64_t dims[3] = {16, (cuuint64_t)r_pad, (cuuint64_t)(m_pad / 16)};
+  cuuint64_t strides[2] = {(cuuint64_t)m_pad * sizeof(float), 64};
+  cuuint32_t box[3] = {16, (cuuint32_t)r_c, (cuuint32_t)(ks::kTcTileS / 16)};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(base), dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(KS_ECUDA, "cuTensorMapEncodeTiled (W^T 3D) failed (CUresult %d)", (int)r);
+  return KS_OK;
+}
+
+int tc_k_pad(int K) { return (int)round_up(K, ks::kTcKC); }
+
+ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M, int R) {
+  const int K = ctx->K;
+  const int k_pad = tc_k_pad(K);
+  const int64_t m_pad = round_up(M > 0 ? M : 1, ks::kTcTileS);
+  const int r_pad = (int)round_up(R, 16);
+  cudaStream_t st = ctx->stream;
+  const size_t nsrc = (size_t)m_pad * k_pad, nw = (size_t)r_pad * m_pad;
+  KS_CUDA(ctx->src_hi.reserve(nsrc, st, false), "allocate source hi");
+  KS_CUDA(ctx->src_lo.reserve(nsrc, st, false), "allocate source lo");
+  KS_CUDA(ctx->na.reserve((size_t)m_pad, st, false), "allocate source norms");
+  KS_CUDA(ctx->wt_hi.reserve(nw, st, false), "allocate W hi");
+  KS_CUDA(ctx->wt_lo.reserve(nw, st, false), "allocate W lo");
+  KS_CUDA(ctx->mu.reserve(k_pad, st, false), "allocate mean buffer");
+  int nparts = (int)((M + 511) / 512);
+  if (nparts < 1) nparts = 1;
+  if (nparts > 1024) nparts = 1024;
+  KS_CUDA(ctx->mean_part.reserve((size_t)nparts * K, st, false), "allocate mean partials");
+  KS_CUDA(ks::launch_source_mean(alpha, M, K, k_pad, ctx->mean_part.p, nparts, ctx->mu.p, st), "source mean");
+  ctx->launches += (M > 0) ? 2 : 1;
+  KS_CUDA(ks::launch_prep_tc_sources(alpha, W, M, m_pad, K, k_pad, R, r_pad, ctx->mu.p, ctx->c, ctx->src_hi.p,
+                                     ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p, st),
+          "source prep (TC)");
+  ctx->launches += 1;
+  ks_status s = encode_2d_sw64(&ctx->tmB_hi, ctx->src_hi.p, k_pad, m_pad, ks::kTcTileS);
+  if (s != KS_OK) return s;
+  s = encode_2d_sw64(&ctx->tmB_lo, ctx->src_lo.p, k_pad, m_pad, ks::kTcTileS);
+  if (s != KS_OK) return s;
+  ctx->k_pad = k_pad;
+  ctx->m_pad = m_pad;
+  ctx->r_pad = r_pad;
+  return KS_OK;
+}
+
+ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
+  cudaStream_t st = ctx->stream;
+  const int k_pad = ctx->k_pad;
+  const int64_t n_pad = round_up(N, ks::kTcTileT);
+  const size_t ntg = (size_t)n_pad * k_pad;
+  KS_CUDA(ctx->tgt_hi.reserve(ntg, st, false), "allocate target hi");
+  KS_CUDA(ctx->tgt_lo.reserve(ntg, st, false), "allocate target lo");
+  KS_CUDA(ctx->nb.reserve((size_t)n_pad, st, false), "allocate target norms");
+  KS_CUDA(ks::launch_prep_tc_targets(beta, N, n_pad, ctx->K, k_pad, ctx->mu.p, ctx->c, ctx->tgt_hi.p, ctx->tgt_lo.p,
+                                     ctx->nb.p, st),
+          "target prep (TC)");
+  ctx->launches += 1;
+  CUtensorMap maps[6];
+  ks_status s = encode_2d_sw64(&maps[0], ctx->tgt_hi.p, k_pad, n_pad, ks::kTcTileT);
+  if (s != KS_OK) return s;
+  s = encode_2d_sw64(&maps[1], ctx->tgt_lo.p, k_pad, n_pad, ks::kTcTileT);
+  if (s != KS_OK) return s;
+  maps[2] = ctx->tmB_hi;
+  maps[3] = ctx->tmB_lo;
+
+  ks::StreamK sk;
+  sk.n_t = n_pad / ks::kTcTileT;
+  sk.n_s = (int32_t)(ctx->m_pad / ks::kTcTileS);
+  sk.units = sk.n_t * (int64_t)sk.n_s;
+  int64_t g = ctx->num_sms;
+  if (g > sk.units) g = sk.units;
+  sk.grid = (int32_t)g;
+  KS_CUDA(ctx->partial.reserve((size_t)sk.grid * 2 * ks::kTcTileT * 32, st, false), "allocate partials");
+  KS_CUDA(ctx->counters.reserve((size_t)sk.n_t, st, true), "allocate tile counters");
+
+  ks::TcArgs a;
+  a.N = N;
+  a.k_pad = k_pad;
+  a.R = ctx->R;
+  a.three = (ctx->prec_eff == KS_PREC_TF32) ? 0 : 1;
+  a.na = ctx->na.p;
+  a.nb = ctx->nb.p;
+  a.V = V;
+  a.partial = ctx->partial.p;
+  a.counters = ctx->counters.p;
+  a.sk = sk;
+  a.cta_times = nullptr;
+  const char* dbg = getenv("KS_CTA_TIMES");
+  if (dbg && *dbg) {
+    KS_CUDA(ctx->dbg_times.reserve((size_t)sk.grid * 2, st, true), "allocate debug timers");
+    a.cta_times = ctx->dbg_times.p;
+  }
+  for (int r_off = 0; r_off < ctx->r_pad;) {
+    const int r_c = (ctx->r_pad - r_off >= 32) ? 32 : 16;
+    a.r_c = r_c;
+    a.r_off = r_off;
+    a.r_valid = (ctx->R - r_off < r_c) ? (ctx->R - r_off) : r_c;
+    s = encode_wt(&maps[4], ctx->wt_hi.p, ctx->m_pad, ctx->r_pad, r_c);
+    if (s != KS_OK) return s;
+    s = encode_wt(&maps[5], ctx->wt_lo.p, ctx->m_pad, ctx->r_pad, r_c);
+    if (s != KS_OK) return s;
+    cudaEvent_t stop;
+    s = timed_begin(ctx, &stop);
+    if (s != KS_OK) return s;
+    KS_CUDA(ks::launch_fused_tc(maps, a, st), "fused TC kernel launch");
+    ctx->launches++;
+    ctx->fused_launches++;
+    ctx->last_grid = sk.grid;
+    s = timed_end(ctx, stop);
+    if (s != KS_OK) return s;
+    r_off += r_c;
+  }
+  if (a.cta_times) {
+    std::vector<unsigned long long> h((size_t)sk.grid * 2);
+    KS_CUDA(cudaMemcpyAsync(h.data(), a.cta_times, h.size() * 8, cudaMemcpyDeviceToHost, st), "copy debug timers");
+    KS_CUDA(cudaStreamSynchronize(st), "synchronize");
+    FILE* f = fopen(dbg, "a");
+    if (f) {
+      for (int i = 0; i < sk.grid; ++i) fprintf(f, "%d %llu %llu\n", i, h[2 * i], h[2 * i + 1]);
+      fprintf(f, "--\n");
+      fclose(f);
+    }
+  }
+  return KS_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -315,6 +468,9 @@ ks_status ks_destroy(ks_ctx* ctx) {
   set_device(ctx);
   cudaStreamSynchronize(ctx->stream);
   ctx->src.release();
+  for (DBuf<float>* bptr : {&ctx->src_hi, &ctx->src_lo, &ctx->na, &ctx->wt_hi, &ctx->wt_lo, &ctx->tgt_hi, &ctx->tgt_lo,
+                            &ctx->nb})
+    bptr->release();
   ctx->mu.release();
   ctx->mean_part.release();
   ctx->partial.release();
@@ -361,12 +517,11 @@ ks_status ks_set_sources(ks_ctx* ctx, const float* alpha, const float* W, int64_
   } else {
     path = KS_PATH_TC;
   }
-  if (path == KS_PATH_TC)
-    return fail(KS_EUNSUPPORTED, "tensor-core path (K=%d, R=%d, precision %d) not built yet", ctx->K, R, prec);
   ks_status s = set_device(ctx);
   if (s != KS_OK) return s;
   ctx->have_src = false;
-  s = prepare_fp32(ctx, alpha, W, M);
+  ctx->prec_eff = prec;
+  s = (path == KS_PATH_TC) ? prepare_tc(ctx, alpha, W, M, R) : prepare_fp32(ctx, alpha, W, M);
   if (s != KS_OK) return s;
   ctx->path = path;
   ctx->prec_eff = prec;
@@ -389,7 +544,7 @@ ks_status ks_eval(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
     KS_CUDA(cudaMemsetAsync(V, 0, (size_t)N * ctx->R * sizeof(float), ctx->stream), "zero V");
     return KS_OK;
   }
-  return eval_fp32(ctx, beta, N, V);
+  return (ctx->path == KS_PATH_TC) ? eval_tc(ctx, beta, N, V) : eval_fp32(ctx, beta, N, V);
 }
 
 ks_status ks_reserve(ks_ctx* ctx, int64_t N_max) {
@@ -397,9 +552,10 @@ ks_status ks_reserve(ks_ctx* ctx, int64_t N_max) {
   if (N_max < 0) return fail(KS_EINVAL, "N_max < 0");
   ks_status s = set_device(ctx);
   if (s != KS_OK) return s;
-  const int64_t n_t = (N_max + ks::kTileT - 1) / ks::kTileT;
-  const int64_t g = (int64_t)ctx->num_sms * 8;  // >= any persistent grid
-  KS_CUDA(ctx->partial.reserve((size_t)g * 2 * ks::kTileT, ctx->stream, false), "allocate partials");
+  const int64_t n_t = (N_max + ks::kTcTileT - 1) / ks::kTcTileT;  // the finer of the two target tilings
+  const int64_t g = (int64_t)ctx->num_sms;  // persistent grids are <= one CTA per SM
+  const size_t per_cta = std::max((size_t)2 * ks::kTileT, (size_t)2 * ks::kTcTileT * 32);
+  KS_CUDA(ctx->partial.reserve((size_t)g * per_cta, ctx->stream, false), "allocate partials");
   KS_CUDA(ctx->counters.reserve((size_t)(n_t > 0 ? n_t : 1), ctx->stream, true), "allocate tile counters");
   return KS_OK;
 }
@@ -449,10 +605,11 @@ ks_status ks_get_info(const ks_ctx* ctx, ks_info* out) {
   out->path = ctx->have_src ? ctx->path : KS_PATH_NONE;
   out->precision = ctx->have_src ? ctx->prec_eff : ctx->prec_req;
   out->k_pad = ctx->k_pad;
-  out->tile_t = ks::kTileT;
-  out->tile_s = ks::kTileS;
+  const bool tc = ctx->have_src && ctx->path == KS_PATH_TC;
+  out->tile_t = tc ? ks::kTcTileT : ks::kTileT;
+  out->tile_s = tc ? ks::kTcTileS : ks::kTileS;
   out->num_ctas = ctx->last_grid;
-  out->stages = ctx->k_pad ? ks::fused_fp32_stages(ctx->k_pad) : 0;
+  out->stages = !ctx->k_pad ? 0 : (tc ? ks::fused_tc_stages() : ks::fused_fp32_stages(ctx->k_pad));
   out->num_sms = ctx->num_sms;
   out->m = ctx->M;
   out->m_pad = ctx->m_pad;

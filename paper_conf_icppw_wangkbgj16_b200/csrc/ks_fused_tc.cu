@@ -1,0 +1,446 @@
+// ks_fused_tc.cu -- the fused tensor-core (tcgen05 / TMEM) kernel-summation
+// kernel for K > 32 or R > 1 weight columns (scope rows a2-a7, TC variant).
+//
+// What it computes (PAPER.md SS III-C, Alg.2; Eq.3):
+//   S_ji = sum_d bh_jd * a_id           (a = 2c alpha_hat, bh = beta_hat)
+//   t_ji = min(S_ji + na_i + nb_j, 0)   (= -log2(e) d^2/(2h^2), clamped d^2 >= 0)
+//   P_ji = ex2(t_ji) = exp(-||alpha_i - beta_j||^2 / (2h^2))        (Eq.1)
+//   V_jr = sum_i P_ji W_ir                                          (Eq.2)
+// Both contractions run on the 5th-generation tensor cores in TF32 with a
+// hi/lo split of every operand ("3xTF32": lo.hi + hi.lo + hi.hi, the lo.lo
+// term is below FP32 rounding), so the result matches FP32 arithmetic
+// (SS3 reading Q16, SS4 tolerances); KS_PREC_TF32 keeps hi.hi only.
+//
+// Structure (one persistent 384-thread CTA per SM, stream-K over
+// (128-target tile x 128-source tile) units, like the FP32 kernel):
+//   warp 0   TMA producer: per unit, the W^T tile (hi/lo, 3-D box) and na into
+//            a 2-slot ring; per 16-wide K chunk, A = targets (hi/lo) and
+//            B = sources (hi/lo) tiles (SWIZZLE_64B) into an S-stage ring.
+//   warp 1   MMA issuer (one thread): S(q) = A B^T into TMEM buffer q%2
+//            (M=128, N=128, K=8 per instruction), then V(q-1) += P(q-1) W
+//            with P read from TMEM (A operand in TMEM, M=128, N=r_c, K=8).
+//   warp 2   TMEM allocation (512 columns: S0 | S1 | P_lo | V).
+//   warps 4-11 epilogue: tcgen05.ld S, add norms, clamp, MUFU ex2, split P into
+//            TF32 hi/lo, tcgen05.st P_hi in place of S and P_lo beside it;
+//            every <= 4 units read V (FP32 TMEM accumulator) into FP64
+//            registers; at segment end write V or a partial + deterministic
+//            last-arriver fix-up (no atomics on V).
+// The M x N kernel matrix exists only as 128x128 TMEM tiles.
+#include "ks_internal.h"
+#include "ks_ptx.cuh"
+
+namespace ks {
+
+namespace {
+
+constexpr int kStages = 4;                       // A/B ring depth (32 KB per stage)
+constexpr int kFlush = 4;                        // units per V accumulation block
+constexpr uint32_t kChunkBytes = kTcTileT * kTcKC * 4;  // one hi or lo operand tile (8 KB)
+constexpr uint32_t kStageBytes = 4 * kChunkBytes;       // A_hi, A_lo, B_hi, B_lo
+constexpr uint32_t kColS0 = 0, kColS1 = 128, kColPlo = 256, kColV = 384;
+
+struct TcSmem {
+  // offsets in bytes from a 1024-aligned base
+  static constexpr uint32_t kStage0 = 0;
+  static constexpr uint32_t wslot(int r_c) { return (uint32_t)r_c * 512u; }  // one of hi/lo: 8 chunks x r_c x 64 B
+  static constexpr uint32_t kW0 = kStages * kStageBytes;
+  // hi, lo, na[128]; slots 1024-aligned so every SWIZZLE_64B atom starts on a 512 B boundary
+  static constexpr uint32_t w_slot_bytes(int r_c) { return (2 * wslot(r_c) + 512 + 1023) & ~1023u; }
+  static constexpr uint32_t bar_off(int r_c) { return kW0 + 2 * w_slot_bytes(r_c); }
+  static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 256 + 1024; }
+};
+
+__device__ __forceinline__ int64_t sk_start(int64_t b, int64_t U, int64_t G) { return (b * U) / G; }
+__device__ __forceinline__ int64_t sk_owner(int64_t u, int64_t U, int64_t G) { return ((u + 1) * G - 1) / U; }
+
+}  // namespace
+
+template <int RC>
+__global__ void __launch_bounds__(kTcThreads, 1)
+    ks_fused_tc_kernel(const __grid_constant__ CUtensorMap mA_hi, const __grid_constant__ CUtensorMap mA_lo,
+                       const __grid_constant__ CUtensorMap mB_hi, const __grid_constant__ CUtensorMap mB_lo,
+                       const __grid_constant__ CUtensorMap mW_hi, const __grid_constant__ CUtensorMap mW_lo,
+                       const TcArgs args) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + TcSmem::bar_off(RC));
+  uint64_t* full = bars;                 // [kStages]
+  uint64_t* empty = full + kStages;      // [kStages]
+  uint64_t* wfull = empty + kStages;     // [2]
+  uint64_t* wempty = wfull + 2;          // [2]
+  uint64_t* sfull = wempty + 2;          // [2]
+  uint64_t* pready = sfull + 2;          // [2]
+  uint64_t* vdone = pready + 2;          // [1]
+  uint32_t* tmem_base_smem = reinterpret_cast<uint32_t*>(vdone + 1);
+  int* flag = reinterpret_cast<int*>(tmem_base_smem + 1);
+
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int64_t U = args.sk.units, G = args.sk.grid;
+  const int n_s = args.sk.n_s;
+  const int64_t b = blockIdx.x;
+  const int64_t u0 = sk_start(b, U, G), u1 = sk_start(b + 1, U, G);
+  const int count = (int)(u1 - u0);
+  const int n_kc = args.k_pad / kTcKC;
+
+  if (args.cta_times != nullptr && tid == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    args.cta_times[2 * b] = t;
+  }
+  if (tid == 0) {
+    for (int i = 0; i < kStages; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&wfull[i], 1);
+      mbar_init(&wempty[i], 1);
+      mbar_init(&sfull[i], 1);
+      mbar_init(&pready[i], 8);  // 8 epilogue warps
+    }
+    mbar_init(vdone, 1);
+    fence_mbar_init();
+  }
+  if (warp == 2) tmem_alloc(tmem_base_smem, 512);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = *tmem_base_smem;
+
+  if (warp == 0) {
+    // ================= TMA producer
+    if (lane == 0) {
+      tma_prefetch_desc(&mA_hi);
+      tma_prefetch_desc(&mB_hi);
+      tma_prefetch_desc(&mW_hi);
+      int it = 0;
+      for (int q = 0; q < count; ++q) {
+        const int64_t u = u0 + q;
+        const int tt = (int)(u / n_s), st = (int)(u % n_s);
+        {
+          const int slot = q & 1;
+          const uint32_t use = (uint32_t)(q >> 1);
+          mbar_wait(&wempty[slot], (use & 1) ^ 1);
+          uint8_t* ws = smem + TcSmem::kW0 + slot * TcSmem::w_slot_bytes(RC);
+          mbar_arrive_expect_tx(&wfull[slot], 2 * TcSmem::wslot(RC) + 512);
+          tma_load_3d(ws, &mW_hi, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
+          tma_load_3d(ws + TcSmem::wslot(RC), &mW_lo, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
+          bulk_load(ws + 2 * TcSmem::wslot(RC), args.na + (int64_t)st * kTcTileS, 512, &wfull[slot]);
+        }
+        for (int kc = 0; kc < n_kc; ++kc, ++it) {
+          const int s = it % kStages;
+          const uint32_t use = (uint32_t)(it / kStages);
+          mbar_wait(&empty[s], (use & 1) ^ 1);
+          uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
+          mbar_arrive_expect_tx(&full[s], kStageBytes);
+          tma_load_2d(sp, &mA_hi, kc * kTcKC, tt * kTcTileT, &full[s]);
+          tma_load_2d(sp + kChunkBytes, &mA_lo, kc * kTcKC, tt * kTcTileT, &full[s]);
+          tma_load_2d(sp + 2 * kChunkBytes, &mB_hi, kc * kTcKC, st * kTcTileS, &full[s]);
+          tma_load_2d(sp + 3 * kChunkBytes, &mB_lo, kc * kTcKC, st * kTcTileS, &full[s]);
+        }
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    // ================= MMA issuer
+    if (lane == 0) {
+      const uint32_t idS = idesc_tf32(128, kTcTileS);
+      const uint32_t idV = idesc_tf32(128, RC);
+      int it = 0;
+      auto v_mma = [&](int p) {
+        const int64_t up = u0 + p;
+        const int sp_ = (int)(up % n_s);
+        const bool first = (p == 0) || (sp_ == 0) || (sp_ % kFlush == 0);
+        const int bp = p & 1;
+        const uint32_t use = (uint32_t)(p >> 1);
+        mbar_wait(&pready[bp], use & 1);
+        mbar_wait(&wfull[p & 1], use & 1);
+        tc_fence_after();
+        uint8_t* ws = smem + TcSmem::kW0 + (p & 1) * TcSmem::w_slot_bytes(RC);
+        const uint32_t colP = bp ? kColS1 : kColS0;
+        // products: P_lo.W_hi, P_hi.W_lo, P_hi.W_hi (small terms first)
+        const int nprod = args.three ? 3 : 1;
+        bool acc = !first;
+        for (int pr = 3 - nprod; pr < 3; ++pr) {
+          const uint32_t aCol = (pr == 0) ? kColPlo : colP;
+          const uint8_t* wB = ws + ((pr == 1) ? TcSmem::wslot(RC) : 0u);
+#pragma unroll 4
+          for (int ks = 0; ks < kTcTileS / 8; ++ks) {
+            const uint64_t bd = sdesc_k_sw64(wB + (ks >> 1) * (RC * 64) + (ks & 1) * 32);
+            mma_tf32_ts(tbase + kColV, tbase + aCol + ks * 8, bd, idV, acc ? 1u : 0u);
+            acc = true;
+          }
+        }
+        tc_commit(vdone);
+        tc_commit(&wempty[p & 1]);
+      };
+      for (int q = 0; q < count; ++q) {
+        const int bq = q & 1;
+        const uint32_t dS = tbase + (bq ? kColS1 : kColS0);
+        for (int kc = 0; kc < n_kc; ++kc, ++it) {
+          const int s = it % kStages;
+          const uint32_t use = (uint32_t)(it / kStages);
+          mbar_wait(&full[s], use & 1);
+          tc_fence_after();
+          uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
+#pragma unroll
+          for (int ks = 0; ks < kTcKC / 8; ++ks) {
+            const uint64_t aH = sdesc_k_sw64(sp + ks * 32);
+            const uint64_t aL = sdesc_k_sw64(sp + kChunkBytes + ks * 32);
+            const uint64_t bH = sdesc_k_sw64(sp + 2 * kChunkBytes + ks * 32);
+            const uint64_t bL = sdesc_k_sw64(sp + 3 * kChunkBytes + ks * 32);
+            const uint32_t acc0 = (kc > 0 || ks > 0) ? 1u : 0u;
+            if (args.three) {
+              mma_tf32_ss(dS, aL, bH, idS, acc0);
+              mma_tf32_ss(dS, aH, bL, idS, 1u);
+              mma_tf32_ss(dS, aH, bH, idS, 1u);
+            } else {
+              mma_tf32_ss(dS, aH, bH, idS, acc0);
+            }
+          }
+          tc_commit(&empty[s]);
+        }
+        tc_commit(&sfull[bq]);
+        if (q > 0) v_mma(q - 1);
+      }
+      if (count > 0) v_mma(count - 1);
+    }
+    __syncwarp();
+  } else if (warp >= 4) {
+    // ================= epilogue (8 warps: lane group g, column half h)
+    const int g = warp & 3;               // TMEM lanes 32g..32g+31
+    const int h = (warp - 4) >> 2;        // columns 64h..64h+63 of the tile
+    const int row = 32 * g + lane;        // target row within the tile
+    const uint32_t lane_off = (uint32_t)(32 * g) << 16;
+    double vacc[RC];
+#pragma unroll
+    for (int r = 0; r < RC; ++r) vacc[r] = 0.0;
+    float nbj = 0.f;
+    int64_t seg_u = u0;  // first unit of the current segment
+
+    // read the V accumulator (unit p finished) into FP64 registers; at the end
+    // of a segment write V / partial.
+    auto v_collect = [&](int p) {
+      const int64_t up = u0 + p;
+      const int spp = (int)(up % n_s);
+      const bool last_in_block = (p == count - 1) || (spp + 1 == n_s) || ((spp + 1) % kFlush == 0);
+      const bool seg_end = (p == count - 1) || (spp + 1 == n_s);
+      if (h == 0 && last_in_block) {
+#pragma unroll
+        for (int r0 = 0; r0 < RC; r0 += 16) {
+          uint32_t v[16];
+          tmem_ld16(tbase + lane_off + kColV + r0, v);
+          tmem_wait_ld();
+#pragma unroll
+          for (int r = 0; r < 16; ++r) vacc[r0 + r] += (double)__uint_as_float(v[r]);
+        }
+      }
+      if (seg_end) {
+        const int64_t tt = up / n_s;
+        const int st0 = (int)(seg_u % n_s);
+        const int seg_len = (int)(up - seg_u + 1);
+        const bool whole = (st0 == 0) && (seg_len == n_s);
+        if (h == 0) {
+          const int64_t grow = tt * kTcTileT + row;
+          if (whole) {
+            if (grow < args.N) {
+#pragma unroll
+              for (int r = 0; r < RC; ++r)
+                if (r < args.r_valid) args.V[grow * args.R + args.r_off + r] = (float)vacc[r];
+            }
+          } else {
+            const int first_tile_of_b = (int)(u0 / n_s);
+            const int slot = (tt == first_tile_of_b) ? 0 : 1;
+            float* pp = args.partial + ((b * 2 + slot) * kTcTileT + row) * RC;
+#pragma unroll
+            for (int r = 0; r < RC; ++r) pp[r] = (float)vacc[r];
+            __threadfence();
+            named_bar_sync(1, 128);
+            const int64_t b_first = sk_owner(tt * n_s, U, G);
+            const int64_t b_last = sk_owner(tt * n_s + n_s - 1, U, G);
+            if (row == 0) {
+              const int old = atomicAdd(&args.counters[tt], 1);
+              const int last = (old == (int)(b_last - b_first));
+              if (last) args.counters[tt] = 0;
+              *flag = last;
+            }
+            named_bar_sync(1, 128);
+            if (*flag) {
+              __threadfence();
+              float sum[RC];
+#pragma unroll
+              for (int r = 0; r < RC; ++r) sum[r] = 0.f;
+              for (int64_t bb = b_first; bb <= b_last; ++bb) {
+                const int sl = (tt == sk_start(bb, U, G) / n_s) ? 0 : 1;
+                const float* qp = args.partial + ((bb * 2 + sl) * kTcTileT + row) * RC;
+#pragma unroll
+                for (int r = 0; r < RC; ++r) sum[r] += __ldcg(qp + r);
+              }
+              if (grow < args.N) {
+#pragma unroll
+                for (int r = 0; r < RC; ++r)
+                  if (r < args.r_valid) args.V[grow * args.R + args.r_off + r] = sum[r];
+              }
+            }
+            named_bar_sync(1, 128);  // flag reuse
+          }
+        }
+#pragma unroll
+        for (int r = 0; r < RC; ++r) vacc[r] = 0.0;
+        seg_u = up + 1;
+      }
+    };
+
+    for (int q = 0; q < count; ++q) {
+      const int64_t u = u0 + q;
+      const int64_t tt = u / n_s;
+      const int bq = q & 1;
+      const uint32_t use = (uint32_t)(q >> 1);
+      if (q == 0 || (u % n_s) == 0) nbj = __ldg(args.nb + tt * kTcTileT + row);
+      mbar_wait(&wfull[q & 1], use & 1);
+      mbar_wait(&sfull[bq], use & 1);
+      tc_fence_after();
+      if (q > 0) {
+        mbar_wait(vdone, (uint32_t)((q - 1) & 1));  // V(q-1) done: P_lo free, V readable
+        tc_fence_after();
+        v_collect(q - 1);
+      }
+      const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC) +
+                                                       2 * TcSmem::wslot(RC));
+      const uint32_t colS = bq ? kColS1 : kColS0;
+#pragma unroll 1
+      for (int cb = 0; cb < 2; ++cb) {
+        const int c0 = 64 * h + 32 * cb;
+        uint32_t sv[32];
+        tmem_ld32(tbase + lane_off + colS + c0, sv);
+        tmem_wait_ld();
+        uint32_t hi[32], lo[32];
+#pragma unroll
+        for (int i = 0; i < 32; i += 4) {
+          const float4 na4 = *reinterpret_cast<const float4*>(nas + c0 + i);
+          const float nav[4] = {na4.x, na4.y, na4.z, na4.w};
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const float t = fminf(__uint_as_float(sv[i + e]) + (nav[e] + nbj), 0.f);
+            const float p = ex2_approx(t);
+            const float ph = to_tf32(p);
+            hi[i + e] = __float_as_uint(ph);
+            lo[i + e] = __float_as_uint(to_tf32(p - ph));
+          }
+        }
+        tmem_st32(tbase + lane_off + colS + c0, hi);
+        if (args.three) tmem_st32(tbase + lane_off + kColPlo + c0, lo);
+      }
+      tmem_wait_st();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&pready[bq]);
+    }
+    if (count > 0) {
+      mbar_wait(vdone, (uint32_t)((count - 1) & 1));
+      tc_fence_after();
+      v_collect(count - 1);
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (warp == 2) tmem_dealloc(tbase, 512);
+  if (args.cta_times != nullptr && tid == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    args.cta_times[2 * b + 1] = t;
+  }
+}
+
+// ---------------------------------------------------------------- prep (a1 / a2 for the TC path)
+__global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const float* __restrict__ W, int64_t M,
+                                       int64_t m_pad, int K, int k_pad, int R, int r_pad,
+                                       const float* __restrict__ mu, double c, float* __restrict__ src_hi,
+                                       float* __restrict__ src_lo, float* __restrict__ na,
+                                       float* __restrict__ wt_hi, float* __restrict__ wt_lo) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= m_pad) return;
+  const bool live = i < M;
+  const double c2 = 2.0 * c;
+  double n = 0.0;
+  for (int d = 0; d < k_pad; ++d) {
+    float x = 0.f;
+    if (live && d < K) x = alpha[i * K + d] - mu[d];
+    n += (double)x * (double)x;
+    const float a = (float)(c2 * (double)x);
+    const float ah = to_tf32(a);
+    src_hi[i * k_pad + d] = ah;
+    src_lo[i * k_pad + d] = to_tf32(a - ah);
+  }
+  na[i] = live ? (float)(-c * n) : 0.f;
+  for (int r = 0; r < r_pad; ++r) {
+    const float w = (live && r < R) ? W[i * R + r] : 0.f;
+    const float wh = to_tf32(w);
+    wt_hi[(int64_t)r * m_pad + i] = wh;
+    wt_lo[(int64_t)r * m_pad + i] = to_tf32(w - wh);
+  }
+}
+
+__global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N, int64_t n_pad, int K, int k_pad,
+                                       const float* __restrict__ mu, double c, float* __restrict__ tgt_hi,
+                                       float* __restrict__ tgt_lo, float* __restrict__ nb) {
+  const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= n_pad) return;
+  const bool live = j < N;
+  double n = 0.0;
+  for (int d = 0; d < k_pad; ++d) {
+    float x = 0.f;
+    if (live && d < K) x = beta[j * K + d] - mu[d];
+    n += (double)x * (double)x;
+    const float xh = to_tf32(x);
+    tgt_hi[j * k_pad + d] = xh;
+    tgt_lo[j * k_pad + d] = to_tf32(x - xh);
+  }
+  nb[j] = live ? (float)(-c * n) : 0.f;
+}
+
+cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
+                                   int R, int r_pad, const float* mu, double c, float* src_hi, float* src_lo,
+                                   float* na, float* wt_hi, float* wt_lo, cudaStream_t st) {
+  if (m_pad == 0) return cudaSuccess;
+  const int bs = 128;
+  prep_tc_sources_kernel<<<(unsigned)((m_pad + bs - 1) / bs), bs, 0, st>>>(alpha, W, M, m_pad, K, k_pad, R, r_pad, mu,
+                                                                          c, src_hi, src_lo, na, wt_hi, wt_lo);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
+                                   double c, float* tgt_hi, float* tgt_lo, float* nb, cudaStream_t st) {
+  if (n_pad == 0) return cudaSuccess;
+  const int bs = 128;
+  prep_tc_targets_kernel<<<(unsigned)((n_pad + bs - 1) / bs), bs, 0, st>>>(beta, N, n_pad, K, k_pad, mu, c, tgt_hi,
+                                                                          tgt_lo, nb);
+  return cudaGetLastError();
+}
+
+size_t fused_tc_smem(int r_c) { return r_c <= 16 ? TcSmem::total(16) : TcSmem::total(32); }
+int fused_tc_stages() { return kStages; }
+
+template <int RC>
+static cudaError_t launch_rc(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
+  static bool attr_done = false;
+  const size_t smem = TcSmem::total(RC);
+  if (!attr_done) {
+    cudaError_t e =
+        cudaFuncSetAttribute(ks_fused_tc_kernel<RC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr_done = true;
+  }
+  ks_fused_tc_kernel<RC><<<a.sk.grid, kTcThreads, smem, st>>>(m[0], m[1], m[2], m[3], m[4], m[5], a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st) {
+  if (a.r_c == 16) return launch_rc<16>(maps, a, st);
+  if (a.r_c == 32) return launch_rc<32>(maps, a, st);
+  return cudaErrorInvalidValue;
+}
+
+}  // namespace ks

@@ -53,3 +53,43 @@ int fused_fp32_ctas_per_sm(int k_pad);
 int fused_fp32_stages(int k_pad);
 
 }  // namespace ks
+
+namespace ks {
+
+// ---------------------------------------------------------------- tensor-core (tcgen05) path
+constexpr int kTcTileT = 128;  // targets per tile = MMA M = TMEM lanes
+constexpr int kTcTileS = 128;  // sources per tile = N of the S MMA = K of the V MMA
+constexpr int kTcKC = 16;      // K floats per pipeline stage (64-byte rows, SWIZZLE_64B)
+constexpr int kTcThreads = 384;  // warp 0 TMA, 1 MMA, 2 TMEM alloc, 3 idle, 4..11 epilogue
+
+struct TcArgs {
+  int64_t N;            // targets
+  int k_pad;            // multiple of kTcKC
+  int r_c;              // weight columns handled by this launch (16 or 32)
+  int r_valid;          // valid columns among them
+  int r_off;            // first weight column of this launch
+  int R;                // row stride of V
+  int three;            // 1: 3xTF32 (hi.hi + hi.lo + lo.hi), 0: plain TF32 (hi.hi)
+  const float* na;      // [m_pad]  -c ||alpha_hat||^2
+  const float* nb;      // [n_pad]  -c ||beta_hat||^2
+  float* V;             // [N][R]
+  float* partial;       // [grid][2][kTcTileT][r_c]
+  int* counters;        // [n_t]
+  StreamK sk;
+  unsigned long long* cta_times;
+};
+
+// sources: src_hi/lo [m_pad][k_pad] = TF32 split of RN(2c (alpha - mu)),
+// na [m_pad], W^T split wt_hi/lo [r_pad][m_pad] (zero padded)
+cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
+                                   int R, int r_pad, const float* mu, double c, float* src_hi, float* src_lo,
+                                   float* na, float* wt_hi, float* wt_lo, cudaStream_t st);
+// targets: tgt_hi/lo [n_pad][k_pad] = TF32 split of (beta - mu), nb [n_pad]
+cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
+                                   double c, float* tgt_hi, float* tgt_lo, float* nb, cudaStream_t st);
+// maps: A_hi, A_lo (targets), B_hi, B_lo (sources), W_hi, W_lo (weights^T)
+cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st);
+int fused_tc_stages();
+size_t fused_tc_smem(int r_c);
+
+}  // namespace ks
