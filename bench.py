@@ -58,6 +58,8 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
     p.add_argument("--no-flush", action="store_true")
+    p.add_argument("--precision", default="auto", choices=["auto", "fp32", "3xtf32", "tf32"],
+                   help="ks_set_precision (auto: FP32 path for K<=32 and R=1, else 3xTF32 tensor cores)")
     return p.parse_args()
 
 
@@ -197,12 +199,19 @@ def l2_flush(buf):
     buf.add_(1.0)  # 256 MiB read+write > 126 MB L2
 
 
-def load_traffic(cfg):
+def load_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+def load_traffic(cfg, precision="auto"):
     """DRAM bytes per launch of the fused kernel from the committed ncu capture, if any."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
         d = json.load(open(p))
-        e = d.get(f"cfg{cfg}", {})
+        e = d.get(f"cfg{cfg}" if precision == "auto" else f"cfg{cfg}_{precision}", {})
         return e.get("dram_bytes_per_launch")
     except Exception:
         return None
@@ -230,7 +239,7 @@ def run_ours(args):
     M, N, K, R = c.M, c.N, c.K, c.R
     lo, hi = shard_bounds(N, world, rank)
 
-    plan = ks.KernelSum(K, float(h))
+    plan = ks.KernelSum(K, float(h), args.precision)
     ta = torch.from_numpy(a).to(dev) if rank == 0 or world == 1 else torch.empty((M, K), device=dev)
     tw = torch.from_numpy(W).to(dev) if rank == 0 or world == 1 else torch.empty((M, R), device=dev)
     tb = torch.from_numpy(b[lo:hi].copy()).to(dev)
@@ -295,23 +304,38 @@ def run_ours(args):
     value = pairs_per_step / (ms_per_step / 1e3)
 
     # ---- roofline of the dominant (fused) kernel, from its own CUDA events
-    kms = kern_ms / max(kern_n, 1)
+    # (ks_timing: events recorded on the launching stream around every fused
+    # launch of the timed region); per step = all fused launches of one step.
+    kms = kern_ms / args.steps
     pairs_launch = M * (hi - lo)
-    fp32_ops, mufu = per_pair_ops(K, R)
-    achieved = pairs_launch * fp32_ops / (kms / 1e3) / 1e12      # T FP32-pipe lane-ops / s
     sms = info1["num_sms"]
     clk_sum = clk.summary()
     max_mhz = clk_sum["sm_max_mhz"] or 1965
-    peak = 128 * sms * max_mhz * 1e6 / 1e12
-    roof = {"bound": "alu", "kernel": "ks_fused_fp32_kernel", "achieved": achieved, "peak": peak,
-            "unit": "Top/s FP32-pipe lane ops (K+2 per pair: K FFMA dot, 1 FADD norm, 1 FFMA weight)",
-            "frac": achieved / peak, "traffic": load_traffic(args.cfg),
-            "peak_derivation": f"128 FP32 lanes/clk/SM x {sms} SMs x {max_mhz} MHz (sm_max); MUFU ex2 "
-                               f"16/clk/SM is not binding at K={K}",
-            "kernel_ms": kms, "kernel_share_of_step": kms / ms_per_step if ms_per_step else None,
-            "pairs_per_launch": pairs_launch}
-    if clk_sum["sm_mhz"]:
-        roof["frac_at_measured_clock"] = achieved / (128 * sms * clk_sum["sm_mhz"] * 1e6 / 1e12)
+    if info1["path"] == ks.KS_PATH_TC:
+        nprod = 3 if info1["precision"] == ks.KS_PREC_3XTF32 else 1
+        flops_pair = nprod * 2 * (K + R)
+        achieved = pairs_launch * flops_pair / (kms / 1e3) / 1e12
+        bf16 = load_peaks().get("bf16_tflops")
+        peak = (bf16 * 0.5) if bf16 else 1100.0
+        roof = {"bound": "tensor", "kernel": "ks_fused_tc_kernel", "achieved": achieved, "peak": peak,
+                "unit": "TFLOP/s (TF32 tensor; %d products x 2(K+R) per pair)" % nprod, "frac": achieved / peak,
+                "traffic": load_traffic(args.cfg, args.precision),
+                "peak_derivation": ("MEASURED_PEAKS bf16_tflops (burst) %.1f x 0.5 (nominal TF32/BF16 = 1.1/2.25 "
+                                    "PFLOP/s)" % bf16) if bf16 else "fallback nominal dense TF32 1.1 PFLOP/s"}
+    else:
+        fp32_ops, mufu = per_pair_ops(K, R)
+        achieved = pairs_launch * fp32_ops / (kms / 1e3) / 1e12      # T FP32-pipe lane-ops / s
+        peak = 128 * sms * max_mhz * 1e6 / 1e12
+        roof = {"bound": "alu", "kernel": "ks_fused_fp32_kernel", "achieved": achieved, "peak": peak,
+                "unit": "Top/s FP32-pipe lane ops (K+2 per pair: K FFMA dot, 1 FADD norm, 1 FFMA weight)",
+                "frac": achieved / peak, "traffic": load_traffic(args.cfg, args.precision),
+                "peak_derivation": f"128 FP32 lanes/clk/SM x {sms} SMs x {max_mhz} MHz (sm_max); MUFU ex2 "
+                                   f"16/clk/SM is not binding at K={K}"}
+        if clk_sum["sm_mhz"]:
+            roof["frac_at_measured_clock"] = achieved / (128 * sms * clk_sum["sm_mhz"] * 1e6 / 1e12)
+    roof.update({"kernel_ms": kms, "kernel_launches_per_step": kern_n / args.steps,
+                 "kernel_share_of_step": kms / ms_per_step if ms_per_step else None,
+                 "pairs_per_step": pairs_launch})
 
     # ---- e2e through the C-ABI host entry points (pinned buffers, copies timed)
     ha = torch.from_numpy(a).pin_memory()
@@ -319,7 +343,7 @@ def run_ours(args):
     hb = torch.from_numpy(b[lo:hi].copy()).pin_memory()
     hv = torch.empty((max(hi - lo, 1), R), dtype=torch.float32).pin_memory()
     an, wn, bn, vn = ha.numpy(), hw.numpy(), hb.numpy(), hv.numpy()
-    e2e_plan = ks.KernelSum(K, float(h))
+    e2e_plan = ks.KernelSum(K, float(h), args.precision)
 
     def e2e_step():
         if world > 1:
@@ -355,13 +379,17 @@ def run_ours(args):
 
     out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-           "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+           "scaling": "strong", "vs_baseline": None,
+           "dtype": "f32" if info1["path"] == ks.KS_PATH_FP32 else "tf32x3" if info1["precision"] == 2 else "tf32",
+           "data": "synthetic",
            "config": {"workload": workload_desc(c),
                       "l2": "flushed before every step (256 MiB write, outside the step events)",
                       "parallelism": f"target-sharded x{world}" + (" (NCCL broadcast alpha,W + all-gather V)"
                                                                     if world > 1 else ""),
                       "step": "ks_set_sources (a1) + ks_eval (a2-a7)" + (" + collectives" if world > 1 else ""),
-                      "path": info1["path"], "k_pad": info1["k_pad"], "ctas": info1["num_ctas"],
+                      "path": {1: "fp32", 2: "tcgen05"}.get(info1["path"], info1["path"]),
+                      "precision": {1: "fp32", 2: "3xtf32", 3: "tf32"}.get(info1["precision"]),
+                      "k_pad": info1["k_pad"], "ctas": info1["num_ctas"],
                       "stages": info1["stages"]},
            "roofline": roof, "e2e": e2e, "clocks": clk_sum, "gpu_launches": launches,
            "gpu": torch.cuda.get_device_name(dev)}

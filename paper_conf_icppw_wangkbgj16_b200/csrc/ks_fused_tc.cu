@@ -29,17 +29,20 @@
 #include "ks_internal.h"
 #include "ks_ptx.cuh"
 
+#include <cstdlib>
+
 namespace ks {
 
 namespace {
 
-constexpr int kStages = 4;                       // A/B ring depth (32 KB per stage)
+constexpr int kMaxStages = 6;                    // A/B ring depth bound (32 KB per stage)
 constexpr int kFlush = 4;                        // units per V accumulation block
 constexpr uint32_t kChunkBytes = kTcTileT * kTcKC * 4;  // one hi or lo operand tile (8 KB)
 constexpr uint32_t kStageBytes = 4 * kChunkBytes;       // A_hi, A_lo, B_hi, B_lo
 constexpr uint32_t kColS0 = 0, kColS1 = 128, kColPlo = 256, kColV = 384;
 
-struct TcSmem {
+template <int kStages>
+struct TcSmemT {
   // offsets in bytes from a 1024-aligned base
   static constexpr uint32_t kStage0 = 0;
   static constexpr uint32_t wslot(int r_c) { return (uint32_t)r_c * 512u; }  // one of hi/lo: 8 chunks x r_c x 64 B
@@ -53,14 +56,44 @@ struct TcSmem {
 __device__ __forceinline__ int64_t sk_start(int64_t b, int64_t U, int64_t G) { return (b * U) / G; }
 __device__ __forceinline__ int64_t sk_owner(int64_t u, int64_t U, int64_t G) { return ((u + 1) * G - 1) / U; }
 
+// Persistent schedule, L2-friendly: `waves` full waves in which CTA b owns the
+// whole target tile w*G + b and every CTA sweeps the source tiles in the same
+// order (the source tile being read is shared by all SMs through L2), then a
+// stream-K split of the remaining r < G target tiles over Gr = min(G, r*n_s)
+// CTAs (fixed partial slots + last-arriver fix-up).
+struct Sched {
+  int64_t G, b, waves, rem_t0, Urem, Gr, v0;
+  int n_s, qw, count;
+  __device__ void init(int64_t n_t, int ns, int64_t grid, int64_t blk) {
+    n_s = ns; G = grid; b = blk;
+    waves = n_t / G;
+    rem_t0 = waves * G;
+    Urem = (n_t - rem_t0) * n_s;
+    Gr = Urem < G ? Urem : G;
+    qw = (int)(waves * n_s);
+    int64_t v1 = 0;
+    v0 = 0;
+    if (b < Gr) { v0 = sk_start(b, Urem, Gr); v1 = sk_start(b + 1, Urem, Gr); }
+    count = qw + (int)(v1 - v0);
+  }
+  __device__ void unit(int q, int64_t& tt, int& st) const {
+    if (q < qw) { tt = (int64_t)(q / n_s) * G + b; st = q % n_s; }
+    else { const int64_t v = v0 + (q - qw); tt = rem_t0 + v / n_s; st = (int)(v % n_s); }
+  }
+  __device__ bool first_in_block(int q, int st) const {
+    return q == 0 || q == qw || st == 0 || (st % kFlush) == 0;
+  }
+};
+
 }  // namespace
 
-template <int RC>
+template <int RC, int kStages>
 __global__ void __launch_bounds__(kTcThreads, 1)
     ks_fused_tc_kernel(const __grid_constant__ CUtensorMap mA_hi, const __grid_constant__ CUtensorMap mA_lo,
                        const __grid_constant__ CUtensorMap mB_hi, const __grid_constant__ CUtensorMap mB_lo,
                        const __grid_constant__ CUtensorMap mW_hi, const __grid_constant__ CUtensorMap mW_lo,
                        const TcArgs args) {
+  using TcSmem = TcSmemT<kStages>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + TcSmem::bar_off(RC));
@@ -75,11 +108,11 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   int* flag = reinterpret_cast<int*>(tmem_base_smem + 1);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int64_t U = args.sk.units, G = args.sk.grid;
   const int n_s = args.sk.n_s;
   const int64_t b = blockIdx.x;
-  const int64_t u0 = sk_start(b, U, G), u1 = sk_start(b + 1, U, G);
-  const int count = (int)(u1 - u0);
+  Sched sc;
+  sc.init(args.sk.n_t, n_s, args.sk.grid, b);
+  const int count = sc.count;
   const int n_kc = args.k_pad / kTcKC;
 
   if (args.cta_times != nullptr && tid == 0) {
@@ -115,8 +148,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       tma_prefetch_desc(&mW_hi);
       int it = 0;
       for (int q = 0; q < count; ++q) {
-        const int64_t u = u0 + q;
-        const int tt = (int)(u / n_s), st = (int)(u % n_s);
+        int64_t tt64;
+        int st;
+        sc.unit(q, tt64, st);
+        const int tt = (int)tt64;
         {
           const int slot = q & 1;
           const uint32_t use = (uint32_t)(q >> 1);
@@ -148,9 +183,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       const uint32_t idV = idesc_tf32(128, RC);
       int it = 0;
       auto v_mma = [&](int p) {
-        const int64_t up = u0 + p;
-        const int sp_ = (int)(up % n_s);
-        const bool first = (p == 0) || (sp_ == 0) || (sp_ % kFlush == 0);
+        int64_t tp;
+        int sp_;
+        sc.unit(p, tp, sp_);
+        const bool first = sc.first_in_block(p, sp_);
         const int bp = p & 1;
         const uint32_t use = (uint32_t)(p >> 1);
         mbar_wait(&pready[bp], use & 1);
@@ -212,91 +248,97 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     const int h = (warp - 4) >> 2;        // columns 64h..64h+63 of the tile
     const int row = 32 * g + lane;        // target row within the tile
     const uint32_t lane_off = (uint32_t)(32 * g) << 16;
-    double vacc[RC];
+    // each epilogue thread owns V columns [h*HC, (h+1)*HC) of its target row
+    constexpr int HC = RC / 2;
+    const int rbase = h * HC;
+    double vacc[HC];
 #pragma unroll
-    for (int r = 0; r < RC; ++r) vacc[r] = 0.0;
+    for (int r = 0; r < HC; ++r) vacc[r] = 0.0;
     float nbj = 0.f;
-    int64_t seg_u = u0;  // first unit of the current segment
+    int seg_q = 0;  // first local unit of the current segment
 
     // read the V accumulator (unit p finished) into FP64 registers; at the end
     // of a segment write V / partial.
     auto v_collect = [&](int p) {
-      const int64_t up = u0 + p;
-      const int spp = (int)(up % n_s);
+      int64_t tt;
+      int spp;
+      sc.unit(p, tt, spp);
       const bool last_in_block = (p == count - 1) || (spp + 1 == n_s) || ((spp + 1) % kFlush == 0);
       const bool seg_end = (p == count - 1) || (spp + 1 == n_s);
-      if (h == 0 && last_in_block) {
-#pragma unroll
-        for (int r0 = 0; r0 < RC; r0 += 16) {
-          uint32_t v[16];
-          tmem_ld16(tbase + lane_off + kColV + r0, v);
-          tmem_wait_ld();
-#pragma unroll
-          for (int r = 0; r < 16; ++r) vacc[r0 + r] += (double)__uint_as_float(v[r]);
+      if (last_in_block) {
+        uint32_t v[HC];
+        if constexpr (HC == 16) {
+          tmem_ld16(tbase + lane_off + kColV + rbase, v);
+        } else {
+          tmem_ld8(tbase + lane_off + kColV + rbase, v);
         }
+        tmem_wait_ld();
+#pragma unroll
+        for (int r = 0; r < HC; ++r) vacc[r] += (double)__uint_as_float(v[r]);
       }
       if (seg_end) {
-        const int64_t tt = up / n_s;
-        const int st0 = (int)(seg_u % n_s);
-        const int seg_len = (int)(up - seg_u + 1);
+        int64_t t0;
+        int st0;
+        sc.unit(seg_q, t0, st0);
+        const int seg_len = p - seg_q + 1;
         const bool whole = (st0 == 0) && (seg_len == n_s);
-        if (h == 0) {
-          const int64_t grow = tt * kTcTileT + row;
-          if (whole) {
+        const int64_t grow = tt * kTcTileT + row;
+        if (whole) {
+          if (grow < args.N) {
+#pragma unroll
+            for (int r = 0; r < HC; ++r)
+              if (rbase + r < args.r_valid) args.V[grow * args.R + args.r_off + rbase + r] = (float)vacc[r];
+          }
+        } else {
+          // split tile: only in the stream-K remainder (tile index relative to rem_t0)
+          const int64_t tr = tt - sc.rem_t0;
+          const int64_t first_tile_of_b = sc.v0 / n_s;
+          const int slot = (tr == first_tile_of_b) ? 0 : 1;
+          float* pp = args.partial + ((b * 2 + slot) * kTcTileT + row) * RC + rbase;
+#pragma unroll
+          for (int r = 0; r < HC; ++r) pp[r] = (float)vacc[r];
+          __threadfence();
+          named_bar_sync(1, 256);
+          const int64_t b_first = sk_owner(tr * n_s, sc.Urem, sc.Gr);
+          const int64_t b_last = sk_owner(tr * n_s + n_s - 1, sc.Urem, sc.Gr);
+          if (row == 0 && h == 0) {
+            const int old = atomicAdd(&args.counters[tt], 1);
+            const int last = (old == (int)(b_last - b_first));
+            if (last) args.counters[tt] = 0;
+            *flag = last;
+          }
+          named_bar_sync(1, 256);
+          if (*flag) {
+            __threadfence();
+            float sum[HC];
+#pragma unroll
+            for (int r = 0; r < HC; ++r) sum[r] = 0.f;
+            for (int64_t bb = b_first; bb <= b_last; ++bb) {
+              const int sl = (tr == sk_start(bb, sc.Urem, sc.Gr) / n_s) ? 0 : 1;
+              const float* qp = args.partial + ((bb * 2 + sl) * kTcTileT + row) * RC + rbase;
+#pragma unroll
+              for (int r = 0; r < HC; ++r) sum[r] += __ldcg(qp + r);
+            }
             if (grow < args.N) {
 #pragma unroll
-              for (int r = 0; r < RC; ++r)
-                if (r < args.r_valid) args.V[grow * args.R + args.r_off + r] = (float)vacc[r];
+              for (int r = 0; r < HC; ++r)
+                if (rbase + r < args.r_valid) args.V[grow * args.R + args.r_off + rbase + r] = sum[r];
             }
-          } else {
-            const int first_tile_of_b = (int)(u0 / n_s);
-            const int slot = (tt == first_tile_of_b) ? 0 : 1;
-            float* pp = args.partial + ((b * 2 + slot) * kTcTileT + row) * RC;
-#pragma unroll
-            for (int r = 0; r < RC; ++r) pp[r] = (float)vacc[r];
-            __threadfence();
-            named_bar_sync(1, 128);
-            const int64_t b_first = sk_owner(tt * n_s, U, G);
-            const int64_t b_last = sk_owner(tt * n_s + n_s - 1, U, G);
-            if (row == 0) {
-              const int old = atomicAdd(&args.counters[tt], 1);
-              const int last = (old == (int)(b_last - b_first));
-              if (last) args.counters[tt] = 0;
-              *flag = last;
-            }
-            named_bar_sync(1, 128);
-            if (*flag) {
-              __threadfence();
-              float sum[RC];
-#pragma unroll
-              for (int r = 0; r < RC; ++r) sum[r] = 0.f;
-              for (int64_t bb = b_first; bb <= b_last; ++bb) {
-                const int sl = (tt == sk_start(bb, U, G) / n_s) ? 0 : 1;
-                const float* qp = args.partial + ((bb * 2 + sl) * kTcTileT + row) * RC;
-#pragma unroll
-                for (int r = 0; r < RC; ++r) sum[r] += __ldcg(qp + r);
-              }
-              if (grow < args.N) {
-#pragma unroll
-                for (int r = 0; r < RC; ++r)
-                  if (r < args.r_valid) args.V[grow * args.R + args.r_off + r] = sum[r];
-              }
-            }
-            named_bar_sync(1, 128);  // flag reuse
           }
+          named_bar_sync(1, 256);  // flag reuse
         }
 #pragma unroll
-        for (int r = 0; r < RC; ++r) vacc[r] = 0.0;
-        seg_u = up + 1;
+        for (int r = 0; r < HC; ++r) vacc[r] = 0.0;
+        seg_q = p + 1;
       }
     };
 
     for (int q = 0; q < count; ++q) {
-      const int64_t u = u0 + q;
-      const int64_t tt = u / n_s;
+      int64_t tt;
+      int stq;
+      sc.unit(q, tt, stq);
       const int bq = q & 1;
       const uint32_t use = (uint32_t)(q >> 1);
-      if (q == 0 || (u % n_s) == 0) nbj = __ldg(args.nb + tt * kTcTileT + row);
       mbar_wait(&wfull[q & 1], use & 1);
       mbar_wait(&sfull[bq], use & 1);
       tc_fence_after();
@@ -305,6 +347,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         tc_fence_after();
         v_collect(q - 1);
       }
+      if (q == seg_q) nbj = __ldg(args.nb + tt * kTcTileT + row);  // new segment: this target tile's norms
       const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC) +
                                                        2 * TcSmem::wslot(RC));
       const uint32_t colS = bq ? kColS1 : kColS0;
@@ -420,26 +463,53 @@ cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, 
   return cudaGetLastError();
 }
 
-size_t fused_tc_smem(int r_c) { return r_c <= 16 ? TcSmem::total(16) : TcSmem::total(32); }
-int fused_tc_stages() { return kStages; }
+// Pipeline depth: KS_TC_STAGES (3..6) overrides the default (measurement knob).
+static int tc_stages(int r_c) {
+  const char* e = getenv("KS_TC_STAGES");
+  int v = (e && e[0] >= '3' && e[0] <= '5') ? (e[0] - '0') : 5;
+  if (r_c > 16 && v > 4) v = 4;  // shared-memory budget (227 KB per CTA)
+  return v;
+}
 
-template <int RC>
-static cudaError_t launch_rc(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
+size_t fused_tc_smem(int r_c) {
+  const int ns = tc_stages(r_c);
+  switch (ns) {
+    case 3: return r_c <= 16 ? TcSmemT<3>::total(16) : TcSmemT<3>::total(32);
+    case 4: return r_c <= 16 ? TcSmemT<4>::total(16) : TcSmemT<4>::total(32);
+    default: return r_c <= 16 ? TcSmemT<5>::total(16) : TcSmemT<4>::total(32);
+  }
+}
+int fused_tc_stages() { return tc_stages(16); }
+
+template <int RC, int NS>
+static cudaError_t launch_rcs(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
   static bool attr_done = false;
-  const size_t smem = TcSmem::total(RC);
+  const size_t smem = TcSmemT<NS>::total(RC);
   if (!attr_done) {
     cudaError_t e =
-        cudaFuncSetAttribute(ks_fused_tc_kernel<RC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(ks_fused_tc_kernel<RC, NS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr_done = true;
   }
-  ks_fused_tc_kernel<RC><<<a.sk.grid, kTcThreads, smem, st>>>(m[0], m[1], m[2], m[3], m[4], m[5], a);
+  ks_fused_tc_kernel<RC, NS><<<a.sk.grid, kTcThreads, smem, st>>>(m[0], m[1], m[2], m[3], m[4], m[5], a);
   return cudaGetLastError();
 }
 
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st) {
-  if (a.r_c == 16) return launch_rc<16>(maps, a, st);
-  if (a.r_c == 32) return launch_rc<32>(maps, a, st);
+  const int ns = tc_stages(a.r_c);
+  if (a.r_c == 16) {
+    switch (ns) {
+      case 3: return launch_rcs<16, 3>(maps, a, st);
+      case 4: return launch_rcs<16, 4>(maps, a, st);
+      default: return launch_rcs<16, 5>(maps, a, st);
+    }
+  }
+  if (a.r_c == 32) {
+    switch (ns) {
+      case 3: return launch_rcs<32, 3>(maps, a, st);
+      default: return launch_rcs<32, 4>(maps, a, st);
+    }
+  }
   return cudaErrorInvalidValue;
 }
 

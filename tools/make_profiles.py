@@ -5,7 +5,7 @@ by bench.py as roofline.traffic)."""
 import csv, io, json, os, shutil, subprocess, sys
 
 tag, rnd = sys.argv[1], sys.argv[2]
-cfgs = sys.argv[3:] or ["3"]
+cfgs = sys.argv[3:] or ["3"]   # entries like "3" or "4" (auto path) or "3_3xtf32"
 src = os.path.join("gpurun_out", tag)
 dst = os.path.join("profiles", rnd)
 os.makedirs(dst, exist_ok=True)
