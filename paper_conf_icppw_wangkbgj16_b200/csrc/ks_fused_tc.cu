@@ -39,6 +39,7 @@ constexpr int kMaxStages = 6;                    // A/B ring depth bound (32 KB 
 constexpr int kFlush = 4;                        // units per V accumulation block
 constexpr uint32_t kChunkBytes = kTcTileT * kTcKC * 4;  // one hi or lo operand tile (8 KB)
 constexpr uint32_t kStageBytes = 4 * kChunkBytes;       // A_hi, A_lo, B_hi, B_lo
+// TMEM columns: S0 | S1 (P_hi written in place) | P_lo for source half 0 | half 1 | V
 constexpr uint32_t kColS0 = 0, kColS1 = 128, kColPlo = 256, kColV = 384;
 
 template <int kStages>
@@ -50,7 +51,7 @@ struct TcSmemT {
   // hi, lo, na[128]; slots 1024-aligned so every SWIZZLE_64B atom starts on a 512 B boundary
   static constexpr uint32_t w_slot_bytes(int r_c) { return (2 * wslot(r_c) + 512 + 1023) & ~1023u; }
   static constexpr uint32_t bar_off(int r_c) { return kW0 + 2 * w_slot_bytes(r_c); }
-  static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 256 + 1024; }
+  static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 256; }
 };
 
 __device__ __forceinline__ int64_t sk_start(int64_t b, int64_t U, int64_t G) { return (b * U) / G; }
@@ -94,17 +95,17 @@ __global__ void __launch_bounds__(kTcThreads, 1)
                        const __grid_constant__ CUtensorMap mW_hi, const __grid_constant__ CUtensorMap mW_lo,
                        const TcArgs args) {
   using TcSmem = TcSmemT<kStages>;
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  extern __shared__ __align__(1024) uint8_t smem[];
+  if ((smem_u32(smem) & 1023u) != 0u) __trap();  // SWIZZLE_64B atoms and descriptors assume 1 KB alignment
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + TcSmem::bar_off(RC));
   uint64_t* full = bars;                 // [kStages]
   uint64_t* empty = full + kStages;      // [kStages]
   uint64_t* wfull = empty + kStages;     // [2]
   uint64_t* wempty = wfull + 2;          // [2]
   uint64_t* sfull = wempty + 2;          // [2]
-  uint64_t* pready = sfull + 2;          // [2]
-  uint64_t* vdone = pready + 2;          // [1]
-  uint32_t* tmem_base_smem = reinterpret_cast<uint32_t*>(vdone + 1);
+  uint64_t* pready = sfull + 2;          // [2 S buffers][2 source halves]
+  uint64_t* vdone = pready + 4;          // [2 source halves]
+  uint32_t* tmem_base_smem = reinterpret_cast<uint32_t*>(vdone + 2);
   int* flag = reinterpret_cast<int*>(tmem_base_smem + 1);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -129,9 +130,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       mbar_init(&wfull[i], 1);
       mbar_init(&wempty[i], 1);
       mbar_init(&sfull[i], 1);
-      mbar_init(&pready[i], 8);  // 8 epilogue warps
+      mbar_init(&vdone[i], 1);
     }
-    mbar_init(vdone, 1);
+    for (int i = 0; i < 4; ++i) mbar_init(&pready[i], 8);  // 8 epilogue warps
     fence_mbar_init();
   }
   if (warp == 2) tmem_alloc(tmem_base_smem, 512);
@@ -141,74 +142,92 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   const uint32_t tbase = *tmem_base_smem;
 
   if (warp == 0) {
-    // ================= TMA producer
-    if (lane == 0) {
+    // ================= TMA producer (whole warp converged; one elected lane issues)
+    const bool leader = elect_one();
+    if (leader) {
       tma_prefetch_desc(&mA_hi);
       tma_prefetch_desc(&mB_hi);
       tma_prefetch_desc(&mW_hi);
-      int it = 0;
-      for (int q = 0; q < count; ++q) {
-        int64_t tt64;
-        int st;
-        sc.unit(q, tt64, st);
-        const int tt = (int)tt64;
-        {
-          const int slot = q & 1;
-          const uint32_t use = (uint32_t)(q >> 1);
-          mbar_wait(&wempty[slot], (use & 1) ^ 1);
-          uint8_t* ws = smem + TcSmem::kW0 + slot * TcSmem::w_slot_bytes(RC);
+    }
+    int it = 0;
+    for (int q = 0; q < count; ++q) {
+      int64_t tt64;
+      int st;
+      sc.unit(q, tt64, st);
+      const int tt = (int)tt64;
+      {
+        const int slot = q & 1;
+        const uint32_t use = (uint32_t)(q >> 1);
+        mbar_wait(&wempty[slot], (use & 1) ^ 1);
+        uint8_t* ws = smem + TcSmem::kW0 + slot * TcSmem::w_slot_bytes(RC);
+        if (leader) {
           mbar_arrive_expect_tx(&wfull[slot], 2 * TcSmem::wslot(RC) + 512);
           tma_load_3d(ws, &mW_hi, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
           tma_load_3d(ws + TcSmem::wslot(RC), &mW_lo, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
           bulk_load(ws + 2 * TcSmem::wslot(RC), args.na + (int64_t)st * kTcTileS, 512, &wfull[slot]);
         }
-        for (int kc = 0; kc < n_kc; ++kc, ++it) {
-          const int s = it % kStages;
-          const uint32_t use = (uint32_t)(it / kStages);
-          mbar_wait(&empty[s], (use & 1) ^ 1);
-          uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
+        __syncwarp();
+      }
+      for (int kc = 0; kc < n_kc; ++kc, ++it) {
+        const int s = it % kStages;
+        const uint32_t use = (uint32_t)(it / kStages);
+        mbar_wait(&empty[s], (use & 1) ^ 1);
+        uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
+        if (leader) {
           mbar_arrive_expect_tx(&full[s], kStageBytes);
           tma_load_2d(sp, &mA_hi, kc * kTcKC, tt * kTcTileT, &full[s]);
           tma_load_2d(sp + kChunkBytes, &mA_lo, kc * kTcKC, tt * kTcTileT, &full[s]);
           tma_load_2d(sp + 2 * kChunkBytes, &mB_hi, kc * kTcKC, st * kTcTileS, &full[s]);
           tma_load_2d(sp + 3 * kChunkBytes, &mB_lo, kc * kTcKC, st * kTcTileS, &full[s]);
         }
+        __syncwarp();
       }
     }
-    __syncwarp();
   } else if (warp == 1) {
-    // ================= MMA issuer
-    if (lane == 0) {
+    // ================= MMA issuer (whole warp converged; one elected lane issues)
+    const bool leader = elect_one();
+    {
       const uint32_t idS = idesc_tf32(128, kTcTileS);
       const uint32_t idV = idesc_tf32(128, RC);
       int it = 0;
-      auto v_mma = [&](int p) {
+      // V(p, hh) += P(p)[:, 64hh : 64hh+64] . W(p)[64hh : 64hh+64, :] on the tensor
+      // cores, A = P read from TMEM.  Issued as soon as the epilogue has
+      // written that source half of P (pready), so it overlaps the epilogue.
+      auto v_mma = [&](int p, int hh) {
         int64_t tp;
         int sp_;
         sc.unit(p, tp, sp_);
-        const bool first = sc.first_in_block(p, sp_);
+        const bool first = (hh == 0) && sc.first_in_block(p, sp_);
         const int bp = p & 1;
         const uint32_t use = (uint32_t)(p >> 1);
-        mbar_wait(&pready[bp], use & 1);
-        mbar_wait(&wfull[p & 1], use & 1);
+        mbar_wait(&pready[bp * 2 + hh], use & 1);
+        if (hh == 0) mbar_wait(&wfull[p & 1], use & 1);
         tc_fence_after();
         uint8_t* ws = smem + TcSmem::kW0 + (p & 1) * TcSmem::w_slot_bytes(RC);
-        const uint32_t colP = bp ? kColS1 : kColS0;
+        const uint32_t colP = (bp ? kColS1 : kColS0) + 64 * hh;
+        const uint32_t colL = kColPlo + 64 * hh;
         // products: P_lo.W_hi, P_hi.W_lo, P_hi.W_hi (small terms first)
         const int nprod = args.three ? 3 : 1;
         bool acc = !first;
         for (int pr = 3 - nprod; pr < 3; ++pr) {
-          const uint32_t aCol = (pr == 0) ? kColPlo : colP;
+          const uint32_t aCol = (pr == 0) ? colL : colP;
           const uint8_t* wB = ws + ((pr == 1) ? TcSmem::wslot(RC) : 0u);
-#pragma unroll 4
-          for (int ks = 0; ks < kTcTileS / 8; ++ks) {
-            const uint64_t bd = sdesc_k_sw64(wB + (ks >> 1) * (RC * 64) + (ks & 1) * 32);
-            mma_tf32_ts(tbase + kColV, tbase + aCol + ks * 8, bd, idV, acc ? 1u : 0u);
+#pragma unroll
+          const uint64_t bd0 = sdesc_k_sw64(wB);
+          for (int ks = 0; ks < 8; ++ks) {
+            const int kk = 8 * hh + ks;  // K step (8 sources) within the tile
+            // descriptor start address advances in 16-byte units
+            const uint64_t bd = bd0 + (uint64_t)(((kk >> 1) * (RC * 64) + (kk & 1) * 32) >> 4);
+            if (leader) mma_tf32_ts(tbase + kColV, tbase + aCol + ks * 8, bd, idV, acc ? 1u : 0u);
             acc = true;
           }
         }
-        tc_commit(vdone);
-        tc_commit(&wempty[p & 1]);
+        __syncwarp();
+        if (leader) {
+          tc_commit(&vdone[hh]);
+          if (hh == 1) tc_commit(&wempty[p & 1]);
+        }
+        __syncwarp();
       };
       for (int q = 0; q < count; ++q) {
         const int bq = q & 1;
@@ -219,33 +238,45 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           mbar_wait(&full[s], use & 1);
           tc_fence_after();
           uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
+          const uint64_t d0 = sdesc_k_sw64(sp);
 #pragma unroll
           for (int ks = 0; ks < kTcKC / 8; ++ks) {
-            const uint64_t aH = sdesc_k_sw64(sp + ks * 32);
-            const uint64_t aL = sdesc_k_sw64(sp + kChunkBytes + ks * 32);
-            const uint64_t bH = sdesc_k_sw64(sp + 2 * kChunkBytes + ks * 32);
-            const uint64_t bL = sdesc_k_sw64(sp + 3 * kChunkBytes + ks * 32);
+            const uint64_t aH = d0 + (uint64_t)((ks * 32) >> 4);
+            const uint64_t aL = d0 + (uint64_t)((kChunkBytes + ks * 32) >> 4);
+            const uint64_t bH = d0 + (uint64_t)((2 * kChunkBytes + ks * 32) >> 4);
+            const uint64_t bL = d0 + (uint64_t)((3 * kChunkBytes + ks * 32) >> 4);
             const uint32_t acc0 = (kc > 0 || ks > 0) ? 1u : 0u;
-            if (args.three) {
-              mma_tf32_ss(dS, aL, bH, idS, acc0);
-              mma_tf32_ss(dS, aH, bL, idS, 1u);
-              mma_tf32_ss(dS, aH, bH, idS, 1u);
-            } else {
-              mma_tf32_ss(dS, aH, bH, idS, acc0);
+            if (leader) {
+              if (args.three) {
+                mma_tf32_ss(dS, aL, bH, idS, acc0);
+                mma_tf32_ss(dS, aH, bL, idS, 1u);
+                mma_tf32_ss(dS, aH, bH, idS, 1u);
+              } else {
+                mma_tf32_ss(dS, aH, bH, idS, acc0);
+              }
             }
           }
-          tc_commit(&empty[s]);
+          __syncwarp();
+          if (leader) tc_commit(&empty[s]);
+          __syncwarp();
         }
-        tc_commit(&sfull[bq]);
-        if (q > 0) v_mma(q - 1);
+        if (leader) tc_commit(&sfull[bq]);
+        __syncwarp();
+        if (q > 0) {
+          v_mma(q - 1, 0);
+          v_mma(q - 1, 1);
+        }
       }
-      if (count > 0) v_mma(count - 1);
+      if (count > 0) {
+        v_mma(count - 1, 0);
+        v_mma(count - 1, 1);
+      }
     }
     __syncwarp();
   } else if (warp >= 4) {
-    // ================= epilogue (8 warps: lane group g, column half h)
+    // ================= epilogue (8 warps: lane group g, sub-split h)
     const int g = warp & 3;               // TMEM lanes 32g..32g+31
-    const int h = (warp - 4) >> 2;        // columns 64h..64h+63 of the tile
+    const int h = (warp - 4) >> 2;        // columns 64hh+32h..+31 of each source half hh; V columns h*RC/2..
     const int row = 32 * g + lane;        // target row within the tile
     const uint32_t lane_off = (uint32_t)(32 * g) << 16;
     // each epilogue thread owns V columns [h*HC, (h+1)*HC) of its target row
@@ -343,17 +374,26 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       mbar_wait(&sfull[bq], use & 1);
       tc_fence_after();
       if (q > 0) {
-        mbar_wait(vdone, (uint32_t)((q - 1) & 1));  // V(q-1) done: P_lo free, V readable
-        tc_fence_after();
-        v_collect(q - 1);
+        int64_t tp;
+        int sp_;
+        sc.unit(q - 1, tp, sp_);
+        if ((sp_ + 1 == n_s) || ((sp_ + 1) % kFlush == 0)) {  // block end: V(q-1) must be read now
+          mbar_wait(&vdone[1], (uint32_t)((q - 1) & 1));
+          tc_fence_after();
+          v_collect(q - 1);
+        }
       }
       if (q == seg_q) nbj = __ldg(args.nb + tt * kTcTileT + row);  // new segment: this target tile's norms
       const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC) +
                                                        2 * TcSmem::wslot(RC));
       const uint32_t colS = bq ? kColS1 : kColS0;
 #pragma unroll 1
-      for (int cb = 0; cb < 2; ++cb) {
-        const int c0 = 64 * h + 32 * cb;
+      for (int hh = 0; hh < 2; ++hh) {
+        if (q > 0) {  // V(q-1, hh) has consumed this source half's P_lo buffer
+          mbar_wait(&vdone[hh], (uint32_t)((q - 1) & 1));
+          tc_fence_after();
+        }
+        const int c0 = 64 * hh + 32 * h;
         uint32_t sv[32];
         tmem_ld32(tbase + lane_off + colS + c0, sv);
         tmem_wait_ld();
@@ -365,22 +405,22 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
             const float t = fminf(__uint_as_float(sv[i + e]) + (nav[e] + nbj), 0.f);
-            const float p = ex2_approx(t);
-            const float ph = to_tf32(p);
-            hi[i + e] = __float_as_uint(ph);
-            lo[i + e] = __float_as_uint(to_tf32(p - ph));
+            const float p = ex2_approx(t);                       // in [0, 1]
+            const uint32_t hb = (__float_as_uint(p) + 0x1000u) & 0xFFFFE000u;  // TF32 round-to-nearest
+            hi[i + e] = hb;
+            lo[i + e] = __float_as_uint(p - __uint_as_float(hb));  // exact remainder; the MMA reads its TF32 bits
           }
         }
         tmem_st32(tbase + lane_off + colS + c0, hi);
         if (args.three) tmem_st32(tbase + lane_off + kColPlo + c0, lo);
+        tmem_wait_st();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&pready[bq * 2 + hh]);
       }
-      tmem_wait_st();
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&pready[bq]);
     }
     if (count > 0) {
-      mbar_wait(vdone, (uint32_t)((count - 1) & 1));
+      mbar_wait(&vdone[1], (uint32_t)((count - 1) & 1));
       tc_fence_after();
       v_collect(count - 1);
     }
