@@ -122,6 +122,7 @@ struct ks_ctx {
   DBuf<float> src_hi, src_lo, na, wt_hi, wt_lo;
   DBuf<float> tgt_hi, tgt_lo, nb;
   int r_pad = 16;
+  int tc_aug = 0;  // norms folded into the contraction as 2 extra K columns
   CUtensorMap tmB_hi, tmB_lo;
   DBuf<float> mu;         // [k_pad]
   DBuf<double> mean_part; // [nparts][K]
@@ -297,11 +298,19 @@ ks_status encode_wt(CUtensorMap* map, const float* base, int64_t m_pad, int r_pa
   return KS_OK;
 }
 
-int tc_k_pad(int K) { return (int)round_up(K, ks::kTcKC); }
+// Fold the norms into the MMA (two extra K columns) when that costs no extra K chunk.
+// KS_TC_AUG=0/1 overrides (measurement knob).
+int tc_aug(int K) {
+  const char* e = getenv("KS_TC_AUG");
+  if (e && (e[0] == '0' || e[0] == '1')) return e[0] - '0';
+  return (round_up(K + 2, ks::kTcKC) == round_up(K, ks::kTcKC)) ? 1 : 0;  // measured: an extra chunk costs more than it saves
+}
+int tc_k_pad(int K) { return (int)round_up(K + 2 * tc_aug(K), ks::kTcKC); }
 
 ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M, int R) {
   const int K = ctx->K;
   const int k_pad = tc_k_pad(K);
+  const int aug = tc_aug(K);
   const int64_t m_pad = round_up(M > 0 ? M : 1, ks::kTcTileS);
   const int r_pad = (int)round_up(R, 16);
   cudaStream_t st = ctx->stream;
@@ -318,8 +327,8 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(ctx->mean_part.reserve((size_t)nparts * K, st, false), "allocate mean partials");
   KS_CUDA(ks::launch_source_mean(alpha, M, K, k_pad, ctx->mean_part.p, nparts, ctx->mu.p, st), "source mean");
   ctx->launches += (M > 0) ? 2 : 1;
-  KS_CUDA(ks::launch_prep_tc_sources(alpha, W, M, m_pad, K, k_pad, R, r_pad, ctx->mu.p, ctx->c, ctx->src_hi.p,
-                                     ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p, st),
+  KS_CUDA(ks::launch_prep_tc_sources(alpha, W, M, m_pad, K, k_pad, R, r_pad, ctx->mu.p, ctx->c, aug,
+                                     ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p, st),
           "source prep (TC)");
   ctx->launches += 1;
   ks_status s = encode_2d_sw64(&ctx->tmB_hi, ctx->src_hi.p, k_pad, m_pad, ks::kTcTileS);
@@ -329,6 +338,7 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   ctx->k_pad = k_pad;
   ctx->m_pad = m_pad;
   ctx->r_pad = r_pad;
+  ctx->tc_aug = aug;
   return KS_OK;
 }
 
@@ -340,8 +350,8 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   KS_CUDA(ctx->tgt_hi.reserve(ntg, st, false), "allocate target hi");
   KS_CUDA(ctx->tgt_lo.reserve(ntg, st, false), "allocate target lo");
   KS_CUDA(ctx->nb.reserve((size_t)n_pad, st, false), "allocate target norms");
-  KS_CUDA(ks::launch_prep_tc_targets(beta, N, n_pad, ctx->K, k_pad, ctx->mu.p, ctx->c, ctx->tgt_hi.p, ctx->tgt_lo.p,
-                                     ctx->nb.p, st),
+  KS_CUDA(ks::launch_prep_tc_targets(beta, N, n_pad, ctx->K, k_pad, ctx->mu.p, ctx->c, ctx->tc_aug, ctx->tgt_hi.p,
+                                     ctx->tgt_lo.p, ctx->nb.p, st),
           "target prep (TC)");
   ctx->launches += 1;
   CUtensorMap maps[6];
@@ -367,6 +377,11 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.k_pad = k_pad;
   a.R = ctx->R;
   a.three = (ctx->prec_eff == KS_PREC_TF32) ? 0 : 1;
+  a.aug = ctx->tc_aug;
+  {
+    const char* e = getenv("KS_TC_DEBUG_SKIP_V");
+    a.dbg_skip_v = (e && e[0] == '1') ? 1 : 0;
+  }
   a.na = ctx->na.p;
   a.nb = ctx->nb.p;
   a.V = V;

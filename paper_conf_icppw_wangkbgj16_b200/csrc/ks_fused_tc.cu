@@ -86,6 +86,32 @@ struct Sched {
   }
 };
 
+// Sequential walk over a CTA's units without divisions in the loop.
+struct UnitIt {
+  int q;
+  int st;
+  int64_t tt;
+};
+__device__ __forceinline__ UnitIt unit_begin(const Sched& s) {
+  UnitIt u;
+  u.q = 0;
+  if (s.qw > 0) { u.tt = s.b; u.st = 0; }
+  else { u.tt = s.rem_t0 + s.v0 / s.n_s; u.st = (int)(s.v0 % s.n_s); }
+  return u;
+}
+__device__ __forceinline__ void unit_next(const Sched& s, UnitIt& u) {
+  ++u.q;
+  if (u.q < s.qw) {
+    if (++u.st == s.n_s) { u.st = 0; u.tt += s.G; }
+  } else if (u.q == s.qw) {
+    u.tt = s.rem_t0 + s.v0 / s.n_s;
+    u.st = (int)(s.v0 % s.n_s);
+  } else if (++u.st == s.n_s) {
+    u.st = 0;
+    ++u.tt;
+  }
+}
+
 }  // namespace
 
 template <int RC, int kStages>
@@ -95,6 +121,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
                        const __grid_constant__ CUtensorMap mW_hi, const __grid_constant__ CUtensorMap mW_lo,
                        const TcArgs args) {
   using TcSmem = TcSmemT<kStages>;
+  constexpr int EW = kTcEpiWarps;        // epilogue warps
+  constexpr int SUB = EW / 4;            // epilogue warps per TMEM lane group
+  constexpr int CB = 64 / SUB;           // columns per warp per source half
+  constexpr int HC = RC / SUB;           // V columns per epilogue thread
   extern __shared__ __align__(1024) uint8_t smem[];
   if ((smem_u32(smem) & 1023u) != 0u) __trap();  // SWIZZLE_64B atoms and descriptors assume 1 KB alignment
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + TcSmem::bar_off(RC));
@@ -132,7 +162,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       mbar_init(&sfull[i], 1);
       mbar_init(&vdone[i], 1);
     }
-    for (int i = 0; i < 4; ++i) mbar_init(&pready[i], 8);  // 8 epilogue warps
+    for (int i = 0; i < 4; ++i) mbar_init(&pready[i], EW);  // one arrival per epilogue warp
     fence_mbar_init();
   }
   if (warp == 2) tmem_alloc(tmem_base_smem, 512);
@@ -150,11 +180,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       tma_prefetch_desc(&mW_hi);
     }
     int it = 0;
-    for (int q = 0; q < count; ++q) {
-      int64_t tt64;
-      int st;
-      sc.unit(q, tt64, st);
-      const int tt = (int)tt64;
+    UnitIt cu = unit_begin(sc);
+    for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
+      const int tt = (int)cu.tt, st = cu.st;
       {
         const int slot = q & 1;
         const uint32_t use = (uint32_t)(q >> 1);
@@ -186,133 +214,119 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   } else if (warp == 1) {
     // ================= MMA issuer (whole warp converged; one elected lane issues)
     const bool leader = elect_one();
-    {
-      const uint32_t idS = idesc_tf32(128, kTcTileS);
-      const uint32_t idV = idesc_tf32(128, RC);
-      int it = 0;
-      // V(p, hh) += P(p)[:, 64hh : 64hh+64] . W(p)[64hh : 64hh+64, :] on the tensor
-      // cores, A = P read from TMEM.  Issued as soon as the epilogue has
-      // written that source half of P (pready), so it overlaps the epilogue.
-      auto v_mma = [&](int p, int hh) {
-        int64_t tp;
-        int sp_;
-        sc.unit(p, tp, sp_);
-        const bool first = (hh == 0) && sc.first_in_block(p, sp_);
-        const int bp = p & 1;
-        const uint32_t use = (uint32_t)(p >> 1);
-        mbar_wait(&pready[bp * 2 + hh], use & 1);
-        if (hh == 0) mbar_wait(&wfull[p & 1], use & 1);
+    const uint32_t idS = idesc_tf32(128, kTcTileS);
+    const uint32_t idV = idesc_tf32(128, RC);
+    const int nprod = args.three ? 3 : 1;
+    const bool skip_v = args.dbg_skip_v != 0;
+    int it = 0;
+    // V(p, hh) += P(p)[:, 64hh : 64hh+64] . W(p)[64hh : 64hh+64, :] on the tensor
+    // cores, A = P read from TMEM.  Issued as soon as the epilogue has
+    // written that source half of P (pready), so it overlaps the epilogue.
+    auto v_mma = [&](int p, int stp, int hh) {
+      const bool first = (hh == 0) && sc.first_in_block(p, stp);
+      const int bp = p & 1;
+      const uint32_t use = (uint32_t)(p >> 1);
+      mbar_wait(&pready[bp * 2 + hh], use & 1);
+      if (hh == 0) mbar_wait(&wfull[p & 1], use & 1);
+      tc_fence_after();
+      uint8_t* ws = smem + TcSmem::kW0 + (p & 1) * TcSmem::w_slot_bytes(RC);
+      const uint32_t colP = (bp ? kColS1 : kColS0) + 64 * hh;
+      const uint32_t colL = kColPlo + 64 * hh;
+      bool acc = !first;
+      // products: P_lo.W_hi, P_hi.W_lo, P_hi.W_hi (small terms first)
+      for (int pr = 3 - nprod; pr < 3 && !skip_v; ++pr) {
+        const uint32_t aCol = (pr == 0) ? colL : colP;
+        const uint64_t bd0 = sdesc_k_sw64(ws + ((pr == 1) ? TcSmem::wslot(RC) : 0u));
+#pragma unroll
+        for (int ks = 0; ks < 8; ++ks) {
+          const int kk = 8 * hh + ks;  // K step (8 sources) within the tile
+          // descriptor start address advances in 16-byte units
+          const uint64_t bd = bd0 + (uint64_t)(((kk >> 1) * (RC * 64) + (kk & 1) * 32) >> 4);
+          if (leader) mma_tf32_ts(tbase + kColV, tbase + aCol + ks * 8, bd, idV, acc ? 1u : 0u);
+          acc = true;
+        }
+      }
+      __syncwarp();
+      if (leader) {
+        tc_commit(&vdone[hh]);
+        if (hh == 1) tc_commit(&wempty[p & 1]);
+      }
+      __syncwarp();
+    };
+    UnitIt cu = unit_begin(sc);
+    int prev_st = 0;
+    for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
+      const int bq = q & 1;
+      const uint32_t dS = tbase + (bq ? kColS1 : kColS0);
+      for (int kc = 0; kc < n_kc; ++kc, ++it) {
+        const int s = it % kStages;
+        const uint32_t use = (uint32_t)(it / kStages);
+        mbar_wait(&full[s], use & 1);
         tc_fence_after();
-        uint8_t* ws = smem + TcSmem::kW0 + (p & 1) * TcSmem::w_slot_bytes(RC);
-        const uint32_t colP = (bp ? kColS1 : kColS0) + 64 * hh;
-        const uint32_t colL = kColPlo + 64 * hh;
-        // products: P_lo.W_hi, P_hi.W_lo, P_hi.W_hi (small terms first)
-        const int nprod = args.three ? 3 : 1;
-        bool acc = !first;
-        for (int pr = 3 - nprod; pr < 3; ++pr) {
-          const uint32_t aCol = (pr == 0) ? colL : colP;
-          const uint8_t* wB = ws + ((pr == 1) ? TcSmem::wslot(RC) : 0u);
+        uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
+        const uint64_t d0 = sdesc_k_sw64(sp);
 #pragma unroll
-          const uint64_t bd0 = sdesc_k_sw64(wB);
-          for (int ks = 0; ks < 8; ++ks) {
-            const int kk = 8 * hh + ks;  // K step (8 sources) within the tile
-            // descriptor start address advances in 16-byte units
-            const uint64_t bd = bd0 + (uint64_t)(((kk >> 1) * (RC * 64) + (kk & 1) * 32) >> 4);
-            if (leader) mma_tf32_ts(tbase + kColV, tbase + aCol + ks * 8, bd, idV, acc ? 1u : 0u);
-            acc = true;
-          }
-        }
-        __syncwarp();
-        if (leader) {
-          tc_commit(&vdone[hh]);
-          if (hh == 1) tc_commit(&wempty[p & 1]);
-        }
-        __syncwarp();
-      };
-      for (int q = 0; q < count; ++q) {
-        const int bq = q & 1;
-        const uint32_t dS = tbase + (bq ? kColS1 : kColS0);
-        for (int kc = 0; kc < n_kc; ++kc, ++it) {
-          const int s = it % kStages;
-          const uint32_t use = (uint32_t)(it / kStages);
-          mbar_wait(&full[s], use & 1);
-          tc_fence_after();
-          uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
-          const uint64_t d0 = sdesc_k_sw64(sp);
-#pragma unroll
-          for (int ks = 0; ks < kTcKC / 8; ++ks) {
-            const uint64_t aH = d0 + (uint64_t)((ks * 32) >> 4);
-            const uint64_t aL = d0 + (uint64_t)((kChunkBytes + ks * 32) >> 4);
-            const uint64_t bH = d0 + (uint64_t)((2 * kChunkBytes + ks * 32) >> 4);
-            const uint64_t bL = d0 + (uint64_t)((3 * kChunkBytes + ks * 32) >> 4);
-            const uint32_t acc0 = (kc > 0 || ks > 0) ? 1u : 0u;
-            if (leader) {
-              if (args.three) {
-                mma_tf32_ss(dS, aL, bH, idS, acc0);
-                mma_tf32_ss(dS, aH, bL, idS, 1u);
-                mma_tf32_ss(dS, aH, bH, idS, 1u);
-              } else {
-                mma_tf32_ss(dS, aH, bH, idS, acc0);
-              }
+        for (int ks = 0; ks < kTcKC / 8; ++ks) {
+          const uint64_t aH = d0 + (uint64_t)((ks * 32) >> 4);
+          const uint64_t aL = d0 + (uint64_t)((kChunkBytes + ks * 32) >> 4);
+          const uint64_t bH = d0 + (uint64_t)((2 * kChunkBytes + ks * 32) >> 4);
+          const uint64_t bL = d0 + (uint64_t)((3 * kChunkBytes + ks * 32) >> 4);
+          const uint32_t acc0 = (kc > 0 || ks > 0) ? 1u : 0u;
+          if (leader) {
+            if (args.three) {
+              mma_tf32_ss(dS, aL, bH, idS, acc0);
+              mma_tf32_ss(dS, aH, bL, idS, 1u);
+              mma_tf32_ss(dS, aH, bH, idS, 1u);
+            } else {
+              mma_tf32_ss(dS, aH, bH, idS, acc0);
             }
           }
-          __syncwarp();
-          if (leader) tc_commit(&empty[s]);
-          __syncwarp();
         }
-        if (leader) tc_commit(&sfull[bq]);
         __syncwarp();
-        if (q > 0) {
-          v_mma(q - 1, 0);
-          v_mma(q - 1, 1);
-        }
+        if (leader) tc_commit(&empty[s]);
+        __syncwarp();
       }
-      if (count > 0) {
-        v_mma(count - 1, 0);
-        v_mma(count - 1, 1);
+      if (leader) tc_commit(&sfull[bq]);
+      __syncwarp();
+      if (q > 0) {
+        v_mma(q - 1, prev_st, 0);
+        v_mma(q - 1, prev_st, 1);
       }
+      prev_st = cu.st;
     }
-    __syncwarp();
+    if (count > 0) {
+      v_mma(count - 1, prev_st, 0);
+      v_mma(count - 1, prev_st, 1);
+    }
   } else if (warp >= 4) {
-    // ================= epilogue (8 warps: lane group g, sub-split h)
-    const int g = warp & 3;               // TMEM lanes 32g..32g+31
-    const int h = (warp - 4) >> 2;        // columns 64hh+32h..+31 of each source half hh; V columns h*RC/2..
+    // ================= epilogue (EW warps: TMEM lane group g, sub-split h)
+    const int ew = warp - 4;
+    const int g = ew & 3;                 // TMEM lanes 32g..32g+31
+    const int h = ew >> 2;                // columns 64hh + CB h .. + CB-1 of each source half hh
     const int row = 32 * g + lane;        // target row within the tile
     const uint32_t lane_off = (uint32_t)(32 * g) << 16;
-    // each epilogue thread owns V columns [h*HC, (h+1)*HC) of its target row
-    constexpr int HC = RC / 2;
-    const int rbase = h * HC;
+    const int rbase = h * HC;             // V columns of this thread
     double vacc[HC];
 #pragma unroll
     for (int r = 0; r < HC; ++r) vacc[r] = 0.0;
     float nbj = 0.f;
-    int seg_q = 0;  // first local unit of the current segment
+    int seg_q = 0;                        // first local unit of the current segment
+    int seg_st0 = 0;                      // its source tile
 
     // read the V accumulator (unit p finished) into FP64 registers; at the end
     // of a segment write V / partial.
-    auto v_collect = [&](int p) {
-      int64_t tt;
-      int spp;
-      sc.unit(p, tt, spp);
-      const bool last_in_block = (p == count - 1) || (spp + 1 == n_s) || ((spp + 1) % kFlush == 0);
+    auto v_collect = [&](int p, int64_t tt, int spp) {
       const bool seg_end = (p == count - 1) || (spp + 1 == n_s);
-      if (last_in_block) {
+      {
         uint32_t v[HC];
-        if constexpr (HC == 16) {
-          tmem_ld16(tbase + lane_off + kColV + rbase, v);
-        } else {
-          tmem_ld8(tbase + lane_off + kColV + rbase, v);
-        }
+        tmem_ldn<HC>(tbase + lane_off + kColV + rbase, v);
         tmem_wait_ld();
 #pragma unroll
         for (int r = 0; r < HC; ++r) vacc[r] += (double)__uint_as_float(v[r]);
       }
       if (seg_end) {
-        int64_t t0;
-        int st0;
-        sc.unit(seg_q, t0, st0);
         const int seg_len = p - seg_q + 1;
-        const bool whole = (st0 == 0) && (seg_len == n_s);
+        const bool whole = (seg_st0 == 0) && (seg_len == n_s);
         const int64_t grow = tt * kTcTileT + row;
         if (whole) {
           if (grow < args.N) {
@@ -329,7 +343,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 #pragma unroll
           for (int r = 0; r < HC; ++r) pp[r] = (float)vacc[r];
           __threadfence();
-          named_bar_sync(1, 256);
+          named_bar_sync(1, 32 * EW);
           const int64_t b_first = sk_owner(tr * n_s, sc.Urem, sc.Gr);
           const int64_t b_last = sk_owner(tr * n_s + n_s - 1, sc.Urem, sc.Gr);
           if (row == 0 && h == 0) {
@@ -338,7 +352,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
             if (last) args.counters[tt] = 0;
             *flag = last;
           }
-          named_bar_sync(1, 256);
+          named_bar_sync(1, 32 * EW);
           if (*flag) {
             __threadfence();
             float sum[HC];
@@ -356,7 +370,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
                 if (rbase + r < args.r_valid) args.V[grow * args.R + args.r_off + rbase + r] = sum[r];
             }
           }
-          named_bar_sync(1, 256);  // flag reuse
+          named_bar_sync(1, 32 * EW);  // flag reuse
         }
 #pragma unroll
         for (int r = 0; r < HC; ++r) vacc[r] = 0.0;
@@ -364,26 +378,25 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       }
     };
 
-    for (int q = 0; q < count; ++q) {
-      int64_t tt;
-      int stq;
-      sc.unit(q, tt, stq);
+    UnitIt cu = unit_begin(sc);
+    int64_t prev_tt = 0;
+    int prev_st = 0;
+    for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
       const int bq = q & 1;
       const uint32_t use = (uint32_t)(q >> 1);
       mbar_wait(&wfull[q & 1], use & 1);
       mbar_wait(&sfull[bq], use & 1);
       tc_fence_after();
-      if (q > 0) {
-        int64_t tp;
-        int sp_;
-        sc.unit(q - 1, tp, sp_);
-        if ((sp_ + 1 == n_s) || ((sp_ + 1) % kFlush == 0)) {  // block end: V(q-1) must be read now
-          mbar_wait(&vdone[1], (uint32_t)((q - 1) & 1));
-          tc_fence_after();
-          v_collect(q - 1);
-        }
+      if (q > 0 && ((prev_st + 1 == n_s) || ((prev_st + 1) % kFlush == 0))) {
+        // block end: V(q-1) complete, fold it into FP64 registers (and write at segment end)
+        mbar_wait(&vdone[1], (uint32_t)((q - 1) & 1));
+        tc_fence_after();
+        v_collect(q - 1, prev_tt, prev_st);
       }
-      if (q == seg_q) nbj = __ldg(args.nb + tt * kTcTileT + row);  // new segment: this target tile's norms
+      if (q == seg_q) {  // new segment: this target tile's norms
+        seg_st0 = cu.st;
+        if (!args.aug) nbj = __ldg(args.nb + cu.tt * kTcTileT + row);
+      }
       const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC) +
                                                        2 * TcSmem::wslot(RC));
       const uint32_t colS = bq ? kColS1 : kColS0;
@@ -393,36 +406,42 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           mbar_wait(&vdone[hh], (uint32_t)((q - 1) & 1));
           tc_fence_after();
         }
-        const int c0 = 64 * hh + 32 * h;
-        uint32_t sv[32];
-        tmem_ld32(tbase + lane_off + colS + c0, sv);
+        const int c0 = 64 * hh + CB * h;
+        uint32_t sv[CB];
+        tmem_ldn<CB>(tbase + lane_off + colS + c0, sv);
         tmem_wait_ld();
-        uint32_t hi[32], lo[32];
+        uint32_t hi[CB], lo[CB];
 #pragma unroll
-        for (int i = 0; i < 32; i += 4) {
-          const float4 na4 = *reinterpret_cast<const float4*>(nas + c0 + i);
-          const float nav[4] = {na4.x, na4.y, na4.z, na4.w};
+        for (int i = 0; i < CB; i += 4) {
+          float nav[4] = {0.f, 0.f, 0.f, 0.f};
+          if (!args.aug) {
+            const float4 na4 = *reinterpret_cast<const float4*>(nas + c0 + i);
+            nav[0] = na4.x + nbj; nav[1] = na4.y + nbj; nav[2] = na4.z + nbj; nav[3] = na4.w + nbj;
+          }
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
-            const float t = fminf(__uint_as_float(sv[i + e]) + (nav[e] + nbj), 0.f);
-            const float p = ex2_approx(t);                       // in [0, 1]
+            // t = S + na_i + nb_j (norms already inside S when args.aug), clamp d^2 >= 0
+            const float t = fminf(__uint_as_float(sv[i + e]) + nav[e], 0.f);
+            const float p = ex2_approx(t);                                    // in [0, 1]
             const uint32_t hb = (__float_as_uint(p) + 0x1000u) & 0xFFFFE000u;  // TF32 round-to-nearest
             hi[i + e] = hb;
             lo[i + e] = __float_as_uint(p - __uint_as_float(hb));  // exact remainder; the MMA reads its TF32 bits
           }
         }
-        tmem_st32(tbase + lane_off + colS + c0, hi);
-        if (args.three) tmem_st32(tbase + lane_off + kColPlo + c0, lo);
+        tmem_stn<CB>(tbase + lane_off + colS + c0, hi);
+        if (args.three) tmem_stn<CB>(tbase + lane_off + kColPlo + c0, lo);
         tmem_wait_st();
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&pready[bq * 2 + hh]);
       }
+      prev_tt = cu.tt;
+      prev_st = cu.st;
     }
     if (count > 0) {
       mbar_wait(&vdone[1], (uint32_t)((count - 1) & 1));
       tc_fence_after();
-      v_collect(count - 1);
+      v_collect(count - 1, prev_tt, prev_st);
     }
   }
 
@@ -440,7 +459,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 // ---------------------------------------------------------------- prep (a1 / a2 for the TC path)
 __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const float* __restrict__ W, int64_t M,
                                        int64_t m_pad, int K, int k_pad, int R, int r_pad,
-                                       const float* __restrict__ mu, double c, float* __restrict__ src_hi,
+                                       const float* __restrict__ mu, double c, int aug, float* __restrict__ src_hi,
                                        float* __restrict__ src_lo, float* __restrict__ na,
                                        float* __restrict__ wt_hi, float* __restrict__ wt_lo) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -448,16 +467,26 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
   const bool live = i < M;
   const double c2 = 2.0 * c;
   double n = 0.0;
-  for (int d = 0; d < k_pad; ++d) {
-    float x = 0.f;
-    if (live && d < K) x = alpha[i * K + d] - mu[d];
+  for (int d = 0; d < K; ++d) {
+    const float x = live ? alpha[i * K + d] - mu[d] : 0.f;  // FP32 centring, same op as the target side
     n += (double)x * (double)x;
-    const float a = (float)(c2 * (double)x);
+  }
+  const float nai = live ? (float)(-c * n) : 0.f;
+  na[i] = nai;
+  for (int d = 0; d < k_pad; ++d) {
+    float a = 0.f;
+    if (d < K) {
+      const float x = live ? alpha[i * K + d] - mu[d] : 0.f;
+      a = (float)(c2 * (double)x);
+    } else if (aug && d == K) {
+      a = 1.f;   // multiplies nb_j of the target
+    } else if (aug && d == K + 1) {
+      a = nai;   // times 1 on the target side
+    }
     const float ah = to_tf32(a);
     src_hi[i * k_pad + d] = ah;
     src_lo[i * k_pad + d] = to_tf32(a - ah);
   }
-  na[i] = live ? (float)(-c * n) : 0.f;
   for (int r = 0; r < r_pad; ++r) {
     const float w = (live && r < R) ? W[i * R + r] : 0.f;
     const float wh = to_tf32(w);
@@ -467,39 +496,45 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
 }
 
 __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N, int64_t n_pad, int K, int k_pad,
-                                       const float* __restrict__ mu, double c, float* __restrict__ tgt_hi,
+                                       const float* __restrict__ mu, double c, int aug, float* __restrict__ tgt_hi,
                                        float* __restrict__ tgt_lo, float* __restrict__ nb) {
   const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (j >= n_pad) return;
   const bool live = j < N;
   double n = 0.0;
+  for (int d = 0; d < K; ++d) {
+    const float x = live ? beta[j * K + d] - mu[d] : 0.f;
+    n += (double)x * (double)x;
+  }
+  const float nbj = live ? (float)(-c * n) : 0.f;
+  nb[j] = nbj;
   for (int d = 0; d < k_pad; ++d) {
     float x = 0.f;
-    if (live && d < K) x = beta[j * K + d] - mu[d];
-    n += (double)x * (double)x;
+    if (d < K) x = live ? beta[j * K + d] - mu[d] : 0.f;
+    else if (aug && d == K) x = nbj;
+    else if (aug && d == K + 1) x = 1.f;
     const float xh = to_tf32(x);
     tgt_hi[j * k_pad + d] = xh;
     tgt_lo[j * k_pad + d] = to_tf32(x - xh);
   }
-  nb[j] = live ? (float)(-c * n) : 0.f;
 }
 
 cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
-                                   int R, int r_pad, const float* mu, double c, float* src_hi, float* src_lo,
-                                   float* na, float* wt_hi, float* wt_lo, cudaStream_t st) {
+                                   int R, int r_pad, const float* mu, double c, int aug, float* src_hi,
+                                   float* src_lo, float* na, float* wt_hi, float* wt_lo, cudaStream_t st) {
   if (m_pad == 0) return cudaSuccess;
   const int bs = 128;
-  prep_tc_sources_kernel<<<(unsigned)((m_pad + bs - 1) / bs), bs, 0, st>>>(alpha, W, M, m_pad, K, k_pad, R, r_pad, mu,
-                                                                          c, src_hi, src_lo, na, wt_hi, wt_lo);
+  prep_tc_sources_kernel<<<(unsigned)((m_pad + bs - 1) / bs), bs, 0, st>>>(
+      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, src_hi, src_lo, na, wt_hi, wt_lo);
   return cudaGetLastError();
 }
 
 cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
-                                   double c, float* tgt_hi, float* tgt_lo, float* nb, cudaStream_t st) {
+                                   double c, int aug, float* tgt_hi, float* tgt_lo, float* nb, cudaStream_t st) {
   if (n_pad == 0) return cudaSuccess;
   const int bs = 128;
-  prep_tc_targets_kernel<<<(unsigned)((n_pad + bs - 1) / bs), bs, 0, st>>>(beta, N, n_pad, K, k_pad, mu, c, tgt_hi,
-                                                                          tgt_lo, nb);
+  prep_tc_targets_kernel<<<(unsigned)((n_pad + bs - 1) / bs), bs, 0, st>>>(beta, N, n_pad, K, k_pad, mu, c, aug,
+                                                                          tgt_hi, tgt_lo, nb);
   return cudaGetLastError();
 }
 

@@ -60,7 +60,8 @@ namespace ks {
 constexpr int kTcTileT = 128;  // targets per tile = MMA M = TMEM lanes
 constexpr int kTcTileS = 128;  // sources per tile = N of the S MMA = K of the V MMA
 constexpr int kTcKC = 16;      // K floats per pipeline stage (64-byte rows, SWIZZLE_64B)
-constexpr int kTcThreads = 384;  // warp 0 TMA, 1 MMA, 2 TMEM alloc, 3 idle, 4..11 epilogue
+constexpr int kTcEpiWarps = 16;  // epilogue warps (4 per TMEM lane group)
+constexpr int kTcThreads = 128 + 32 * kTcEpiWarps;  // warp 0 TMA, 1 MMA, 2 TMEM alloc, 3 idle, 4.. epilogue
 
 struct TcArgs {
   int64_t N;            // targets
@@ -70,6 +71,8 @@ struct TcArgs {
   int r_off;            // first weight column of this launch
   int R;                // row stride of V
   int three;            // 1: 3xTF32 (hi.hi + hi.lo + lo.hi), 0: plain TF32 (hi.hi)
+  int aug;              // 1: norms folded into the contraction (2 extra K columns), epilogue adds nothing
+  int dbg_skip_v;       // measurement only (KS_TC_DEBUG_SKIP_V=1): do not issue the V MMAs (wrong results)
   const float* na;      // [m_pad]  -c ||alpha_hat||^2
   const float* nb;      // [n_pad]  -c ||beta_hat||^2
   float* V;             // [N][R]
@@ -81,12 +84,14 @@ struct TcArgs {
 
 // sources: src_hi/lo [m_pad][k_pad] = TF32 split of RN(2c (alpha - mu)),
 // na [m_pad], W^T split wt_hi/lo [r_pad][m_pad] (zero padded)
+// aug: columns K, K+1 hold (1, na_i) so that S already contains the norms
 cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
-                                   int R, int r_pad, const float* mu, double c, float* src_hi, float* src_lo,
-                                   float* na, float* wt_hi, float* wt_lo, cudaStream_t st);
+                                   int R, int r_pad, const float* mu, double c, int aug, float* src_hi,
+                                   float* src_lo, float* na, float* wt_hi, float* wt_lo, cudaStream_t st);
 // targets: tgt_hi/lo [n_pad][k_pad] = TF32 split of (beta - mu), nb [n_pad]
+// aug: columns K, K+1 hold (nb_j, 1)
 cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
-                                   double c, float* tgt_hi, float* tgt_lo, float* nb, cudaStream_t st);
+                                   double c, int aug, float* tgt_hi, float* tgt_lo, float* nb, cudaStream_t st);
 // maps: A_hi, A_lo (targets), B_hi, B_lo (sources), W_hi, W_lo (weights^T)
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st);
 int fused_tc_stages();
