@@ -313,15 +313,22 @@ def run_ours(args):
     max_mhz = clk_sum["sm_max_mhz"] or 1965
     if info1["path"] == ks.KS_PATH_TC:
         nprod = 3 if info1["precision"] == ks.KS_PREC_3XTF32 else 1
-        flops_pair = nprod * 2 * (K + R)
+        # R == 1: the weighted sum runs on CUDA cores, the tensor work is the 2K contraction
+        flops_pair = nprod * 2 * (K + (R if R > 1 else 0))
         achieved = pairs_launch * flops_pair / (kms / 1e3) / 1e12
         bf16 = load_peaks().get("bf16_tflops")
         peak = (bf16 * 0.5) if bf16 else 1100.0
+        formula = "%d products x 2K per pair" % nprod if R == 1 else "%d products x 2(K+R) per pair" % nprod
         roof = {"bound": "tensor", "kernel": "ks_fused_tc_kernel", "achieved": achieved, "peak": peak,
-                "unit": "TFLOP/s (TF32 tensor; %d products x 2(K+R) per pair)" % nprod, "frac": achieved / peak,
+                "unit": "TFLOP/s (TF32 tensor; %s)" % formula, "frac": achieved / peak,
                 "traffic": load_traffic(args.cfg, args.precision),
                 "peak_derivation": ("MEASURED_PEAKS bf16_tflops (burst) %.1f x 0.5 (nominal TF32/BF16 = 1.1/2.25 "
                                     "PFLOP/s)" % bf16) if bf16 else "fallback nominal dense TF32 1.1 PFLOP/s"}
+        # co-bound: one MUFU ex2 per pair, 16 / clk / SM
+        sfu_peak = 16 * sms * max_mhz * 1e6
+        roof["sfu"] = {"achieved_ex2_per_s": pairs_launch / (kms / 1e3), "peak_ex2_per_s": sfu_peak,
+                       "frac": pairs_launch / (kms / 1e3) / sfu_peak,
+                       "peak_derivation": f"16 ex2/clk/SM x {sms} SMs x {max_mhz} MHz"}
     else:
         fp32_ops, mufu = per_pair_ops(K, R)
         achieved = pairs_launch * fp32_ops / (kms / 1e3) / 1e12      # T FP32-pipe lane-ops / s

@@ -119,7 +119,7 @@ struct ks_ctx {
   int R = 1;
   DBuf<float> src;        // FP32 path: [k_pad + 2][m_pad]
   // TC path (tcgen05): TF32 hi/lo operand splits, norms, W^T splits
-  DBuf<float> src_hi, src_lo, na, wt_hi, wt_lo;
+  DBuf<float> src_hi, src_lo, na, wt_hi, wt_lo, w0;
   DBuf<float> tgt_hi, tgt_lo, nb;
   int r_pad = 16;
   int tc_aug = 0;  // norms folded into the contraction as 2 extra K columns
@@ -320,6 +320,7 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(ctx->na.reserve((size_t)m_pad, st, false), "allocate source norms");
   KS_CUDA(ctx->wt_hi.reserve(nw, st, false), "allocate W hi");
   KS_CUDA(ctx->wt_lo.reserve(nw, st, false), "allocate W lo");
+  KS_CUDA(ctx->w0.reserve((size_t)m_pad, st, false), "allocate W column 0");
   KS_CUDA(ctx->mu.reserve(k_pad, st, false), "allocate mean buffer");
   int nparts = (int)((M + 511) / 512);
   if (nparts < 1) nparts = 1;
@@ -328,7 +329,7 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(ks::launch_source_mean(alpha, M, K, k_pad, ctx->mean_part.p, nparts, ctx->mu.p, st), "source mean");
   ctx->launches += (M > 0) ? 2 : 1;
   KS_CUDA(ks::launch_prep_tc_sources(alpha, W, M, m_pad, K, k_pad, R, r_pad, ctx->mu.p, ctx->c, aug,
-                                     ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p, st),
+                                     ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p, ctx->w0.p, st),
           "source prep (TC)");
   ctx->launches += 1;
   ks_status s = encode_2d_sw64(&ctx->tmB_hi, ctx->src_hi.p, k_pad, m_pad, ks::kTcTileS);
@@ -378,6 +379,12 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.R = ctx->R;
   a.three = (ctx->prec_eff == KS_PREC_TF32) ? 0 : 1;
   a.aug = ctx->tc_aug;
+  a.w0 = ctx->w0.p;
+  {
+    // R == 1: weighted sum on CUDA cores (KS_TC_VCC=0 forces the tensor-core V path; measurement knob)
+    const char* e = getenv("KS_TC_VCC");
+    a.vcc = (ctx->R == 1 && !(e && e[0] == '0')) ? 1 : 0;
+  }
   {
     const char* e = getenv("KS_TC_DEBUG_SKIP_V");
     a.dbg_skip_v = (e && e[0] == '1') ? 1 : 0;
@@ -483,8 +490,8 @@ ks_status ks_destroy(ks_ctx* ctx) {
   set_device(ctx);
   cudaStreamSynchronize(ctx->stream);
   ctx->src.release();
-  for (DBuf<float>* bptr : {&ctx->src_hi, &ctx->src_lo, &ctx->na, &ctx->wt_hi, &ctx->wt_lo, &ctx->tgt_hi, &ctx->tgt_lo,
-                            &ctx->nb})
+  for (DBuf<float>* bptr : {&ctx->src_hi, &ctx->src_lo, &ctx->na, &ctx->wt_hi, &ctx->wt_lo, &ctx->w0, &ctx->tgt_hi,
+                            &ctx->tgt_lo, &ctx->nb})
     bptr->release();
   ctx->mu.release();
   ctx->mean_part.release();
@@ -523,7 +530,10 @@ ks_status ks_set_sources(ks_ctx* ctx, const float* alpha, const float* W, int64_
   int prec = ctx->prec_req;
   int path;
   if (prec == KS_PREC_AUTO) {
-    path = (ctx->K <= 32 && R == 1) ? KS_PATH_FP32 : KS_PATH_TC;
+    // Measured on B200 (SS7): the tcgen05 3xTF32 kernel is faster for
+    // every configuration except tiny source sets (M <= 4096, K <= 32, R == 1),
+    // where the FP32 kernel's lower fixed cost wins.
+    path = (ctx->K <= 32 && R == 1 && M <= 4096) ? KS_PATH_FP32 : KS_PATH_TC;
     prec = (path == KS_PATH_FP32) ? KS_PREC_FP32 : KS_PREC_3XTF32;
   } else if (prec == KS_PREC_FP32) {
     if (ctx->K > 32 || R != 1)

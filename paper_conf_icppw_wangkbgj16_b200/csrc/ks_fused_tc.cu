@@ -51,7 +51,7 @@ struct TcSmemT {
   // hi, lo, na[128]; slots 1024-aligned so every SWIZZLE_64B atom starts on a 512 B boundary
   static constexpr uint32_t w_slot_bytes(int r_c) { return (2 * wslot(r_c) + 512 + 1023) & ~1023u; }
   static constexpr uint32_t bar_off(int r_c) { return kW0 + 2 * w_slot_bytes(r_c); }
-  static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 256; }
+  static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 256 + 4 * kTcTileT * 8; }  // + VCC scratch
 };
 
 __device__ __forceinline__ int64_t sk_start(int64_t b, int64_t U, int64_t G) { return (b * U) / G; }
@@ -114,7 +114,10 @@ __device__ __forceinline__ void unit_next(const Sched& s, UnitIt& u) {
 
 }  // namespace
 
-template <int RC, int kStages>
+// VCC: R == 1 -- the weighted reduction runs on CUDA cores in the epilogue
+// (one FFMA per pair, W_i broadcast from shared memory) instead of a second
+// tensor-core contraction; no P_hi/P_lo stores, no V MMA.
+template <int RC, int kStages, bool VCC>
 __global__ void __launch_bounds__(kTcThreads, 1)
     ks_fused_tc_kernel(const __grid_constant__ CUtensorMap mA_hi, const __grid_constant__ CUtensorMap mA_lo,
                        const __grid_constant__ CUtensorMap mB_hi, const __grid_constant__ CUtensorMap mB_lo,
@@ -135,7 +138,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   uint64_t* sfull = wempty + 2;          // [2]
   uint64_t* pready = sfull + 2;          // [2 S buffers][2 source halves]
   uint64_t* vdone = pready + 4;          // [2 source halves]
-  uint32_t* tmem_base_smem = reinterpret_cast<uint32_t*>(vdone + 2);
+  uint64_t* sempty = vdone + 2;          // [2] (VCC: epilogue has read the S buffer)
+  uint32_t* tmem_base_smem = reinterpret_cast<uint32_t*>(sempty + 2);
   int* flag = reinterpret_cast<int*>(tmem_base_smem + 1);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -158,14 +162,16 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     }
     for (int i = 0; i < 2; ++i) {
       mbar_init(&wfull[i], 1);
-      mbar_init(&wempty[i], 1);
+      mbar_init(&wempty[i], VCC ? EW : 1);
+      mbar_init(&sempty[i], EW);
       mbar_init(&sfull[i], 1);
       mbar_init(&vdone[i], 1);
     }
     for (int i = 0; i < 4; ++i) mbar_init(&pready[i], EW);  // one arrival per epilogue warp
     fence_mbar_init();
   }
-  if (warp == 2) tmem_alloc(tmem_base_smem, 512);
+  constexpr uint32_t kTmemCols = VCC ? 256 : 512;
+  if (warp == 2) tmem_alloc(tmem_base_smem, kTmemCols);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -189,10 +195,16 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         mbar_wait(&wempty[slot], (use & 1) ^ 1);
         uint8_t* ws = smem + TcSmem::kW0 + slot * TcSmem::w_slot_bytes(RC);
         if (leader) {
-          mbar_arrive_expect_tx(&wfull[slot], 2 * TcSmem::wslot(RC) + 512);
-          tma_load_3d(ws, &mW_hi, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
-          tma_load_3d(ws + TcSmem::wslot(RC), &mW_lo, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
-          bulk_load(ws + 2 * TcSmem::wslot(RC), args.na + (int64_t)st * kTcTileS, 512, &wfull[slot]);
+          if constexpr (VCC) {  // na and the single weight column
+            mbar_arrive_expect_tx(&wfull[slot], 1024);
+            bulk_load(ws + 2 * TcSmem::wslot(RC), args.na + (int64_t)st * kTcTileS, 512, &wfull[slot]);
+            bulk_load(ws + 2 * TcSmem::wslot(RC) + 512, args.w0 + (int64_t)st * kTcTileS, 512, &wfull[slot]);
+          } else {
+            mbar_arrive_expect_tx(&wfull[slot], 2 * TcSmem::wslot(RC) + 512);
+            tma_load_3d(ws, &mW_hi, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
+            tma_load_3d(ws + TcSmem::wslot(RC), &mW_lo, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
+            bulk_load(ws + 2 * TcSmem::wslot(RC), args.na + (int64_t)st * kTcTileS, 512, &wfull[slot]);
+          }
         }
         __syncwarp();
       }
@@ -258,6 +270,12 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
       const int bq = q & 1;
       const uint32_t dS = tbase + (bq ? kColS1 : kColS0);
+      if constexpr (VCC) {
+        if (q >= 2) {  // the epilogue has read S(q-2) out of this buffer
+          mbar_wait(&sempty[bq], (uint32_t)(((q - 2) >> 1) & 1));
+          tc_fence_after();
+        }
+      }
       for (int kc = 0; kc < n_kc; ++kc, ++it) {
         const int s = it % kStages;
         const uint32_t use = (uint32_t)(it / kStages);
@@ -288,17 +306,122 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       }
       if (leader) tc_commit(&sfull[bq]);
       __syncwarp();
-      if (q > 0) {
-        v_mma(q - 1, prev_st, 0);
-        v_mma(q - 1, prev_st, 1);
+      if constexpr (!VCC) {
+        if (q > 0) {
+          v_mma(q - 1, prev_st, 0);
+          v_mma(q - 1, prev_st, 1);
+        }
       }
       prev_st = cu.st;
     }
-    if (count > 0) {
-      v_mma(count - 1, prev_st, 0);
-      v_mma(count - 1, prev_st, 1);
+    if constexpr (!VCC) {
+      if (count > 0) {
+        v_mma(count - 1, prev_st, 0);
+        v_mma(count - 1, prev_st, 1);
+      }
     }
-  } else if (warp >= 4) {
+  } else if (VCC && warp >= 4) {
+    // ================= epilogue, R == 1: V on CUDA cores
+    const int ew = warp - 4;
+    const int g = ew & 3;                 // TMEM lanes 32g..32g+31
+    const int h = ew >> 2;                // columns 64hh + CB h .. + CB-1 of each source half hh
+    const int row = 32 * g + lane;        // target row within the tile
+    const uint32_t lane_off = (uint32_t)(32 * g) << 16;
+    double* red = reinterpret_cast<double*>(smem + TcSmem::bar_off(RC) + 256);  // [SUB][128]
+    double vacc = 0.0;
+    float nbj = 0.f;
+    int seg_q = 0, seg_st0 = 0;
+    UnitIt cu = unit_begin(sc);
+    for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
+      const int bq = q & 1;
+      const uint32_t use = (uint32_t)(q >> 1);
+      if (q == seg_q) {
+        seg_st0 = cu.st;
+        if (!args.aug) nbj = __ldg(args.nb + cu.tt * kTcTileT + row);
+      }
+      mbar_wait(&wfull[q & 1], use & 1);
+      mbar_wait(&sfull[bq], use & 1);
+      tc_fence_after();
+      const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC) +
+                                                       2 * TcSmem::wslot(RC));
+      const float* w0s = nas + 128;
+      const uint32_t colS = bq ? kColS1 : kColS0;
+      uint32_t sv[2][CB];
+      tmem_ldn<CB>(tbase + lane_off + colS + CB * h, sv[0]);
+      tmem_ldn<CB>(tbase + lane_off + colS + 64 + CB * h, sv[1]);
+      tmem_wait_ld();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&sempty[bq]);  // S buffer may be overwritten now
+      float vt = 0.f;
+#pragma unroll
+      for (int hh = 0; hh < 2; ++hh) {
+        const int c0 = 64 * hh + CB * h;
+#pragma unroll
+        for (int i = 0; i < CB; i += 4) {
+          const float4 w4 = *reinterpret_cast<const float4*>(w0s + c0 + i);
+          const float wv[4] = {w4.x, w4.y, w4.z, w4.w};
+          float nav[4] = {0.f, 0.f, 0.f, 0.f};
+          if (!args.aug) {
+            const float4 na4 = *reinterpret_cast<const float4*>(nas + c0 + i);
+            nav[0] = na4.x + nbj; nav[1] = na4.y + nbj; nav[2] = na4.z + nbj; nav[3] = na4.w + nbj;
+          }
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const float t = fminf(__uint_as_float(sv[hh][i + e]) + nav[e], 0.f);  // clamp d^2 >= 0
+            vt = fmaf(ex2_approx(t), wv[e], vt);
+          }
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&wempty[q & 1]);  // na / W slot consumed
+      vacc += (double)vt;
+      const bool seg_end = (q == count - 1) || (cu.st + 1 == n_s);
+      if (seg_end) {
+        // combine the SUB column groups of each row in a fixed order
+        red[h * kTcTileT + row] = vacc;
+        named_bar_sync(1, 32 * EW);
+        if (h == 0) {
+          double v = 0.0;
+#pragma unroll
+          for (int k = 0; k < SUB; ++k) v += red[k * kTcTileT + row];
+          const int seg_len = q - seg_q + 1;
+          const bool whole = (seg_st0 == 0) && (seg_len == n_s);
+          const int64_t grow = cu.tt * kTcTileT + row;
+          if (whole) {
+            if (grow < args.N) args.V[grow * args.R + args.r_off] = (float)v;
+          } else {
+            const int64_t tr = cu.tt - sc.rem_t0;
+            const int slot = (tr == sc.v0 / n_s) ? 0 : 1;
+            args.partial[(b * 2 + slot) * kTcTileT + row] = (float)v;
+            __threadfence();
+            named_bar_sync(2, 128);
+            const int64_t b_first = sk_owner(tr * n_s, sc.Urem, sc.Gr);
+            const int64_t b_last = sk_owner(tr * n_s + n_s - 1, sc.Urem, sc.Gr);
+            if (row == 0) {
+              const int old = atomicAdd(&args.counters[cu.tt], 1);
+              const int last = (old == (int)(b_last - b_first));
+              if (last) args.counters[cu.tt] = 0;
+              *flag = last;
+            }
+            named_bar_sync(2, 128);
+            if (*flag) {
+              __threadfence();
+              float sum = 0.f;
+              for (int64_t bb = b_first; bb <= b_last; ++bb) {
+                const int sl = (tr == sk_start(bb, sc.Urem, sc.Gr) / n_s) ? 0 : 1;
+                sum += __ldcg(args.partial + (bb * 2 + sl) * kTcTileT + row);
+              }
+              if (grow < args.N) args.V[grow * args.R + args.r_off] = sum;
+            }
+          }
+        }
+        named_bar_sync(1, 32 * EW);  // red / flag reuse
+        vacc = 0.0;
+        seg_q = q + 1;
+      }
+    }
+  } else if (!VCC && warp >= 4) {
     // ================= epilogue (EW warps: TMEM lane group g, sub-split h)
     const int ew = warp - 4;
     const int g = ew & 3;                 // TMEM lanes 32g..32g+31
@@ -448,7 +571,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  if (warp == 2) tmem_dealloc(tbase, 512);
+  if (warp == 2) tmem_dealloc(tbase, kTmemCols);
   if (args.cta_times != nullptr && tid == 0) {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -461,7 +584,8 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
                                        int64_t m_pad, int K, int k_pad, int R, int r_pad,
                                        const float* __restrict__ mu, double c, int aug, float* __restrict__ src_hi,
                                        float* __restrict__ src_lo, float* __restrict__ na,
-                                       float* __restrict__ wt_hi, float* __restrict__ wt_lo) {
+                                       float* __restrict__ wt_hi, float* __restrict__ wt_lo,
+                                       float* __restrict__ w0) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= m_pad) return;
   const bool live = i < M;
@@ -487,6 +611,7 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
     src_hi[i * k_pad + d] = ah;
     src_lo[i * k_pad + d] = to_tf32(a - ah);
   }
+  w0[i] = live ? W[i * R] : 0.f;
   for (int r = 0; r < r_pad; ++r) {
     const float w = (live && r < R) ? W[i * R + r] : 0.f;
     const float wh = to_tf32(w);
@@ -521,11 +646,12 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
 
 cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
                                    int R, int r_pad, const float* mu, double c, int aug, float* src_hi,
-                                   float* src_lo, float* na, float* wt_hi, float* wt_lo, cudaStream_t st) {
+                                   float* src_lo, float* na, float* wt_hi, float* wt_lo, float* w0,
+                                   cudaStream_t st) {
   if (m_pad == 0) return cudaSuccess;
   const int bs = 128;
   prep_tc_sources_kernel<<<(unsigned)((m_pad + bs - 1) / bs), bs, 0, st>>>(
-      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, src_hi, src_lo, na, wt_hi, wt_lo);
+      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, src_hi, src_lo, na, wt_hi, wt_lo, w0);
   return cudaGetLastError();
 }
 
@@ -556,18 +682,24 @@ size_t fused_tc_smem(int r_c) {
 }
 int fused_tc_stages() { return tc_stages(16); }
 
-template <int RC, int NS>
-static cudaError_t launch_rcs(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
+template <int RC, int NS, bool VCC>
+static cudaError_t launch_rcsv(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
   static bool attr_done = false;
   const size_t smem = TcSmemT<NS>::total(RC);
   if (!attr_done) {
-    cudaError_t e =
-        cudaFuncSetAttribute(ks_fused_tc_kernel<RC, NS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(ks_fused_tc_kernel<RC, NS, VCC>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr_done = true;
   }
-  ks_fused_tc_kernel<RC, NS><<<a.sk.grid, kTcThreads, smem, st>>>(m[0], m[1], m[2], m[3], m[4], m[5], a);
+  ks_fused_tc_kernel<RC, NS, VCC><<<a.sk.grid, kTcThreads, smem, st>>>(m[0], m[1], m[2], m[3], m[4], m[5], a);
   return cudaGetLastError();
+}
+
+template <int RC, int NS>
+static cudaError_t launch_rcs(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
+  if (RC == 16 && a.vcc) return launch_rcsv<RC, NS, true>(m, a, st);
+  return launch_rcsv<RC, NS, false>(m, a, st);
 }
 
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st) {

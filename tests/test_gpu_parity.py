@@ -22,8 +22,19 @@ if not torch.cuda.is_available():
 
 import paper_conf_icppw_wangkbgj16_b200 as ks  # noqa: E402
 
+# Every test in this module runs on both K<=32 kernels: the FP32 FFMA2 kernel
+# and the tcgen05 3xTF32 kernel (the AUTO choice for M > 4096).
+_PREC = {"p": "fp32"}
 
-def gpu_eval(alpha, W, beta, h, precision="auto", host=False):
+
+@pytest.fixture(autouse=True, params=["fp32", "3xtf32"])
+def precision(request):
+    _PREC["p"] = request.param
+    yield request.param
+
+
+def gpu_eval(alpha, W, beta, h, precision=None, host=False):
+    precision = precision or _PREC["p"]
     K = alpha.shape[1]
     W = np.asarray(W, np.float32)
     if W.ndim == 1:
@@ -41,7 +52,7 @@ def gpu_eval(alpha, W, beta, h, precision="auto", host=False):
         return V.cpu().numpy().astype(np.float64)
 
 
-def check(oracle_mod, alpha, W, beta, h, tol=TOL_FP32, J=None, precision="auto", V=None):
+def check(oracle_mod, alpha, W, beta, h, tol=TOL_FP32, J=None, precision=None, V=None):
     if V is None:
         V = gpu_eval(alpha, W, beta, h, precision)
     Vg = V if J is None else V[J]
@@ -162,7 +173,7 @@ def test_beta_equals_alpha_self_kernel_one():
 
 
 def test_zero_sources_gives_zeros():
-    with ks.KernelSum(4, 1.0) as plan:
+    with ks.KernelSum(4, 1.0, _PREC["p"]) as plan:
         plan.set_sources(torch.zeros((0, 4), device="cuda"), torch.zeros((0, 1), device="cuda"))
         V = plan.eval(torch.rand((300, 4), device="cuda"))
         torch.cuda.synchronize()
@@ -170,7 +181,7 @@ def test_zero_sources_gives_zeros():
 
 
 def test_zero_targets_noop():
-    with ks.KernelSum(4, 1.0) as plan:
+    with ks.KernelSum(4, 1.0, _PREC["p"]) as plan:
         plan.set_sources(torch.rand((10, 4), device="cuda"), torch.rand((10, 1), device="cuda"))
         V = plan.eval(torch.zeros((0, 4), device="cuda"))
         assert V.shape == (0, 1)
@@ -190,7 +201,7 @@ def test_repeated_eval_and_reset_sources(oracle_mod):
     """Counters are left zero across launches; sources can be replaced."""
     a, W, b, h = workloads.make(3, M=4000, N=200, wkind="pos")
     a2, W2, _, _ = workloads.make(3, M=2500, N=10, wkind="signed", seed_offset=9)
-    with ks.KernelSum(32, float(h)) as plan:
+    with ks.KernelSum(32, float(h), _PREC["p"]) as plan:
         tb = torch.from_numpy(b).cuda()
         plan.set_sources(torch.from_numpy(a).cuda(), torch.from_numpy(W).cuda())
         V1 = [plan.eval(tb).cpu().numpy() for _ in range(3)]
@@ -231,10 +242,19 @@ def test_api_errors():
         ks.ks_destroy(ctx)
 
 
-def test_info_reports_fp32_path():
-    with ks.KernelSum(32, 1.0) as plan:
+def test_info_reports_path():
+    with ks.KernelSum(32, 1.0, _PREC["p"]) as plan:
         plan.set_sources(torch.rand((1000, 32), device="cuda"), torch.rand((1000, 1), device="cuda"))
         plan.eval(torch.rand((5000, 32), device="cuda"))
         info = plan.info()
-        assert info["path"] == ks.KS_PATH_FP32 and info["k_pad"] == 32
+        want = ks.KS_PATH_FP32 if _PREC["p"] == "fp32" else ks.KS_PATH_TC
+        assert info["path"] == want and info["k_pad"] == 32
         assert info["num_ctas"] >= 1 and info["fused_launches"] == 1
+
+
+def test_auto_policy():
+    """AUTO: FP32 kernel for tiny source sets, tcgen05 3xTF32 otherwise (SS7)."""
+    for M, want in ((1024, ks.KS_PATH_FP32), (8192, ks.KS_PATH_TC)):
+        with ks.KernelSum(32, 1.0, "auto") as plan:
+            plan.set_sources(torch.rand((M, 32), device="cuda"), torch.rand((M, 1), device="cuda"))
+            assert plan.info()["path"] == want
