@@ -123,6 +123,7 @@ struct ks_ctx {
   DBuf<float> tgt_hi, tgt_lo, nb;
   int r_pad = 16;
   int tc_aug = 0;  // norms folded into the contraction as 2 extra K columns
+  int tc_vcc = 0;  // R == 1: weighted sum on CUDA cores (W^T tiles not needed)
   CUtensorMap tmB_hi, tmB_lo;
   DBuf<float> mu;         // [k_pad]
   DBuf<double> mean_part; // [nparts][K]
@@ -191,9 +192,9 @@ ks_status prepare_fp32(ks_ctx* ctx, const float* alpha, const float* W, int64_t 
   const size_t need = (size_t)(k_pad + 2) * (size_t)m_pad;
   KS_CUDA(ctx->src.reserve(need, st, false), "allocate source buffer");
   KS_CUDA(ctx->mu.reserve(k_pad, st, false), "allocate mean buffer");
-  int nparts = (int)((M + 511) / 512);
+  int nparts = (int)((M + 63) / 64);  // source-mean blocks of <= 64 rows each
   if (nparts < 1) nparts = 1;
-  if (nparts > 1024) nparts = 1024;
+  if (nparts > 2048) nparts = 2048;
   KS_CUDA(ctx->mean_part.reserve((size_t)nparts * K, st, false), "allocate mean partials");
   KS_CUDA(ks::launch_source_mean(alpha, M, K, k_pad, ctx->mean_part.p, nparts, ctx->mu.p, st), "source mean");
   ctx->launches += (M > 0) ? 2 : 1;
@@ -311,6 +312,9 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   const int K = ctx->K;
   const int k_pad = tc_k_pad(K);
   const int aug = tc_aug(K);
+  // R == 1: weighted sum on CUDA cores (KS_TC_VCC=0 forces the tensor-core V path; measurement knob)
+  const char* ev = getenv("KS_TC_VCC");
+  const int vcc = (R == 1 && !(ev && ev[0] == '0')) ? 1 : 0;
   const int64_t m_pad = round_up(M > 0 ? M : 1, ks::kTcTileS);
   const int r_pad = (int)round_up(R, 16);
   cudaStream_t st = ctx->stream;
@@ -322,13 +326,13 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(ctx->wt_lo.reserve(nw, st, false), "allocate W lo");
   KS_CUDA(ctx->w0.reserve((size_t)m_pad, st, false), "allocate W column 0");
   KS_CUDA(ctx->mu.reserve(k_pad, st, false), "allocate mean buffer");
-  int nparts = (int)((M + 511) / 512);
+  int nparts = (int)((M + 63) / 64);  // source-mean blocks of <= 64 rows each
   if (nparts < 1) nparts = 1;
-  if (nparts > 1024) nparts = 1024;
+  if (nparts > 2048) nparts = 2048;
   KS_CUDA(ctx->mean_part.reserve((size_t)nparts * K, st, false), "allocate mean partials");
   KS_CUDA(ks::launch_source_mean(alpha, M, K, k_pad, ctx->mean_part.p, nparts, ctx->mu.p, st), "source mean");
   ctx->launches += (M > 0) ? 2 : 1;
-  KS_CUDA(ks::launch_prep_tc_sources(alpha, W, M, m_pad, K, k_pad, R, r_pad, ctx->mu.p, ctx->c, aug,
+  KS_CUDA(ks::launch_prep_tc_sources(alpha, W, M, m_pad, K, k_pad, R, vcc ? 0 : r_pad, ctx->mu.p, ctx->c, aug,
                                      ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p, ctx->w0.p, st),
           "source prep (TC)");
   ctx->launches += 1;
@@ -340,6 +344,7 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   ctx->m_pad = m_pad;
   ctx->r_pad = r_pad;
   ctx->tc_aug = aug;
+  ctx->tc_vcc = vcc;
   return KS_OK;
 }
 
@@ -380,11 +385,7 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.three = (ctx->prec_eff == KS_PREC_TF32) ? 0 : 1;
   a.aug = ctx->tc_aug;
   a.w0 = ctx->w0.p;
-  {
-    // R == 1: weighted sum on CUDA cores (KS_TC_VCC=0 forces the tensor-core V path; measurement knob)
-    const char* e = getenv("KS_TC_VCC");
-    a.vcc = (ctx->R == 1 && !(e && e[0] == '0')) ? 1 : 0;
-  }
+  a.vcc = ctx->tc_vcc;
   {
     const char* e = getenv("KS_TC_DEBUG_SKIP_V");
     a.dbg_skip_v = (e && e[0] == '1') ? 1 : 0;

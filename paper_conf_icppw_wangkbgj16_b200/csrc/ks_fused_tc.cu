@@ -580,24 +580,34 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 }
 
 // ---------------------------------------------------------------- prep (a1 / a2 for the TC path)
+// One warp per point: lanes stride over the coordinates (coalesced reads of a
+// row and coalesced writes of its padded split row), the norm is a fixed-order
+// FP64 warp reduction (lane partials in lane order via shuffles).
+__device__ __forceinline__ double warp_sum_fixed(double v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
+  return __shfl_sync(0xffffffffu, v, 0);
+}
+
 __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const float* __restrict__ W, int64_t M,
                                        int64_t m_pad, int K, int k_pad, int R, int r_pad,
                                        const float* __restrict__ mu, double c, int aug, float* __restrict__ src_hi,
                                        float* __restrict__ src_lo, float* __restrict__ na,
                                        float* __restrict__ wt_hi, float* __restrict__ wt_lo,
                                        float* __restrict__ w0) {
-  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
   if (i >= m_pad) return;
   const bool live = i < M;
-  const double c2 = 2.0 * c;
   double n = 0.0;
-  for (int d = 0; d < K; ++d) {
+  for (int d = lane; d < K; d += 32) {
     const float x = live ? alpha[i * K + d] - mu[d] : 0.f;  // FP32 centring, same op as the target side
     n += (double)x * (double)x;
   }
+  n = warp_sum_fixed(n);
   const float nai = live ? (float)(-c * n) : 0.f;
-  na[i] = nai;
-  for (int d = 0; d < k_pad; ++d) {
+  const double c2 = 2.0 * c;
+  for (int d = lane; d < k_pad; d += 32) {
     float a = 0.f;
     if (d < K) {
       const float x = live ? alpha[i * K + d] - mu[d] : 0.f;
@@ -611,8 +621,11 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
     src_hi[i * k_pad + d] = ah;
     src_lo[i * k_pad + d] = to_tf32(a - ah);
   }
-  w0[i] = live ? W[i * R] : 0.f;
-  for (int r = 0; r < r_pad; ++r) {
+  if (lane == 0) {
+    na[i] = nai;
+    w0[i] = live ? W[i * R] : 0.f;
+  }
+  for (int r = lane; r < r_pad; r += 32) {
     const float w = (live && r < R) ? W[i * R + r] : 0.f;
     const float wh = to_tf32(w);
     wt_hi[(int64_t)r * m_pad + i] = wh;
@@ -623,17 +636,18 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
 __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N, int64_t n_pad, int K, int k_pad,
                                        const float* __restrict__ mu, double c, int aug, float* __restrict__ tgt_hi,
                                        float* __restrict__ tgt_lo, float* __restrict__ nb) {
-  const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
   if (j >= n_pad) return;
   const bool live = j < N;
   double n = 0.0;
-  for (int d = 0; d < K; ++d) {
+  for (int d = lane; d < K; d += 32) {
     const float x = live ? beta[j * K + d] - mu[d] : 0.f;
     n += (double)x * (double)x;
   }
+  n = warp_sum_fixed(n);
   const float nbj = live ? (float)(-c * n) : 0.f;
-  nb[j] = nbj;
-  for (int d = 0; d < k_pad; ++d) {
+  for (int d = lane; d < k_pad; d += 32) {
     float x = 0.f;
     if (d < K) x = live ? beta[j * K + d] - mu[d] : 0.f;
     else if (aug && d == K) x = nbj;
@@ -642,6 +656,7 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
     tgt_hi[j * k_pad + d] = xh;
     tgt_lo[j * k_pad + d] = to_tf32(x - xh);
   }
+  if (lane == 0) nb[j] = nbj;
 }
 
 cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
@@ -649,8 +664,8 @@ cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M
                                    float* src_lo, float* na, float* wt_hi, float* wt_lo, float* w0,
                                    cudaStream_t st) {
   if (m_pad == 0) return cudaSuccess;
-  const int bs = 128;
-  prep_tc_sources_kernel<<<(unsigned)((m_pad + bs - 1) / bs), bs, 0, st>>>(
+  const int bs = 256;  // 8 points per block
+  prep_tc_sources_kernel<<<(unsigned)((m_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
       alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, src_hi, src_lo, na, wt_hi, wt_lo, w0);
   return cudaGetLastError();
 }
@@ -658,9 +673,9 @@ cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M
 cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
                                    double c, int aug, float* tgt_hi, float* tgt_lo, float* nb, cudaStream_t st) {
   if (n_pad == 0) return cudaSuccess;
-  const int bs = 128;
-  prep_tc_targets_kernel<<<(unsigned)((n_pad + bs - 1) / bs), bs, 0, st>>>(beta, N, n_pad, K, k_pad, mu, c, aug,
-                                                                          tgt_hi, tgt_lo, nb);
+  const int bs = 256;
+  prep_tc_targets_kernel<<<(unsigned)((n_pad * 32 + bs - 1) / bs), bs, 0, st>>>(beta, N, n_pad, K, k_pad, mu, c, aug,
+                                                                                tgt_hi, tgt_lo, nb);
   return cudaGetLastError();
 }
 

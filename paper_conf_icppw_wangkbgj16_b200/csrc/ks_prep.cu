@@ -49,17 +49,19 @@ __global__ void source_mean_partial_kernel(const float* __restrict__ alpha, int6
   }
 }
 
+// One warp per dimension: lanes sum the block partials in a fixed strided
+// order, then a fixed shuffle tree (deterministic).
 __global__ void source_mean_final_kernel(const double* __restrict__ part, int nparts, int64_t M, int K,
                                          int k_pad, float* __restrict__ mu) {
-  for (int d = threadIdx.x; d < k_pad; d += blockDim.x) {
-    float m = 0.f;
-    if (d < K && M > 0) {
-      double s = 0.0;
-      for (int b = 0; b < nparts; ++b) s += part[(int64_t)b * K + d];
-      m = (float)(s / (double)M);
-    }
-    mu[d] = m;
-  }
+  const int d = (int)(((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+  const int lane = threadIdx.x & 31;
+  if (d >= k_pad) return;
+  double s = 0.0;
+  if (d < K)
+    for (int b = lane; b < nparts; b += 32) s += part[(int64_t)b * K + d];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_down_sync(0xffffffffu, s, o);
+  if (lane == 0) mu[d] = (d < K && M > 0) ? (float)(s / (double)M) : 0.f;
 }
 
 cudaError_t launch_source_mean(const float* alpha, int64_t M, int K, int k_pad, double* part, int nparts,
@@ -67,7 +69,9 @@ cudaError_t launch_source_mean(const float* alpha, int64_t M, int K, int k_pad, 
   if (M > 0) {
     source_mean_partial_kernel<<<nparts, 256, 0, st>>>(alpha, M, K, nparts, part);
   }
-  source_mean_final_kernel<<<1, 256, 0, st>>>(part, M > 0 ? nparts : 0, M, K, k_pad, mu);
+  const int warps_per_block = 8;
+  source_mean_final_kernel<<<(k_pad + warps_per_block - 1) / warps_per_block, 32 * warps_per_block, 0, st>>>(
+      part, M > 0 ? nparts : 0, M, K, k_pad, mu);
   return cudaGetLastError();
 }
 
