@@ -315,7 +315,8 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   // R == 1: weighted sum on CUDA cores (KS_TC_VCC=0 forces the tensor-core V path; measurement knob)
   const char* ev = getenv("KS_TC_VCC");
   const int vcc = (R == 1 && !(ev && ev[0] == '0')) ? 1 : 0;
-  const int64_t m_pad = round_up(M > 0 ? M : 1, ks::kTcTileS);
+  const int tile_s = ks::fused_tc_tile_s(vcc);
+  const int64_t m_pad = round_up(M > 0 ? M : 1, tile_s);
   const int r_pad = (int)round_up(R, 16);
   cudaStream_t st = ctx->stream;
   const size_t nsrc = (size_t)m_pad * k_pad, nw = (size_t)r_pad * m_pad;
@@ -336,9 +337,9 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
                                      ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p, ctx->w0.p, st),
           "source prep (TC)");
   ctx->launches += 1;
-  ks_status s = encode_2d_sw64(&ctx->tmB_hi, ctx->src_hi.p, k_pad, m_pad, ks::kTcTileS);
+  ks_status s = encode_2d_sw64(&ctx->tmB_hi, ctx->src_hi.p, k_pad, m_pad, tile_s);
   if (s != KS_OK) return s;
-  s = encode_2d_sw64(&ctx->tmB_lo, ctx->src_lo.p, k_pad, m_pad, ks::kTcTileS);
+  s = encode_2d_sw64(&ctx->tmB_lo, ctx->src_lo.p, k_pad, m_pad, tile_s);
   if (s != KS_OK) return s;
   ctx->k_pad = k_pad;
   ctx->m_pad = m_pad;
@@ -370,7 +371,7 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
 
   ks::StreamK sk;
   sk.n_t = n_pad / ks::kTcTileT;
-  sk.n_s = (int32_t)(ctx->m_pad / ks::kTcTileS);
+  sk.n_s = (int32_t)(ctx->m_pad / ks::fused_tc_tile_s(ctx->tc_vcc));
   sk.units = sk.n_t * (int64_t)sk.n_s;
   int64_t g = ctx->num_sms;
   if (g > sk.units) g = sk.units;
@@ -633,7 +634,7 @@ ks_status ks_get_info(const ks_ctx* ctx, ks_info* out) {
   out->k_pad = ctx->k_pad;
   const bool tc = ctx->have_src && ctx->path == KS_PATH_TC;
   out->tile_t = tc ? ks::kTcTileT : ks::kTileT;
-  out->tile_s = tc ? ks::kTcTileS : ks::kTileS;
+  out->tile_s = tc ? ks::fused_tc_tile_s(ctx->tc_vcc) : ks::kTileS;
   out->num_ctas = ctx->last_grid;
   out->stages = !ctx->k_pad ? 0 : (tc ? ks::fused_tc_stages() : ks::fused_fp32_stages(ctx->k_pad));
   out->num_sms = ctx->num_sms;

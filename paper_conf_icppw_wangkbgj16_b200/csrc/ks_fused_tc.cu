@@ -37,19 +37,24 @@ namespace {
 
 constexpr int kMaxStages = 6;                    // A/B ring depth bound (32 KB per stage)
 constexpr int kFlush = 4;                        // units per V accumulation block
-constexpr uint32_t kChunkBytes = kTcTileT * kTcKC * 4;  // one hi or lo operand tile (8 KB)
-constexpr uint32_t kStageBytes = 4 * kChunkBytes;       // A_hi, A_lo, B_hi, B_lo
+constexpr uint32_t kChunkA = kTcTileT * kTcKC * 4;  // one hi or lo target-operand chunk (8 KB)
 // TMEM columns: S0 | S1 (P_hi written in place) | P_lo for source half 0 | half 1 | V
 constexpr uint32_t kColS0 = 0, kColS1 = 128, kColPlo = 256, kColV = 384;
 
-template <int kStages>
+// Shared-memory layout (bytes from a 1 KB-aligned base).  TS = sources per
+// tile (128 with the tensor-core V path, 256 in the R == 1 VCC mode).
+template <int kStages, int TS, bool VCC>
 struct TcSmemT {
-  // offsets in bytes from a 1024-aligned base
+  static constexpr uint32_t kChunkB = TS * kTcKC * 4;                 // one hi or lo source chunk
+  static constexpr uint32_t kStageBytes = 2 * kChunkA + 2 * kChunkB;  // A_hi, A_lo, B_hi, B_lo
   static constexpr uint32_t kStage0 = 0;
-  static constexpr uint32_t wslot(int r_c) { return (uint32_t)r_c * 512u; }  // one of hi/lo: 8 chunks x r_c x 64 B
+  static constexpr uint32_t wslot(int r_c) { return (uint32_t)r_c * 512u; }  // one of W^T hi/lo: 8 chunks x r_c x 64 B
   static constexpr uint32_t kW0 = kStages * kStageBytes;
-  // hi, lo, na[128]; slots 1024-aligned so every SWIZZLE_64B atom starts on a 512 B boundary
-  static constexpr uint32_t w_slot_bytes(int r_c) { return (2 * wslot(r_c) + 512 + 1023) & ~1023u; }
+  // VCC: na[TS] | w0[TS];  else W^T hi | W^T lo | na[128].  Slots 1 KB aligned (SWIZZLE_64B atoms).
+  static constexpr uint32_t w_slot_bytes(int r_c) {
+    return VCC ? ((uint32_t)(8 * TS) + 1023u) & ~1023u : (2 * wslot(r_c) + 512 + 1023) & ~1023u;
+  }
+  static constexpr uint32_t na_off(int r_c) { return VCC ? 0u : 2 * wslot(r_c); }
   static constexpr uint32_t bar_off(int r_c) { return kW0 + 2 * w_slot_bytes(r_c); }
   static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 256 + 4 * kTcTileT * 8; }  // + VCC scratch
 };
@@ -123,7 +128,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
                        const __grid_constant__ CUtensorMap mB_hi, const __grid_constant__ CUtensorMap mB_lo,
                        const __grid_constant__ CUtensorMap mW_hi, const __grid_constant__ CUtensorMap mW_lo,
                        const TcArgs args) {
-  using TcSmem = TcSmemT<kStages>;
+  constexpr int TS = VCC ? 256 : kTcTileS;  // sources per tile
+  using TcSmem = TcSmemT<kStages, TS, VCC>;
+  constexpr uint32_t kChunkB = TcSmem::kChunkB;
+  constexpr uint32_t kStageBytes = TcSmem::kStageBytes;
   constexpr int EW = kTcEpiWarps;        // epilogue warps
   constexpr int SUB = EW / 4;            // epilogue warps per TMEM lane group
   constexpr int CB = 64 / SUB;           // columns per warp per source half
@@ -170,7 +178,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     for (int i = 0; i < 4; ++i) mbar_init(&pready[i], EW);  // one arrival per epilogue warp
     fence_mbar_init();
   }
-  constexpr uint32_t kTmemCols = VCC ? 256 : 512;
+  constexpr uint32_t kTmemCols = 512;  // VCC: two 256-column S buffers; else S0|S1|P_lo|V
   if (warp == 2) tmem_alloc(tmem_base_smem, kTmemCols);
   tc_fence_before();
   __syncthreads();
@@ -196,9 +204,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         uint8_t* ws = smem + TcSmem::kW0 + slot * TcSmem::w_slot_bytes(RC);
         if (leader) {
           if constexpr (VCC) {  // na and the single weight column
-            mbar_arrive_expect_tx(&wfull[slot], 1024);
-            bulk_load(ws + 2 * TcSmem::wslot(RC), args.na + (int64_t)st * kTcTileS, 512, &wfull[slot]);
-            bulk_load(ws + 2 * TcSmem::wslot(RC) + 512, args.w0 + (int64_t)st * kTcTileS, 512, &wfull[slot]);
+            mbar_arrive_expect_tx(&wfull[slot], 8 * TS);
+            bulk_load(ws, args.na + (int64_t)st * TS, 4 * TS, &wfull[slot]);
+            bulk_load(ws + 4 * TS, args.w0 + (int64_t)st * TS, 4 * TS, &wfull[slot]);
           } else {
             mbar_arrive_expect_tx(&wfull[slot], 2 * TcSmem::wslot(RC) + 512);
             tma_load_3d(ws, &mW_hi, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
@@ -216,9 +224,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         if (leader) {
           mbar_arrive_expect_tx(&full[s], kStageBytes);
           tma_load_2d(sp, &mA_hi, kc * kTcKC, tt * kTcTileT, &full[s]);
-          tma_load_2d(sp + kChunkBytes, &mA_lo, kc * kTcKC, tt * kTcTileT, &full[s]);
-          tma_load_2d(sp + 2 * kChunkBytes, &mB_hi, kc * kTcKC, st * kTcTileS, &full[s]);
-          tma_load_2d(sp + 3 * kChunkBytes, &mB_lo, kc * kTcKC, st * kTcTileS, &full[s]);
+          tma_load_2d(sp + kChunkA, &mA_lo, kc * kTcKC, tt * kTcTileT, &full[s]);
+          tma_load_2d(sp + 2 * kChunkA, &mB_hi, kc * kTcKC, st * TS, &full[s]);
+          tma_load_2d(sp + 2 * kChunkA + kChunkB, &mB_lo, kc * kTcKC, st * TS, &full[s]);
         }
         __syncwarp();
       }
@@ -226,7 +234,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   } else if (warp == 1) {
     // ================= MMA issuer (whole warp converged; one elected lane issues)
     const bool leader = elect_one();
-    const uint32_t idS = idesc_tf32(128, kTcTileS);
+    const uint32_t idS = idesc_tf32(128, TS);
     const uint32_t idV = idesc_tf32(128, RC);
     const int nprod = args.three ? 3 : 1;
     const bool skip_v = args.dbg_skip_v != 0;
@@ -269,7 +277,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     int prev_st = 0;
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
       const int bq = q & 1;
-      const uint32_t dS = tbase + (bq ? kColS1 : kColS0);
+      const uint32_t dS = tbase + (bq ? (uint32_t)TS : 0u);
       if constexpr (VCC) {
         if (q >= 2) {  // the epilogue has read S(q-2) out of this buffer
           mbar_wait(&sempty[bq], (uint32_t)(((q - 2) >> 1) & 1));
@@ -286,9 +294,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 #pragma unroll
         for (int ks = 0; ks < kTcKC / 8; ++ks) {
           const uint64_t aH = d0 + (uint64_t)((ks * 32) >> 4);
-          const uint64_t aL = d0 + (uint64_t)((kChunkBytes + ks * 32) >> 4);
-          const uint64_t bH = d0 + (uint64_t)((2 * kChunkBytes + ks * 32) >> 4);
-          const uint64_t bL = d0 + (uint64_t)((3 * kChunkBytes + ks * 32) >> 4);
+          const uint64_t aL = d0 + (uint64_t)((kChunkA + ks * 32) >> 4);
+          const uint64_t bH = d0 + (uint64_t)((2 * kChunkA + ks * 32) >> 4);
+          const uint64_t bL = d0 + (uint64_t)((2 * kChunkA + kChunkB + ks * 32) >> 4);
           const uint32_t acc0 = (kc > 0 || ks > 0) ? 1u : 0u;
           if (leader) {
             if (args.three) {
@@ -342,23 +350,24 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       mbar_wait(&wfull[q & 1], use & 1);
       mbar_wait(&sfull[bq], use & 1);
       tc_fence_after();
-      const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC) +
-                                                       2 * TcSmem::wslot(RC));
-      const float* w0s = nas + 128;
-      const uint32_t colS = bq ? kColS1 : kColS0;
-      uint32_t sv[2][CB];
-      tmem_ldn<CB>(tbase + lane_off + colS + CB * h, sv[0]);
-      tmem_ldn<CB>(tbase + lane_off + colS + 64 + CB * h, sv[1]);
-      tmem_wait_ld();
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&sempty[bq]);  // S buffer may be overwritten now
+      const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC));
+      const float* w0s = nas + TS;
+      const uint32_t colS = bq ? (uint32_t)TS : 0u;
+      constexpr int CW = TS / SUB;          // columns per warp (64)
       float vt = 0.f;
 #pragma unroll
       for (int hh = 0; hh < 2; ++hh) {
-        const int c0 = 64 * hh + CB * h;
+        const int c0 = CW * h + 32 * hh;
+        uint32_t sv[32];
+        tmem_ldn<32>(tbase + lane_off + colS + c0, sv);
+        tmem_wait_ld();
+        if (hh == 1) {
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&sempty[bq]);  // S buffer may be overwritten now
+        }
 #pragma unroll
-        for (int i = 0; i < CB; i += 4) {
+        for (int i = 0; i < 32; i += 4) {
           const float4 w4 = *reinterpret_cast<const float4*>(w0s + c0 + i);
           const float wv[4] = {w4.x, w4.y, w4.z, w4.w};
           float nav[4] = {0.f, 0.f, 0.f, 0.f};
@@ -368,7 +377,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           }
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
-            const float t = fminf(__uint_as_float(sv[hh][i + e]) + nav[e], 0.f);  // clamp d^2 >= 0
+            const float t = fminf(__uint_as_float(sv[i + e]) + nav[e], 0.f);  // clamp d^2 >= 0
             vt = fmaf(ex2_approx(t), wv[e], vt);
           }
         }
@@ -521,7 +530,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         if (!args.aug) nbj = __ldg(args.nb + cu.tt * kTcTileT + row);
       }
       const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC) +
-                                                       2 * TcSmem::wslot(RC));
+                                                       TcSmem::na_off(RC));
       const uint32_t colS = bq ? kColS1 : kColS0;
 #pragma unroll 1
       for (int hh = 0; hh < 2; ++hh) {
@@ -690,17 +699,18 @@ static int tc_stages(int r_c) {
 size_t fused_tc_smem(int r_c) {
   const int ns = tc_stages(r_c);
   switch (ns) {
-    case 3: return r_c <= 16 ? TcSmemT<3>::total(16) : TcSmemT<3>::total(32);
-    case 4: return r_c <= 16 ? TcSmemT<4>::total(16) : TcSmemT<4>::total(32);
-    default: return r_c <= 16 ? TcSmemT<5>::total(16) : TcSmemT<4>::total(32);
+    case 3: return r_c <= 16 ? TcSmemT<3, 128, false>::total(16) : TcSmemT<3, 128, false>::total(32);
+    case 4: return r_c <= 16 ? TcSmemT<4, 128, false>::total(16) : TcSmemT<4, 128, false>::total(32);
+    default: return r_c <= 16 ? TcSmemT<5, 128, false>::total(16) : TcSmemT<4, 128, false>::total(32);
   }
 }
 int fused_tc_stages() { return tc_stages(16); }
+int fused_tc_tile_s(int vcc) { return vcc ? 256 : kTcTileS; }
 
 template <int RC, int NS, bool VCC>
 static cudaError_t launch_rcsv(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
   static bool attr_done = false;
-  const size_t smem = TcSmemT<NS>::total(RC);
+  const size_t smem = TcSmemT<NS, VCC ? 256 : kTcTileS, VCC>::total(RC);
   if (!attr_done) {
     cudaError_t e = cudaFuncSetAttribute(ks_fused_tc_kernel<RC, NS, VCC>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -713,7 +723,7 @@ static cudaError_t launch_rcsv(const CUtensorMap* m, const TcArgs& a, cudaStream
 
 template <int RC, int NS>
 static cudaError_t launch_rcs(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
-  if (RC == 16 && a.vcc) return launch_rcsv<RC, NS, true>(m, a, st);
+  if (RC == 16 && a.vcc) return launch_rcsv<RC, 4, true>(m, a, st);  // 48 KB stages: 4 fit
   return launch_rcsv<RC, NS, false>(m, a, st);
 }
 

@@ -97,6 +97,7 @@ cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, 
 // maps: A_hi, A_lo (targets), B_hi, B_lo (sources), W_hi, W_lo (weights^T)
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st);
 int fused_tc_stages();
+int fused_tc_tile_s(int vcc);  // sources per tile: 256 in the R == 1 mode, 128 otherwise
 size_t fused_tc_smem(int r_c);
 
 }  // namespace ks
