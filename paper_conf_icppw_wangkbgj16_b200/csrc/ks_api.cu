@@ -388,6 +388,10 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.w0 = ctx->w0.p;
   a.vcc = ctx->tc_vcc;
   {
+    const char* e = getenv("KS_TC_WSLOTS");  // measurement knob
+    a.wslots = (e && e[0] >= '2' && e[0] <= '4') ? (e[0] - '0') : 0;
+  }
+  {
     const char* e = getenv("KS_TC_DEBUG_SKIP_V");
     a.dbg_skip_v = (e && e[0] == '1') ? 1 : 0;
   }

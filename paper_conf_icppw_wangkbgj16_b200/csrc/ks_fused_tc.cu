@@ -55,7 +55,8 @@ struct TcSmemT {
     return VCC ? ((uint32_t)(8 * TS) + 1023u) & ~1023u : (2 * wslot(r_c) + 512 + 1023) & ~1023u;
   }
   static constexpr uint32_t na_off(int r_c) { return VCC ? 0u : 2 * wslot(r_c); }
-  static constexpr uint32_t bar_off(int r_c) { return kW0 + 2 * w_slot_bytes(r_c); }
+  static constexpr int kWSlots = VCC ? 4 : 2;  // W/na ring depth
+  static constexpr uint32_t bar_off(int r_c) { return kW0 + kWSlots * w_slot_bytes(r_c); }
   static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 256 + 4 * kTcTileT * 8; }  // + VCC scratch
 };
 
@@ -141,9 +142,12 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + TcSmem::bar_off(RC));
   uint64_t* full = bars;                 // [kStages]
   uint64_t* empty = full + kStages;      // [kStages]
-  uint64_t* wfull = empty + kStages;     // [2]
-  uint64_t* wempty = wfull + 2;          // [2]
-  uint64_t* sfull = wempty + 2;          // [2]
+  constexpr int WSA = TcSmem::kWSlots;   // allocated W/na slots
+  // measured: a 2-deep W/na ring is faster than 4 (KS_TC_WSLOTS knob)
+  const int WS = (VCC && args.wslots >= 2 && args.wslots <= WSA) ? args.wslots : 2;
+  uint64_t* wfull = empty + kStages;     // [WSA]
+  uint64_t* wempty = wfull + WSA;        // [WSA]
+  uint64_t* sfull = wempty + WSA;        // [2]
   uint64_t* pready = sfull + 2;          // [2 S buffers][2 source halves]
   uint64_t* vdone = pready + 4;          // [2 source halves]
   uint64_t* sempty = vdone + 2;          // [2] (VCC: epilogue has read the S buffer)
@@ -168,9 +172,11 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       mbar_init(&full[i], 1);
       mbar_init(&empty[i], 1);
     }
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < WSA; ++i) {
       mbar_init(&wfull[i], 1);
       mbar_init(&wempty[i], VCC ? EW : 1);
+    }
+    for (int i = 0; i < 2; ++i) {
       mbar_init(&sempty[i], EW);
       mbar_init(&sfull[i], 1);
       mbar_init(&vdone[i], 1);
@@ -198,8 +204,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
       const int tt = (int)cu.tt, st = cu.st;
       {
-        const int slot = q & 1;
-        const uint32_t use = (uint32_t)(q >> 1);
+        const int slot = q % WS;
+        const uint32_t use = (uint32_t)(q / WS);
         mbar_wait(&wempty[slot], (use & 1) ^ 1);
         uint8_t* ws = smem + TcSmem::kW0 + slot * TcSmem::w_slot_bytes(RC);
         if (leader) {
@@ -347,10 +353,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         seg_st0 = cu.st;
         if (!args.aug) nbj = __ldg(args.nb + cu.tt * kTcTileT + row);
       }
-      mbar_wait(&wfull[q & 1], use & 1);
+      mbar_wait(&wfull[q % WS], (uint32_t)((q / WS) & 1));
       mbar_wait(&sfull[bq], use & 1);
       tc_fence_after();
-      const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC));
+      const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q % WS) * TcSmem::w_slot_bytes(RC));
       const float* w0s = nas + TS;
       const uint32_t colS = bq ? (uint32_t)TS : 0u;
       constexpr int CW = TS / SUB;          // columns per warp (64)
@@ -383,7 +389,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         }
       }
       __syncwarp();
-      if (lane == 0) mbar_arrive(&wempty[q & 1]);  // na / W slot consumed
+      if (lane == 0) mbar_arrive(&wempty[q % WS]);  // na / W slot consumed
       vacc += (double)vt;
       const bool seg_end = (q == count - 1) || (cu.st + 1 == n_s);
       if (seg_end) {

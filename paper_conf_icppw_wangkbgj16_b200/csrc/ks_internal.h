@@ -74,6 +74,7 @@ struct TcArgs {
   int aug;              // 1: norms folded into the contraction (2 extra K columns), epilogue adds nothing
   int vcc;              // 1: R == 1, weighted sum on CUDA cores (w0 used, no W^T tiles, no V MMA)
   const float* w0;      // [m_pad] W[:, 0] (vcc)
+  int wslots;           // VCC W/na ring depth (2..4; 0 = default)
   int dbg_skip_v;       // measurement only (KS_TC_DEBUG_SKIP_V=1): do not issue the V MMAs (wrong results)
   const float* na;      // [m_pad]  -c ||alpha_hat||^2
   const float* nb;      // [n_pad]  -c ||beta_hat||^2
