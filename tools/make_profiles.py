@@ -11,7 +11,7 @@ dst = os.path.join("profiles", rnd)
 os.makedirs(dst, exist_ok=True)
 summ_path = os.path.join("profiles", "ncu_summary.json")
 summ = json.load(open(summ_path)) if os.path.exists(summ_path) else {}
-for c in cfgs:
+for c in cfgs:   # "3", "4", "3_fp32", ... -> prof_cfg<c>.ncu-rep
     rep = os.path.join(src, f"prof_cfg{c}.ncu-rep")
     if os.path.exists(rep):
         out = subprocess.run([sys.executable, "tools/ncu_summary.py", rep], capture_output=True, text=True).stdout
