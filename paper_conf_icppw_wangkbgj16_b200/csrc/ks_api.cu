@@ -119,11 +119,11 @@ struct ks_ctx {
   int R = 1;
   DBuf<float> src;        // FP32 path: [k_pad + 2][m_pad]
   // TC path (tcgen05): TF32 hi/lo operand splits, norms, W^T splits
-  DBuf<float> src_hi, src_lo, na, wt_hi, wt_lo, w0;
+  DBuf<float> src_hi, src_lo, na, wt_hi, wt_lo, wv;
   DBuf<float> tgt_hi, tgt_lo, nb;
   int r_pad = 16;
   int tc_aug = 0;  // norms folded into the contraction as 2 extra K columns
-  int tc_vcc = 0;  // R == 1: weighted sum on CUDA cores (W^T tiles not needed)
+  int tc_vcc = 0;  // RV: weighted sum on CUDA cores over RV padded columns (0: tensor-core V path)
   CUtensorMap tmB_hi, tmB_lo;
   DBuf<float> mu;         // [k_pad]
   DBuf<double> mean_part; // [nparts][K]
@@ -314,7 +314,7 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   const int aug = tc_aug(K);
   // R == 1: weighted sum on CUDA cores (KS_TC_VCC=0 forces the tensor-core V path; measurement knob)
   const char* ev = getenv("KS_TC_VCC");
-  const int vcc = (R == 1 && !(ev && ev[0] == '0')) ? 1 : 0;
+  const int vcc = (ev && ev[0] == '0') ? 0 : ks::fused_tc_rv(R);
   const int tile_s = ks::fused_tc_tile_s(vcc);
   const int64_t m_pad = round_up(M > 0 ? M : 1, tile_s);
   const int r_pad = (int)round_up(R, 16);
@@ -325,7 +325,7 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(ctx->na.reserve((size_t)m_pad, st, false), "allocate source norms");
   KS_CUDA(ctx->wt_hi.reserve(nw, st, false), "allocate W hi");
   KS_CUDA(ctx->wt_lo.reserve(nw, st, false), "allocate W lo");
-  KS_CUDA(ctx->w0.reserve((size_t)m_pad, st, false), "allocate W column 0");
+  KS_CUDA(ctx->wv.reserve((size_t)m_pad * (vcc ? vcc : 1), st, false), "allocate W rows");
   KS_CUDA(ctx->mu.reserve(k_pad, st, false), "allocate mean buffer");
   int nparts = (int)((M + 63) / 64);  // source-mean blocks of <= 64 rows each
   if (nparts < 1) nparts = 1;
@@ -334,7 +334,7 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(ks::launch_source_mean(alpha, M, K, k_pad, ctx->mean_part.p, nparts, ctx->mu.p, st), "source mean");
   ctx->launches += (M > 0) ? 2 : 1;
   KS_CUDA(ks::launch_prep_tc_sources(alpha, W, M, m_pad, K, k_pad, R, vcc ? 0 : r_pad, ctx->mu.p, ctx->c, aug,
-                                     ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p, ctx->w0.p, st),
+                                     ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p, ctx->wv.p, vcc, st),
           "source prep (TC)");
   ctx->launches += 1;
   ks_status s = encode_2d_sw64(&ctx->tmB_hi, ctx->src_hi.p, k_pad, m_pad, tile_s);
@@ -385,7 +385,7 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.R = ctx->R;
   a.three = (ctx->prec_eff == KS_PREC_TF32) ? 0 : 1;
   a.aug = ctx->tc_aug;
-  a.w0 = ctx->w0.p;
+  a.wv = ctx->wv.p;
   a.vcc = ctx->tc_vcc;
   {
     const char* e = getenv("KS_TC_WSLOTS");  // measurement knob
@@ -496,7 +496,7 @@ ks_status ks_destroy(ks_ctx* ctx) {
   set_device(ctx);
   cudaStreamSynchronize(ctx->stream);
   ctx->src.release();
-  for (DBuf<float>* bptr : {&ctx->src_hi, &ctx->src_lo, &ctx->na, &ctx->wt_hi, &ctx->wt_lo, &ctx->w0, &ctx->tgt_hi,
+  for (DBuf<float>* bptr : {&ctx->src_hi, &ctx->src_lo, &ctx->na, &ctx->wt_hi, &ctx->wt_lo, &ctx->wv, &ctx->tgt_hi,
                             &ctx->tgt_lo, &ctx->nb})
     bptr->release();
   ctx->mu.release();

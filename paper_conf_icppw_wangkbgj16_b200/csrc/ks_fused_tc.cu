@@ -42,20 +42,22 @@ constexpr uint32_t kChunkA = kTcTileT * kTcKC * 4;  // one hi or lo target-opera
 constexpr uint32_t kColS0 = 0, kColS1 = 128, kColPlo = 256, kColV = 384;
 
 // Shared-memory layout (bytes from a 1 KB-aligned base).  TS = sources per
-// tile (128 with the tensor-core V path, 256 in the R == 1 VCC mode).
-template <int kStages, int TS, bool VCC>
+// tile (128 with the tensor-core V path, 256 when the weighted sum runs on CUDA
+// cores, RV = padded weight columns of that mode, 0 = tensor-core V path).
+template <int kStages, int TS, int RV>
 struct TcSmemT {
+  static constexpr bool VCC = RV > 0;
   static constexpr uint32_t kChunkB = TS * kTcKC * 4;                 // one hi or lo source chunk
   static constexpr uint32_t kStageBytes = 2 * kChunkA + 2 * kChunkB;  // A_hi, A_lo, B_hi, B_lo
   static constexpr uint32_t kStage0 = 0;
   static constexpr uint32_t wslot(int r_c) { return (uint32_t)r_c * 512u; }  // one of W^T hi/lo: 8 chunks x r_c x 64 B
   static constexpr uint32_t kW0 = kStages * kStageBytes;
-  // VCC: na[TS] | w0[TS];  else W^T hi | W^T lo | na[128].  Slots 1 KB aligned (SWIZZLE_64B atoms).
+  // VCC: na[TS] | W[TS][RV];  else W^T hi | W^T lo | na[128].  Slots 1 KB aligned (SWIZZLE_64B atoms).
   static constexpr uint32_t w_slot_bytes(int r_c) {
-    return VCC ? ((uint32_t)(8 * TS) + 1023u) & ~1023u : (2 * wslot(r_c) + 512 + 1023) & ~1023u;
+    return VCC ? ((uint32_t)(4 * TS * (1 + RV)) + 1023u) & ~1023u : (2 * wslot(r_c) + 512 + 1023) & ~1023u;
   }
   static constexpr uint32_t na_off(int r_c) { return VCC ? 0u : 2 * wslot(r_c); }
-  static constexpr int kWSlots = VCC ? 4 : 2;  // W/na ring depth
+  static constexpr int kWSlots = VCC && RV < 8 ? 4 : 2;  // W/na ring depth (RV >= 8: 2 to fit 4 stages)
   static constexpr uint32_t bar_off(int r_c) { return kW0 + kWSlots * w_slot_bytes(r_c); }
   static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 256 + 4 * kTcTileT * 8; }  // + VCC scratch
 };
@@ -120,17 +122,19 @@ __device__ __forceinline__ void unit_next(const Sched& s, UnitIt& u) {
 
 }  // namespace
 
-// VCC: R == 1 -- the weighted reduction runs on CUDA cores in the epilogue
-// (one FFMA per pair, W_i broadcast from shared memory) instead of a second
-// tensor-core contraction; no P_hi/P_lo stores, no V MMA.
-template <int RC, int kStages, bool VCC>
+// RV > 0 ("VCC", R <= 16): the weighted reduction runs on CUDA cores in the
+// epilogue (R FMAs per pair, W_i broadcast from shared memory) instead of a
+// second tensor-core contraction: no P_hi/P_lo stores, no V MMA, and 256-source
+// tiles (two 256-column S buffers fill TMEM).
+template <int RC, int kStages, int RV>
 __global__ void __launch_bounds__(kTcThreads, 1)
     ks_fused_tc_kernel(const __grid_constant__ CUtensorMap mA_hi, const __grid_constant__ CUtensorMap mA_lo,
                        const __grid_constant__ CUtensorMap mB_hi, const __grid_constant__ CUtensorMap mB_lo,
                        const __grid_constant__ CUtensorMap mW_hi, const __grid_constant__ CUtensorMap mW_lo,
                        const TcArgs args) {
+  constexpr bool VCC = RV > 0;
   constexpr int TS = VCC ? 256 : kTcTileS;  // sources per tile
-  using TcSmem = TcSmemT<kStages, TS, VCC>;
+  using TcSmem = TcSmemT<kStages, TS, RV>;
   constexpr uint32_t kChunkB = TcSmem::kChunkB;
   constexpr uint32_t kStageBytes = TcSmem::kStageBytes;
   constexpr int EW = kTcEpiWarps;        // epilogue warps
@@ -209,10 +213,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         mbar_wait(&wempty[slot], (use & 1) ^ 1);
         uint8_t* ws = smem + TcSmem::kW0 + slot * TcSmem::w_slot_bytes(RC);
         if (leader) {
-          if constexpr (VCC) {  // na and the single weight column
-            mbar_arrive_expect_tx(&wfull[slot], 8 * TS);
+          if constexpr (VCC) {  // na and the tile's weight rows
+            mbar_arrive_expect_tx(&wfull[slot], 4 * TS * (1 + RV));
             bulk_load(ws, args.na + (int64_t)st * TS, 4 * TS, &wfull[slot]);
-            bulk_load(ws + 4 * TS, args.w0 + (int64_t)st * TS, 4 * TS, &wfull[slot]);
+            bulk_load(ws + 4 * TS, args.wv + (int64_t)st * TS * RV, 4 * TS * RV, &wfull[slot]);
           } else {
             mbar_arrive_expect_tx(&wfull[slot], 2 * TcSmem::wslot(RC) + 512);
             tma_load_3d(ws, &mW_hi, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
@@ -335,14 +339,21 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       }
     }
   } else if (VCC && warp >= 4) {
-    // ================= epilogue, R == 1: V on CUDA cores
+    // ================= epilogue, R <= 16: V on CUDA cores
     const int ew = warp - 4;
     const int g = ew & 3;                 // TMEM lanes 32g..32g+31
-    const int h = ew >> 2;                // columns 64hh + CB h .. + CB-1 of each source half hh
+    const int h = ew >> 2;                // columns CW h .. CW h + CW - 1 of the tile
     const int row = 32 * g + lane;        // target row within the tile
     const uint32_t lane_off = (uint32_t)(32 * g) << 16;
+    constexpr int CW = TS / SUB;          // columns per warp (64)
+    constexpr int BC = (RV >= 8) ? 16 : 32;  // TMEM columns per load batch (register budget)
     double* red = reinterpret_cast<double*>(smem + TcSmem::bar_off(RC) + 256);  // [SUB][128]
-    double vacc = 0.0;
+    constexpr int RVA = RV > 0 ? RV : 1;  // (this branch only runs with RV > 0)
+    double vacc[RVA];
+    float vblk[RVA];                      // FP32 sums over <= 8 tiles
+#pragma unroll
+    for (int r = 0; r < RVA; ++r) { vacc[r] = 0.0; vblk[r] = 0.f; }
+    int nblk = 0;
     float nbj = 0.f;
     int seg_q = 0, seg_st0 = 0;
     UnitIt cu = unit_begin(sc);
@@ -357,82 +368,111 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       mbar_wait(&sfull[bq], use & 1);
       tc_fence_after();
       const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q % WS) * TcSmem::w_slot_bytes(RC));
-      const float* w0s = nas + TS;
+      const float* wvs = nas + TS;        // [TS][RV]
       const uint32_t colS = bq ? (uint32_t)TS : 0u;
-      constexpr int CW = TS / SUB;          // columns per warp (64)
-      float vt = 0.f;
 #pragma unroll
-      for (int hh = 0; hh < 2; ++hh) {
-        const int c0 = CW * h + 32 * hh;
-        uint32_t sv[32];
-        tmem_ldn<32>(tbase + lane_off + colS + c0, sv);
+      for (int hh = 0; hh < CW / BC; ++hh) {
+        const int c0 = CW * h + BC * hh;
+        uint32_t sv[BC];
+        tmem_ldn<BC>(tbase + lane_off + colS + c0, sv);
         tmem_wait_ld();
-        if (hh == 1) {
+        if (hh == CW / BC - 1) {
           tc_fence_before();
           __syncwarp();
           if (lane == 0) mbar_arrive(&sempty[bq]);  // S buffer may be overwritten now
         }
 #pragma unroll
-        for (int i = 0; i < 32; i += 4) {
-          const float4 w4 = *reinterpret_cast<const float4*>(w0s + c0 + i);
-          const float wv[4] = {w4.x, w4.y, w4.z, w4.w};
+        for (int i = 0; i < BC; i += 4) {
           float nav[4] = {0.f, 0.f, 0.f, 0.f};
           if (!args.aug) {
             const float4 na4 = *reinterpret_cast<const float4*>(nas + c0 + i);
             nav[0] = na4.x + nbj; nav[1] = na4.y + nbj; nav[2] = na4.z + nbj; nav[3] = na4.w + nbj;
           }
+          if constexpr (RV == 1) {
+            const float4 w4 = *reinterpret_cast<const float4*>(wvs + c0 + i);
+            const float wv[4] = {w4.x, w4.y, w4.z, w4.w};
 #pragma unroll
-          for (int e = 0; e < 4; ++e) {
-            const float t = fminf(__uint_as_float(sv[i + e]) + nav[e], 0.f);  // clamp d^2 >= 0
-            vt = fmaf(ex2_approx(t), wv[e], vt);
+            for (int e = 0; e < 4; ++e) {
+              const float t = fminf(__uint_as_float(sv[i + e]) + nav[e], 0.f);  // clamp d^2 >= 0
+              vblk[0] = fmaf(ex2_approx(t), wv[e], vblk[0]);
+            }
+          } else {
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const float t = fminf(__uint_as_float(sv[i + e]) + nav[e], 0.f);  // clamp d^2 >= 0
+              const float pk = ex2_approx(t);
+              const float* wrow = wvs + (c0 + i + e) * RVA;
+#pragma unroll
+              for (int r4 = 0; r4 < RVA; r4 += 4) {
+                const float4 w4 = *reinterpret_cast<const float4*>(wrow + r4);
+                vblk[r4 + 0] = fmaf(pk, w4.x, vblk[r4 + 0]);
+                vblk[r4 + 1] = fmaf(pk, w4.y, vblk[r4 + 1]);
+                vblk[r4 + 2] = fmaf(pk, w4.z, vblk[r4 + 2]);
+                vblk[r4 + 3] = fmaf(pk, w4.w, vblk[r4 + 3]);
+              }
+            }
           }
         }
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&wempty[q % WS]);  // na / W slot consumed
-      vacc += (double)vt;
       const bool seg_end = (q == count - 1) || (cu.st + 1 == n_s);
-      if (seg_end) {
-        // combine the SUB column groups of each row in a fixed order
-        red[h * kTcTileT + row] = vacc;
-        named_bar_sync(1, 32 * EW);
-        if (h == 0) {
-          double v = 0.0;
+      if (++nblk == 8 || seg_end) {  // FP32 over <= 8 tiles, then FP64
 #pragma unroll
-          for (int k = 0; k < SUB; ++k) v += red[k * kTcTileT + row];
-          const int seg_len = q - seg_q + 1;
-          const bool whole = (seg_st0 == 0) && (seg_len == n_s);
-          const int64_t grow = cu.tt * kTcTileT + row;
-          if (whole) {
-            if (grow < args.N) args.V[grow * args.R + args.r_off] = (float)v;
-          } else {
-            const int64_t tr = cu.tt - sc.rem_t0;
-            const int slot = (tr == sc.v0 / n_s) ? 0 : 1;
-            args.partial[(b * 2 + slot) * kTcTileT + row] = (float)v;
-            __threadfence();
-            named_bar_sync(2, 128);
-            const int64_t b_first = sk_owner(tr * n_s, sc.Urem, sc.Gr);
-            const int64_t b_last = sk_owner(tr * n_s + n_s - 1, sc.Urem, sc.Gr);
-            if (row == 0) {
-              const int old = atomicAdd(&args.counters[cu.tt], 1);
-              const int last = (old == (int)(b_last - b_first));
-              if (last) args.counters[cu.tt] = 0;
-              *flag = last;
+        for (int r = 0; r < RVA; ++r) { vacc[r] += (double)vblk[r]; vblk[r] = 0.f; }
+        nblk = 0;
+      }
+      if (seg_end) {
+        const int seg_len = q - seg_q + 1;
+        const bool whole = (seg_st0 == 0) && (seg_len == n_s);
+        const int64_t grow = cu.tt * kTcTileT + row;
+        const int64_t tr = cu.tt - sc.rem_t0;
+        const int slot = (!whole && tr == sc.v0 / n_s) ? 0 : 1;
+        // combine the SUB column groups of each row, column by column, in a fixed order
+#pragma unroll 1
+        for (int r = 0; r < RVA; ++r) {
+          red[h * kTcTileT + row] = vacc[r];
+          named_bar_sync(1, 32 * EW);
+          if (h == 0) {
+            double v = 0.0;
+#pragma unroll
+            for (int k = 0; k < SUB; ++k) v += red[k * kTcTileT + row];
+            if (whole) {
+              if (grow < args.N && r < args.r_valid) args.V[grow * args.R + args.r_off + r] = (float)v;
+            } else {
+              args.partial[((b * 2 + slot) * kTcTileT + row) * RVA + r] = (float)v;
             }
-            named_bar_sync(2, 128);
-            if (*flag) {
-              __threadfence();
+          }
+          named_bar_sync(1, 32 * EW);  // red reuse
+        }
+        if (!whole && h == 0) {
+          __threadfence();
+          named_bar_sync(2, 128);
+          const int64_t b_first = sk_owner(tr * n_s, sc.Urem, sc.Gr);
+          const int64_t b_last = sk_owner(tr * n_s + n_s - 1, sc.Urem, sc.Gr);
+          if (row == 0) {
+            const int old = atomicAdd(&args.counters[cu.tt], 1);
+            const int last = (old == (int)(b_last - b_first));
+            if (last) args.counters[cu.tt] = 0;
+            *flag = last;
+          }
+          named_bar_sync(2, 128);
+          if (*flag) {
+            __threadfence();
+#pragma unroll 1
+            for (int r = 0; r < RVA; ++r) {
               float sum = 0.f;
               for (int64_t bb = b_first; bb <= b_last; ++bb) {
                 const int sl = (tr == sk_start(bb, sc.Urem, sc.Gr) / n_s) ? 0 : 1;
-                sum += __ldcg(args.partial + (bb * 2 + sl) * kTcTileT + row);
+                sum += __ldcg(args.partial + ((bb * 2 + sl) * kTcTileT + row) * RVA + r);
               }
-              if (grow < args.N) args.V[grow * args.R + args.r_off] = sum;
+              if (grow < args.N && r < args.r_valid) args.V[grow * args.R + args.r_off + r] = sum;
             }
           }
+          named_bar_sync(2, 128);  // flag reuse
         }
-        named_bar_sync(1, 32 * EW);  // red / flag reuse
-        vacc = 0.0;
+#pragma unroll
+        for (int r = 0; r < RVA; ++r) vacc[r] = 0.0;
         seg_q = q + 1;
       }
     }
@@ -609,7 +649,7 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
                                        const float* __restrict__ mu, double c, int aug, float* __restrict__ src_hi,
                                        float* __restrict__ src_lo, float* __restrict__ na,
                                        float* __restrict__ wt_hi, float* __restrict__ wt_lo,
-                                       float* __restrict__ w0) {
+                                       float* __restrict__ wv, int rv) {
   const int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   if (i >= m_pad) return;
@@ -636,10 +676,8 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
     src_hi[i * k_pad + d] = ah;
     src_lo[i * k_pad + d] = to_tf32(a - ah);
   }
-  if (lane == 0) {
-    na[i] = nai;
-    w0[i] = live ? W[i * R] : 0.f;
-  }
+  if (lane == 0) na[i] = nai;
+  for (int r = lane; r < rv; r += 32) wv[i * rv + r] = (live && r < R) ? W[i * R + r] : 0.f;
   for (int r = lane; r < r_pad; r += 32) {
     const float w = (live && r < R) ? W[i * R + r] : 0.f;
     const float wh = to_tf32(w);
@@ -676,12 +714,12 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
 
 cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
                                    int R, int r_pad, const float* mu, double c, int aug, float* src_hi,
-                                   float* src_lo, float* na, float* wt_hi, float* wt_lo, float* w0,
+                                   float* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv, int rv,
                                    cudaStream_t st) {
   if (m_pad == 0) return cudaSuccess;
   const int bs = 256;  // 8 points per block
   prep_tc_sources_kernel<<<(unsigned)((m_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
-      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, src_hi, src_lo, na, wt_hi, wt_lo, w0);
+      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv);
   return cudaGetLastError();
 }
 
@@ -705,47 +743,52 @@ static int tc_stages(int r_c) {
 size_t fused_tc_smem(int r_c) {
   const int ns = tc_stages(r_c);
   switch (ns) {
-    case 3: return r_c <= 16 ? TcSmemT<3, 128, false>::total(16) : TcSmemT<3, 128, false>::total(32);
-    case 4: return r_c <= 16 ? TcSmemT<4, 128, false>::total(16) : TcSmemT<4, 128, false>::total(32);
-    default: return r_c <= 16 ? TcSmemT<5, 128, false>::total(16) : TcSmemT<4, 128, false>::total(32);
+    case 3: return r_c <= 16 ? TcSmemT<3, 128, 0>::total(16) : TcSmemT<3, 128, 0>::total(32);
+    case 4: return r_c <= 16 ? TcSmemT<4, 128, 0>::total(16) : TcSmemT<4, 128, 0>::total(32);
+    default: return r_c <= 16 ? TcSmemT<5, 128, 0>::total(16) : TcSmemT<4, 128, 0>::total(32);
   }
 }
 int fused_tc_stages() { return tc_stages(16); }
-int fused_tc_tile_s(int vcc) { return vcc ? 256 : kTcTileS; }
+int fused_tc_tile_s(int rv) { return rv ? 256 : kTcTileS; }
+int fused_tc_rv(int R) { return R <= 1 ? 1 : R <= 2 ? 2 : R <= 4 ? 4 : R <= 8 ? 8 : R <= 16 ? 16 : 0; }
 
-template <int RC, int NS, bool VCC>
+template <int RC, int NS, int RV>
 static cudaError_t launch_rcsv(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
   static bool attr_done = false;
-  const size_t smem = TcSmemT<NS, VCC ? 256 : kTcTileS, VCC>::total(RC);
+  const size_t smem = TcSmemT<NS, RV ? 256 : kTcTileS, RV>::total(RC);
+  static_assert(TcSmemT<NS, RV ? 256 : kTcTileS, RV>::total(RC) <= 232448, "exceeds 227 KB of shared memory");
   if (!attr_done) {
-    cudaError_t e = cudaFuncSetAttribute(ks_fused_tc_kernel<RC, NS, VCC>,
+    cudaError_t e = cudaFuncSetAttribute(ks_fused_tc_kernel<RC, NS, RV>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr_done = true;
   }
-  ks_fused_tc_kernel<RC, NS, VCC><<<a.sk.grid, kTcThreads, smem, st>>>(m[0], m[1], m[2], m[3], m[4], m[5], a);
+  ks_fused_tc_kernel<RC, NS, RV><<<a.sk.grid, kTcThreads, smem, st>>>(m[0], m[1], m[2], m[3], m[4], m[5], a);
   return cudaGetLastError();
 }
 
-template <int RC, int NS>
-static cudaError_t launch_rcs(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
-  if (RC == 16 && a.vcc) return launch_rcsv<RC, 4, true>(m, a, st);  // 48 KB stages: 4 fit
-  return launch_rcsv<RC, NS, false>(m, a, st);
-}
-
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st) {
+  // CUDA-core weighted sum (256-source tiles): 48 KB stages, 4 fit (3 with the 16 KB weight slots)
+  switch (a.vcc) {
+    case 1: return launch_rcsv<16, 4, 1>(maps, a, st);
+    case 2: return launch_rcsv<16, 4, 2>(maps, a, st);
+    case 4: return launch_rcsv<16, 4, 4>(maps, a, st);
+    case 8: return launch_rcsv<16, 4, 8>(maps, a, st);
+    case 16: return launch_rcsv<16, 3, 16>(maps, a, st);
+    default: break;
+  }
   const int ns = tc_stages(a.r_c);
   if (a.r_c == 16) {
     switch (ns) {
-      case 3: return launch_rcs<16, 3>(maps, a, st);
-      case 4: return launch_rcs<16, 4>(maps, a, st);
-      default: return launch_rcs<16, 5>(maps, a, st);
+      case 3: return launch_rcsv<16, 3, 0>(maps, a, st);
+      case 4: return launch_rcsv<16, 4, 0>(maps, a, st);
+      default: return launch_rcsv<16, 5, 0>(maps, a, st);
     }
   }
   if (a.r_c == 32) {
     switch (ns) {
-      case 3: return launch_rcs<32, 3>(maps, a, st);
-      default: return launch_rcs<32, 4>(maps, a, st);
+      case 3: return launch_rcsv<32, 3, 0>(maps, a, st);
+      default: return launch_rcsv<32, 4, 0>(maps, a, st);
     }
   }
   return cudaErrorInvalidValue;

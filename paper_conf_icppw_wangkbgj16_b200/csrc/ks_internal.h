@@ -72,8 +72,8 @@ struct TcArgs {
   int R;                // row stride of V
   int three;            // 1: 3xTF32 (hi.hi + hi.lo + lo.hi), 0: plain TF32 (hi.hi)
   int aug;              // 1: norms folded into the contraction (2 extra K columns), epilogue adds nothing
-  int vcc;              // 1: R == 1, weighted sum on CUDA cores (w0 used, no W^T tiles, no V MMA)
-  const float* w0;      // [m_pad] W[:, 0] (vcc)
+  int vcc;              // RV > 0: weighted sum on CUDA cores over RV padded columns (no W^T tiles, no V MMA)
+  const float* wv;      // [m_pad][RV] weights, zero padded (vcc)
   int wslots;           // VCC W/na ring depth (2..4; 0 = default)
   int dbg_skip_v;       // measurement only (KS_TC_DEBUG_SKIP_V=1): do not issue the V MMAs (wrong results)
   const float* na;      // [m_pad]  -c ||alpha_hat||^2
@@ -90,7 +90,8 @@ struct TcArgs {
 // aug: columns K, K+1 hold (1, na_i) so that S already contains the norms
 cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
                                    int R, int r_pad, const float* mu, double c, int aug, float* src_hi,
-                                   float* src_lo, float* na, float* wt_hi, float* wt_lo, float* w0, cudaStream_t st);
+                                   float* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv, int rv,
+                                   cudaStream_t st);
 // targets: tgt_hi/lo [n_pad][k_pad] = TF32 split of (beta - mu), nb [n_pad]
 // aug: columns K, K+1 hold (nb_j, 1)
 cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
@@ -98,7 +99,8 @@ cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, 
 // maps: A_hi, A_lo (targets), B_hi, B_lo (sources), W_hi, W_lo (weights^T)
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st);
 int fused_tc_stages();
-int fused_tc_tile_s(int vcc);  // sources per tile: 256 in the R == 1 mode, 128 otherwise
+int fused_tc_tile_s(int rv);  // sources per tile: 256 with the CUDA-core weighted sum, 128 otherwise
+int fused_tc_rv(int R);       // padded weight columns of the CUDA-core weighted sum, 0 if R > 16
 size_t fused_tc_smem(int r_c);
 
 }  // namespace ks

@@ -55,7 +55,8 @@ def test_cfg4_tight_cluster_separates_tf32(oracle_mod):
     assert e1 > 10 * e3
 
 
-@pytest.mark.parametrize("K,R", [(33, 1), (48, 2), (64, 16), (100, 5), (255, 16), (300, 17), (40, 40),
+@pytest.mark.parametrize("K,R", [(33, 1), (48, 2), (64, 3), (40, 4), (64, 16), (100, 5), (96, 8), (72, 12),
+                                 (255, 16), (300, 17), (40, 40),
                                  (16, 33), (128, 64)])
 def test_shapes_k_r(oracle_mod, K, R):
     a, W, b, h = workloads.custom(1500 + K, 400 + R, K, R, 0.35 * np.sqrt(K), seed=K * 31 + R, wkind="signed")
@@ -110,3 +111,12 @@ def test_cfg4_full_size_sampled(oracle_mod):
     a, W, b, h = workloads.make(4)                                 # M = N = 262,144
     J = workloads.sample_targets(b.shape[0], 48, seed=44)
     check(oracle_mod, a, W, b, h, J=J)
+
+
+@pytest.mark.parametrize("R", [1, 16])
+def test_tensor_core_v_path(oracle_mod, monkeypatch, R):
+    """R <= 16 takes the CUDA-core weighted sum by default; KS_TC_VCC=0 keeps
+    the second (P x W) tcgen05 MMA of the R > 16 path on these shapes too."""
+    monkeypatch.setenv("KS_TC_VCC", "0")
+    a, W, b, h = workloads.custom(2100, 333, 64, R, 3.0, seed=11 + R, wkind="signed")
+    check(oracle_mod, a, W, b, h)
