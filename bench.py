@@ -313,12 +313,14 @@ def run_ours(args):
     max_mhz = clk_sum["sm_max_mhz"] or 1965
     if info1["path"] == ks.KS_PATH_TC:
         nprod = 3 if info1["precision"] == ks.KS_PREC_3XTF32 else 1
-        # R == 1: the weighted sum runs on CUDA cores, the tensor work is the 2K contraction
-        flops_pair = nprod * 2 * (K + (R if R > 1 else 0))
+        # R <= 16 (256-source tiles): the weighted sum runs on CUDA cores and the
+        # tensor work is the 2K contraction; R > 16: a second MMA adds 2R per pair
+        vcc = info1["tile_s"] == 256
+        flops_pair = nprod * 2 * (K + (0 if vcc else R))
         achieved = pairs_launch * flops_pair / (kms / 1e3) / 1e12
         bf16 = load_peaks().get("bf16_tflops")
         peak = (bf16 * 0.5) if bf16 else 1100.0
-        formula = "%d products x 2K per pair" % nprod if R == 1 else "%d products x 2(K+R) per pair" % nprod
+        formula = "%d products x 2K per pair" % nprod if vcc else "%d products x 2(K+R) per pair" % nprod
         roof = {"bound": "tensor", "kernel": "ks_fused_tc_kernel", "achieved": achieved, "peak": peak,
                 "unit": "TFLOP/s (TF32 tensor; %s)" % formula, "frac": achieved / peak,
                 "traffic": load_traffic(args.cfg, args.precision),
@@ -329,6 +331,12 @@ def run_ours(args):
         roof["sfu"] = {"achieved_ex2_per_s": pairs_launch / (kms / 1e3), "peak_ex2_per_s": sfu_peak,
                        "frac": pairs_launch / (kms / 1e3) / sfu_peak,
                        "peak_derivation": f"16 ex2/clk/SM x {sms} SMs x {max_mhz} MHz"}
+        if vcc:
+            # co-bound: CUDA-core epilogue, R FFMA (weighted sum) + 1 FADD (exponent) per pair
+            ops = pairs_launch * (R + 1) / (kms / 1e3) / 1e12
+            roof["fp32_epilogue"] = {"achieved": ops, "peak": 128 * sms * max_mhz * 1e6 / 1e12,
+                                     "unit": "Top/s FP32-pipe lane ops (R+1 per pair)",
+                                     "frac": ops / (128 * sms * max_mhz * 1e6 / 1e12)}
     else:
         fp32_ops, mufu = per_pair_ops(K, R)
         achieved = pairs_launch * fp32_ops / (kms / 1e3) / 1e12      # T FP32-pipe lane-ops / s

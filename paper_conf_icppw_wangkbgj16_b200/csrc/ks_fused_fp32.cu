@@ -66,37 +66,6 @@ __device__ __forceinline__ int64_t sk_start(int64_t b, int64_t U, int64_t G) { r
 // CTA that owns unit u: the largest b with floor(b*U/G) <= u.
 __device__ __forceinline__ int64_t sk_owner(int64_t u, int64_t U, int64_t G) { return ((u + 1) * G - 1) / U; }
 
-// ---------------------------------------------------------------- packed FP32x2 (FFMA2 / FADD2)
-// A pair holds two FP32 lanes (lo = element 0).  fma.rn.f32x2 / add.rn.f32x2
-// do two IEEE FP32 operations in one issue slot; a scalar operand packed as
-// {x, x} is encoded as a broadcast register operand (no extra move).
-typedef unsigned long long f2_t;
-
-__device__ __forceinline__ f2_t f2_bcast(float x) {
-  f2_t r;
-  asm("mov.b64 %0, {%1, %1};" : "=l"(r) : "f"(x));
-  return r;
-}
-__device__ __forceinline__ f2_t f2_pack(float lo, float hi) {
-  f2_t r;
-  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
-  return r;
-}
-__device__ __forceinline__ void f2_unpack(f2_t v, float& lo, float& hi) {
-  asm("mov.b64 {%0, %1}, %2;" : "=f"(lo), "=f"(hi) : "l"(v));
-}
-__device__ __forceinline__ f2_t ffma2(f2_t a, f2_t b, f2_t c) {
-  f2_t d;
-  asm volatile("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
-  return d;
-}
-__device__ __forceinline__ f2_t fadd2(f2_t a, f2_t b) {
-  f2_t d;
-  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
-  return d;
-}
-__device__ __forceinline__ ulonglong2 lds_pairs(const float* p) { return *reinterpret_cast<const ulonglong2*>(p); }
-
 __device__ __forceinline__ uint32_t atom_add_acqrel_smem(uint32_t* p, uint32_t v) {
   uint32_t old;
   asm volatile("atom.acq_rel.cta.shared::cta.add.u32 %0, [%1], %2;"

@@ -126,7 +126,7 @@ __device__ __forceinline__ void unit_next(const Sched& s, UnitIt& u) {
 // epilogue (R FMAs per pair, W_i broadcast from shared memory) instead of a
 // second tensor-core contraction: no P_hi/P_lo stores, no V MMA, and 256-source
 // tiles (two 256-column S buffers fill TMEM).
-template <int RC, int kStages, int RV>
+template <int RC, int kStages, int RV, int PP>
 __global__ void __launch_bounds__(kTcThreads, 1)
     ks_fused_tc_kernel(const __grid_constant__ CUtensorMap mA_hi, const __grid_constant__ CUtensorMap mA_lo,
                        const __grid_constant__ CUtensorMap mB_hi, const __grid_constant__ CUtensorMap mB_lo,
@@ -353,6 +353,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     float vblk[RVA];                      // FP32 sums over <= 8 tiles
 #pragma unroll
     for (int r = 0; r < RVA; ++r) { vacc[r] = 0.0; vblk[r] = 0.f; }
+    f2_t vacc2[2] = {0ull, 0ull};         // RV == 1: FFMA2 partial sums (4 lanes)
     int nblk = 0;
     float nbj = 0.f;
     int seg_q = 0, seg_st0 = 0;
@@ -362,7 +363,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       const uint32_t use = (uint32_t)(q >> 1);
       if (q == seg_q) {
         seg_st0 = cu.st;
-        if (!args.aug) nbj = __ldg(args.nb + cu.tt * kTcTileT + row);
+        nbj = __ldg(args.nb + cu.tt * kTcTileT + row);  // 0 when args.aug
       }
       mbar_wait(&wfull[q % WS], (uint32_t)((q / WS) & 1));
       mbar_wait(&sfull[bq], use & 1);
@@ -381,22 +382,42 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           __syncwarp();
           if (lane == 0) mbar_arrive(&sempty[bq]);  // S buffer may be overwritten now
         }
+        if (args.dbg_skip_v) {  // measurement knob: MMA/TMA-only timing
+          if (__uint_as_float(sv[0]) == 12345.f) vblk[0] += 1.f;
+          continue;
+        }
+        if constexpr (RV == 1) {
+          // two elements per FADD2/FFMA2; PP of every 16 pairs take 2^t on the
+          // FMA pipe (exp2_poly2) instead of MUFU.EX2 -- the MUFU rate is the
+          // epilogue's bound (SS6)
+          const f2_t nb2 = f2_bcast(nbj);
 #pragma unroll
-        for (int i = 0; i < BC; i += 4) {
-          float nav[4] = {0.f, 0.f, 0.f, 0.f};
-          if (!args.aug) {
-            const float4 na4 = *reinterpret_cast<const float4*>(nas + c0 + i);
-            nav[0] = na4.x + nbj; nav[1] = na4.y + nbj; nav[2] = na4.z + nbj; nav[3] = na4.w + nbj;
-          }
-          if constexpr (RV == 1) {
-            const float4 w4 = *reinterpret_cast<const float4*>(wvs + c0 + i);
-            const float wv[4] = {w4.x, w4.y, w4.z, w4.w};
+          for (int i = 0; i < BC; i += 4) {
+            const ulonglong2 na2 = lds_pairs(nas + c0 + i);
+            const ulonglong2 w2 = lds_pairs(wvs + c0 + i);
 #pragma unroll
-            for (int e = 0; e < 4; ++e) {
-              const float t = fminf(__uint_as_float(sv[i + e]) + nav[e], 0.f);  // clamp d^2 >= 0
-              vblk[0] = fmaf(ex2_approx(t), wv[e], vblk[0]);
+            for (int u = 0; u < 2; ++u) {
+              const int k = (i >> 1) + u;  // pair index within the batch
+              float t0, t1;
+              f2_unpack(fadd2(f2_pack(__uint_as_float(sv[i + 2 * u]), __uint_as_float(sv[i + 2 * u + 1])),
+                              fadd2(u ? na2.y : na2.x, nb2)),
+                        t0, t1);
+              t0 = fminf(t0, 0.f);  // clamp d^2 >= 0
+              t1 = fminf(t1, 0.f);
+              f2_t pk;
+              if (((k * PP) & 15) < PP) {
+                pk = exp2_poly2(f2_pack(fmaxf(t0, -125.f), fmaxf(t1, -125.f)));
+              } else {
+                pk = f2_pack(ex2_approx(t0), ex2_approx(t1));
+              }
+              vacc2[u] = ffma2f(pk, u ? w2.y : w2.x, vacc2[u]);
             }
-          } else {
+          }
+        } else {
+#pragma unroll
+          for (int i = 0; i < BC; i += 4) {
+            const float4 na4 = *reinterpret_cast<const float4*>(nas + c0 + i);
+            const float nav[4] = {na4.x + nbj, na4.y + nbj, na4.z + nbj, na4.w + nbj};
 #pragma unroll
             for (int e = 0; e < 4; ++e) {
               const float t = fminf(__uint_as_float(sv[i + e]) + nav[e], 0.f);  // clamp d^2 >= 0
@@ -418,6 +439,13 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       if (lane == 0) mbar_arrive(&wempty[q % WS]);  // na / W slot consumed
       const bool seg_end = (q == count - 1) || (cu.st + 1 == n_s);
       if (++nblk == 8 || seg_end) {  // FP32 over <= 8 tiles, then FP64
+        if constexpr (RV == 1) {  // the 4 FFMA2 lanes, fixed order
+          float a0, a1, a2, a3;
+          f2_unpack(vacc2[0], a0, a1);
+          f2_unpack(vacc2[1], a2, a3);
+          vblk[0] = (a0 + a1) + (a2 + a3);
+          vacc2[0] = vacc2[1] = 0ull;
+        }
 #pragma unroll
         for (int r = 0; r < RVA; ++r) { vacc[r] += (double)vblk[r]; vblk[r] = 0.f; }
         nblk = 0;
@@ -573,7 +601,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       }
       if (q == seg_q) {  // new segment: this target tile's norms
         seg_st0 = cu.st;
-        if (!args.aug) nbj = __ldg(args.nb + cu.tt * kTcTileT + row);
+        nbj = __ldg(args.nb + cu.tt * kTcTileT + row);  // 0 when args.aug
       }
       const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC) +
                                                        TcSmem::na_off(RC));
@@ -676,7 +704,7 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
     src_hi[i * k_pad + d] = ah;
     src_lo[i * k_pad + d] = to_tf32(a - ah);
   }
-  if (lane == 0) na[i] = nai;
+  if (lane == 0) na[i] = aug ? 0.f : nai;  // aug: the norms ride in the contraction, the epilogue adds 0
   for (int r = lane; r < rv; r += 32) wv[i * rv + r] = (live && r < R) ? W[i * R + r] : 0.f;
   for (int r = lane; r < r_pad; r += 32) {
     const float w = (live && r < R) ? W[i * R + r] : 0.f;
@@ -709,7 +737,7 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
     tgt_hi[j * k_pad + d] = xh;
     tgt_lo[j * k_pad + d] = to_tf32(x - xh);
   }
-  if (lane == 0) nb[j] = nbj;
+  if (lane == 0) nb[j] = aug ? 0.f : nbj;
 }
 
 cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
@@ -752,25 +780,37 @@ int fused_tc_stages() { return tc_stages(16); }
 int fused_tc_tile_s(int rv) { return rv ? 256 : kTcTileS; }
 int fused_tc_rv(int R) { return R <= 1 ? 1 : R <= 2 ? 2 : R <= 4 ? 4 : R <= 8 ? 8 : R <= 16 ? 16 : 0; }
 
-template <int RC, int NS, int RV>
+template <int RC, int NS, int RV, int PP = 0>
 static cudaError_t launch_rcsv(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
   static bool attr_done = false;
   const size_t smem = TcSmemT<NS, RV ? 256 : kTcTileS, RV>::total(RC);
   static_assert(TcSmemT<NS, RV ? 256 : kTcTileS, RV>::total(RC) <= 232448, "exceeds 227 KB of shared memory");
   if (!attr_done) {
-    cudaError_t e = cudaFuncSetAttribute(ks_fused_tc_kernel<RC, NS, RV>,
+    cudaError_t e = cudaFuncSetAttribute(ks_fused_tc_kernel<RC, NS, RV, PP>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr_done = true;
   }
-  ks_fused_tc_kernel<RC, NS, RV><<<a.sk.grid, kTcThreads, smem, st>>>(m[0], m[1], m[2], m[3], m[4], m[5], a);
+  ks_fused_tc_kernel<RC, NS, RV, PP><<<a.sk.grid, kTcThreads, smem, st>>>(m[0], m[1], m[2], m[3], m[4], m[5], a);
   return cudaGetLastError();
 }
+
+static constexpr int kTcPolyDefault = 0;  // measured (cfg3): PP 0 1.60 ms, 4 1.63, 6 1.69, 8 1.76
 
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st) {
   // CUDA-core weighted sum (256-source tiles): 48 KB stages, 4 fit (3 with the 16 KB weight slots)
   switch (a.vcc) {
-    case 1: return launch_rcsv<16, 4, 1>(maps, a, st);
+    case 1: {
+      // R = 1: PP of 16 exponential pairs on the FMA pipe (KS_TC_POLY = 0/4/6/8; measurement knob)
+      const char* e = getenv("KS_TC_POLY");
+      const int pp = e ? atoi(e) : kTcPolyDefault;
+      switch (pp) {
+        case 0: return launch_rcsv<16, 4, 1, 0>(maps, a, st);
+        case 4: return launch_rcsv<16, 4, 1, 4>(maps, a, st);
+        case 8: return launch_rcsv<16, 4, 1, 8>(maps, a, st);
+        default: return launch_rcsv<16, 4, 1, 6>(maps, a, st);
+      }
+    }
     case 2: return launch_rcsv<16, 4, 2>(maps, a, st);
     case 4: return launch_rcsv<16, 4, 4>(maps, a, st);
     case 8: return launch_rcsv<16, 4, 8>(maps, a, st);

@@ -105,6 +105,69 @@ __device__ __forceinline__ float ex2_approx(float x) {
 
 // Round an FP32 value to TF32 (10-bit mantissa, round-to-nearest-away),
 // returned as an FP32 bit pattern with the low 13 bits zero.
+// ---------------------------------------------------------------- packed FP32x2 (FFMA2 / FADD2)
+// A pair holds two FP32 lanes (lo = element 0).  fma.rn.f32x2 / add.rn.f32x2
+// do two IEEE FP32 operations in one issue slot; a scalar operand packed as
+// {x, x} is encoded as a broadcast register operand (no extra move).
+typedef unsigned long long f2_t;
+
+__device__ __forceinline__ f2_t f2_bcast(float x) {
+  f2_t r;
+  asm("mov.b64 %0, {%1, %1};" : "=l"(r) : "f"(x));
+  return r;
+}
+__device__ __forceinline__ f2_t f2_pack(float lo, float hi) {
+  f2_t r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
+  return r;
+}
+__device__ __forceinline__ void f2_unpack(f2_t v, float& lo, float& hi) {
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(lo), "=f"(hi) : "l"(v));
+}
+__device__ __forceinline__ f2_t ffma2(f2_t a, f2_t b, f2_t c) {
+  f2_t d;
+  asm volatile("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+  return d;
+}
+__device__ __forceinline__ f2_t fadd2(f2_t a, f2_t b) {
+  f2_t d;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+__device__ __forceinline__ ulonglong2 lds_pairs(const float* p) { return *reinterpret_cast<const ulonglong2*>(p); }
+
+__device__ __forceinline__ f2_t ffma2f(f2_t a, f2_t b, f2_t c) {  // schedulable (non-volatile) FFMA2
+  f2_t d;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+  return d;
+}
+
+// 2^x for a pair of lanes, x in [-125, 0], on the FMA/ALU pipes (no MUFU):
+// x = j + f with j = rint(x) (1.5*2^23 rounding trick), f in [-0.5, 0.5];
+// 2^f by a degree-5 polynomial with p(0) = 1 (minimax for relative error on
+// [-0.5, 0.5], fitted by tools/exp2_coeffs.py: 8.1e-8 exact, 1.6e-7 with FP32
+// Horner; ex2.approx.ftz is ~2^-22 relative); 2^j added to the exponent
+// field (valid because j >= -125 keeps the result normal).
+__device__ __forceinline__ f2_t exp2_poly2(f2_t x) {
+  const f2_t magic = f2_bcast(12582912.f);  // 1.5 * 2^23
+  const f2_t y = fadd2(x, magic);           // low mantissa bits of y = j (RN)
+  const f2_t jn = ffma2f(y, f2_bcast(-1.f), magic);  // -j, exact
+  const f2_t f = fadd2(x, jn);              // x - j, exact
+  f2_t p = ffma2f(f2_bcast(1.327463309e-03f), f, f2_bcast(9.671961889e-03f));
+  p = ffma2f(p, f, f2_bcast(5.550678447e-02f));
+  p = ffma2f(p, f, f2_bcast(2.402223498e-01f));
+  p = ffma2f(p, f, f2_bcast(6.931470633e-01f));
+  p = ffma2f(p, f, f2_bcast(1.f));
+  uint32_t plo, phi, ylo, yhi;
+  asm("mov.b64 {%0, %1}, %2;" : "=r"(plo), "=r"(phi) : "l"(p));
+  asm("mov.b64 {%0, %1}, %2;" : "=r"(ylo), "=r"(yhi) : "l"(y));
+  plo += ylo << 23;  // (0x4B400000 + j) << 23 == j << 23 (mod 2^32)
+  phi += yhi << 23;
+  f2_t r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "r"(plo), "r"(phi));
+  return r;
+}
+
 __device__ __forceinline__ float to_tf32(float x) {
   uint32_t r;
   asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));

@@ -8,7 +8,8 @@ import paper_conf_icppw_wangkbgj16_b200 as ks
 cfg = int(sys.argv[1]) if len(sys.argv) > 1 else 3
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 10
 a, W, b, h = workloads.make(cfg)
-plan = ks.KernelSum(a.shape[1], float(h))
+prec = sys.argv[3] if len(sys.argv) > 3 else "auto"
+plan = ks.KernelSum(a.shape[1], float(h), prec)
 ta, tw, tb = (torch.from_numpy(x).cuda() for x in (a, W, b))
 plan.set_sources(ta, tw)
 V = plan.eval(tb)
