@@ -58,7 +58,7 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
     p.add_argument("--no-flush", action="store_true")
-    p.add_argument("--precision", default="auto", choices=["auto", "fp32", "3xtf32", "tf32"],
+    p.add_argument("--precision", default="auto", choices=["auto", "fp32", "3xtf32", "3xf16", "tf32"],
                    help="ks_set_precision (auto: FP32 path for K<=32 and R=1, else 3xTF32 tensor cores)")
     return p.parse_args()
 
@@ -312,20 +312,33 @@ def run_ours(args):
     clk_sum = clk.summary()
     max_mhz = clk_sum["sm_max_mhz"] or 1965
     if info1["path"] == ks.KS_PATH_TC:
-        nprod = 3 if info1["precision"] == ks.KS_PREC_3XTF32 else 1
+        f16 = info1["precision"] == ks.KS_PREC_3XF16
+        nprod = 3 if info1["precision"] in (ks.KS_PREC_3XTF32, ks.KS_PREC_3XF16) else 1
         # R <= 16 (256-source tiles): the weighted sum runs on CUDA cores and the
         # tensor work is the 2K contraction; R > 16: a second MMA adds 2R per pair
         vcc = info1["tile_s"] == 256
-        flops_pair = nprod * 2 * (K + (0 if vcc else R))
-        achieved = pairs_launch * flops_pair / (kms / 1e3) / 1e12
         bf16 = load_peaks().get("bf16_tflops")
-        peak = (bf16 * 0.5) if bf16 else 1100.0
-        formula = "%d products x 2K per pair" % nprod if vcc else "%d products x 2(K+R) per pair" % nprod
+        if f16:
+            # S contraction on kind::f16 (BF16/FP16 rate); the R > 16 V-MMA stays TF32 and is
+            # counted at twice its FLOPs (TF32 runs at half the FP16 rate): FP16-equivalent FLOPs
+            flops_pair = nprod * 2 * (K + (0 if vcc else 2 * R))
+            peak = bf16 if bf16 else 2250.0
+            formula = ("%d products x 2K per pair" % nprod) if vcc else \
+                      ("%d products x 2(K+2R) per pair, FP16-equivalent" % nprod)
+            unit = "TFLOP/s (FP16 tensor; %s)" % formula
+            deriv = ("MEASURED_PEAKS bf16_tflops (burst) %.1f (kind::f16 = BF16 rate)" % bf16) if bf16 else \
+                    "fallback nominal dense FP16 2.25 PFLOP/s"
+        else:
+            flops_pair = nprod * 2 * (K + (0 if vcc else R))
+            peak = (bf16 * 0.5) if bf16 else 1100.0
+            formula = ("%d products x 2K per pair" % nprod) if vcc else ("%d products x 2(K+R) per pair" % nprod)
+            unit = "TFLOP/s (TF32 tensor; %s)" % formula
+            deriv = ("MEASURED_PEAKS bf16_tflops (burst) %.1f x 0.5 (nominal TF32/BF16 = 1.1/2.25 "
+                     "PFLOP/s)" % bf16) if bf16 else "fallback nominal dense TF32 1.1 PFLOP/s"
+        achieved = pairs_launch * flops_pair / (kms / 1e3) / 1e12
         roof = {"bound": "tensor", "kernel": "ks_fused_tc_kernel", "achieved": achieved, "peak": peak,
-                "unit": "TFLOP/s (TF32 tensor; %s)" % formula, "frac": achieved / peak,
-                "traffic": load_traffic(args.cfg, args.precision),
-                "peak_derivation": ("MEASURED_PEAKS bf16_tflops (burst) %.1f x 0.5 (nominal TF32/BF16 = 1.1/2.25 "
-                                    "PFLOP/s)" % bf16) if bf16 else "fallback nominal dense TF32 1.1 PFLOP/s"}
+                "unit": unit, "frac": achieved / peak,
+                "traffic": load_traffic(args.cfg, args.precision), "peak_derivation": deriv}
         # co-bound: one MUFU ex2 per pair, 16 / clk / SM
         sfu_peak = 16 * sms * max_mhz * 1e6
         roof["sfu"] = {"achieved_ex2_per_s": pairs_launch / (kms / 1e3), "peak_ex2_per_s": sfu_peak,
@@ -395,7 +408,8 @@ def run_ours(args):
     out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
            "scaling": "strong", "vs_baseline": None,
-           "dtype": "f32" if info1["path"] == ks.KS_PATH_FP32 else "tf32x3" if info1["precision"] == 2 else "tf32",
+           "dtype": "f32" if info1["path"] == ks.KS_PATH_FP32 else
+                    {2: "tf32x3", 3: "tf32", 4: "f16x3"}.get(info1["precision"], "?"),
            "data": "synthetic",
            "config": {"workload": workload_desc(c),
                       "l2": "flushed before every step (256 MiB write, outside the step events)",
@@ -403,7 +417,7 @@ def run_ours(args):
                                                                     if world > 1 else ""),
                       "step": "ks_set_sources (a1) + ks_eval (a2-a7)" + (" + collectives" if world > 1 else ""),
                       "path": {1: "fp32", 2: "tcgen05"}.get(info1["path"], info1["path"]),
-                      "precision": {1: "fp32", 2: "3xtf32", 3: "tf32"}.get(info1["precision"]),
+                      "precision": {1: "fp32", 2: "3xtf32", 3: "tf32", 4: "3xf16"}.get(info1["precision"]),
                       "k_pad": info1["k_pad"], "ctas": info1["num_ctas"],
                       "stages": info1["stages"]},
            "roofline": roof, "e2e": e2e, "clocks": clk_sum, "gpu_launches": launches,

@@ -56,10 +56,13 @@ typedef enum {
 } ks_status;
 
 typedef enum {
-  KS_PREC_AUTO = 0,     /* 3XTF32; FP32 path if K <= 32, R == 1, M <= 4096   */
+  KS_PREC_AUTO = 0,     /* 3XF16; FP32 path if K <= 32, R == 1, M <= 4096    */
   KS_PREC_FP32 = 1,     /* FP32 FFMA2 contraction (K <= 32, R == 1)          */
-  KS_PREC_3XTF32 = 2,   /* tcgen05 tensor cores, hi/lo split (3 products)    */
-  KS_PREC_TF32 = 3      /* tcgen05 tensor cores, single TF32 product         */
+  KS_PREC_3XTF32 = 2,   /* tcgen05 tensor cores, TF32 hi/lo split, 3 products */
+  KS_PREC_TF32 = 3,     /* tcgen05 tensor cores, single TF32 product         */
+  KS_PREC_3XF16 = 4     /* tcgen05 tensor cores, FP16 hi/lo split of power-of-2
+                           scaled operands, 3 products (same 22-bit operand
+                           precision as 3XTF32 at twice the MMA rate)        */
 } ks_precision;
 
 typedef enum { KS_PATH_NONE = 0, KS_PATH_FP32 = 1, KS_PATH_TC = 2 } ks_path;

@@ -22,9 +22,10 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libks.so")
 
 KS_OK, KS_EINVAL, KS_ESTATE, KS_ENOMEM, KS_ECUDA, KS_EUNSUPPORTED = range(6)
-KS_PREC_AUTO, KS_PREC_FP32, KS_PREC_3XTF32, KS_PREC_TF32 = range(4)
+KS_PREC_AUTO, KS_PREC_FP32, KS_PREC_3XTF32, KS_PREC_TF32, KS_PREC_3XF16 = range(5)
 KS_PATH_NONE, KS_PATH_FP32, KS_PATH_TC = range(3)
-PRECISIONS = {"auto": KS_PREC_AUTO, "fp32": KS_PREC_FP32, "3xtf32": KS_PREC_3XTF32, "tf32": KS_PREC_TF32}
+PRECISIONS = {"auto": KS_PREC_AUTO, "fp32": KS_PREC_FP32, "3xtf32": KS_PREC_3XTF32, "tf32": KS_PREC_TF32,
+              "3xf16": KS_PREC_3XF16}
 
 # every symbol include/ks.h declares (checked by tests/test_abi.py)
 EXPORTED = ("ks_create", "ks_destroy", "ks_set_precision", "ks_set_stream", "ks_set_sources", "ks_eval",

@@ -120,7 +120,9 @@ struct ks_ctx {
   DBuf<float> src;        // FP32 path: [k_pad + 2][m_pad]
   // TC path (tcgen05): TF32 hi/lo operand splits, norms, W^T splits
   DBuf<float> src_hi, src_lo, na, wt_hi, wt_lo, wv;
-  DBuf<float> tgt_hi, tgt_lo, nb;
+  DBuf<float> tgt_hi, tgt_lo, nb, tsc;   // FP16 mode: the hi/lo buffers hold halves
+  DBuf<unsigned> amax;                   // FP16 mode: max |alpha - mu| (FP32 bits)
+  int tc_f16 = 0;
   int r_pad = 16;
   int tc_aug = 0;  // norms folded into the contraction as 2 extra K columns
   int tc_vcc = 0;  // RV: weighted sum on CUDA cores over RV padded columns (0: tensor-core V path)
@@ -269,14 +271,19 @@ ks_status eval_fp32(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
 }
 
 
-ks_status encode_2d_sw64(CUtensorMap* map, const float* base, int64_t inner, int64_t rows, int box_rows) {
+// Row-major [rows][inner] operand, one box = box_rows x 64 bytes (16 FP32 or
+// 32 FP16 elements), SWIZZLE_64B: the K-major smem layout of the MMA operands.
+ks_status encode_2d_sw64(CUtensorMap* map, const void* base, int64_t inner, int64_t rows, int box_rows,
+                         bool f16 = false) {
   PFN_encodeTiled enc = get_encode();
   if (!enc) return fail(KS_ECUDA, "cuTensorMapEncodeTiled unavailable from the driver");
+  const size_t es = f16 ? 2 : 4;
   cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)rows};
-  cuuint64_t strides[1] = {(cuuint64_t)inner * sizeof(float)};
-  cuuint32_t box[2] = {(cuuint32_t)ks::kTcKC, (cuuint32_t)box_rows};
+  cuuint64_t strides[1] = {(cuuint64_t)inner * es};
+  cuuint32_t box[2] = {(cuuint32_t)(64 / es), (cuuint32_t)box_rows};
   cuuint32_t estr[2] = {1, 1};
-  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, estr,
+  CUresult r = enc(map, f16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
+                   const_cast<void*>(base), dims, strides, box, estr,
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return fail(KS_ECUDA, "cuTensorMapEncodeTiled (2D SW64) failed (CUresult %d)", (int)r);
@@ -310,8 +317,10 @@ int tc_k_pad(int K) { return (int)round_up(K + 2 * tc_aug(K), ks::kTcKC); }
 
 ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M, int R) {
   const int K = ctx->K;
-  const int k_pad = tc_k_pad(K);
-  const int aug = tc_aug(K);
+  const bool f16 = ctx->prec_eff == KS_PREC_3XF16;
+  // k_pad in elements: one 64-byte row chunk per pipeline stage = 16 FP32 or 32 FP16
+  const int k_pad = f16 ? (int)round_up(K, 2 * ks::kTcKC) : tc_k_pad(K);
+  const int aug = f16 ? 0 : tc_aug(K);  // FP16 mode: norms stay in FP32 in the epilogue
   // R == 1: weighted sum on CUDA cores (KS_TC_VCC=0 forces the tensor-core V path; measurement knob)
   const char* ev = getenv("KS_TC_VCC");
   const int vcc = (ev && ev[0] == '0') ? 0 : ks::fused_tc_rv(R);
@@ -319,7 +328,7 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   const int64_t m_pad = round_up(M > 0 ? M : 1, tile_s);
   const int r_pad = (int)round_up(R, 16);
   cudaStream_t st = ctx->stream;
-  const size_t nsrc = (size_t)m_pad * k_pad, nw = (size_t)r_pad * m_pad;
+  const size_t nsrc = f16 ? ((size_t)m_pad * k_pad + 1) / 2 : (size_t)m_pad * k_pad, nw = (size_t)r_pad * m_pad;
   KS_CUDA(ctx->src_hi.reserve(nsrc, st, false), "allocate source hi");
   KS_CUDA(ctx->src_lo.reserve(nsrc, st, false), "allocate source lo");
   KS_CUDA(ctx->na.reserve((size_t)m_pad, st, false), "allocate source norms");
@@ -333,19 +342,31 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(ctx->mean_part.reserve((size_t)nparts * K, st, false), "allocate mean partials");
   KS_CUDA(ks::launch_source_mean(alpha, M, K, k_pad, ctx->mean_part.p, nparts, ctx->mu.p, st), "source mean");
   ctx->launches += (M > 0) ? 2 : 1;
-  KS_CUDA(ks::launch_prep_tc_sources(alpha, W, M, m_pad, K, k_pad, R, vcc ? 0 : r_pad, ctx->mu.p, ctx->c, aug,
-                                     ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p, ctx->wv.p, vcc, st),
-          "source prep (TC)");
+  if (f16) {
+    KS_CUDA(ctx->amax.reserve(1, st, false), "allocate source max");
+    KS_CUDA(ks::launch_source_absmax(alpha, M, K, ctx->mu.p, ctx->amax.p, st), "source max (FP16 scaling)");
+    ctx->launches += (M > 0) ? 1 : 0;
+    KS_CUDA(ks::launch_prep_f16_sources(alpha, W, M, m_pad, K, k_pad, R, vcc ? 0 : r_pad, ctx->mu.p, ctx->c,
+                                        ctx->amax.p, ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p,
+                                        ctx->wt_lo.p, ctx->wv.p, vcc, st),
+            "source prep (TC, FP16)");
+  } else {
+    KS_CUDA(ks::launch_prep_tc_sources(alpha, W, M, m_pad, K, k_pad, R, vcc ? 0 : r_pad, ctx->mu.p, ctx->c, aug,
+                                       ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p,
+                                       ctx->wv.p, vcc, st),
+            "source prep (TC)");
+  }
   ctx->launches += 1;
-  ks_status s = encode_2d_sw64(&ctx->tmB_hi, ctx->src_hi.p, k_pad, m_pad, tile_s);
+  ks_status s = encode_2d_sw64(&ctx->tmB_hi, ctx->src_hi.p, k_pad, m_pad, tile_s, f16);
   if (s != KS_OK) return s;
-  s = encode_2d_sw64(&ctx->tmB_lo, ctx->src_lo.p, k_pad, m_pad, tile_s);
+  s = encode_2d_sw64(&ctx->tmB_lo, ctx->src_lo.p, k_pad, m_pad, tile_s, f16);
   if (s != KS_OK) return s;
   ctx->k_pad = k_pad;
   ctx->m_pad = m_pad;
   ctx->r_pad = r_pad;
   ctx->tc_aug = aug;
   ctx->tc_vcc = vcc;
+  ctx->tc_f16 = f16 ? 1 : 0;
   return KS_OK;
 }
 
@@ -353,18 +374,26 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   cudaStream_t st = ctx->stream;
   const int k_pad = ctx->k_pad;
   const int64_t n_pad = round_up(N, ks::kTcTileT);
-  const size_t ntg = (size_t)n_pad * k_pad;
+  const bool f16 = ctx->tc_f16 != 0;
+  const size_t ntg = f16 ? ((size_t)n_pad * k_pad + 1) / 2 : (size_t)n_pad * k_pad;
   KS_CUDA(ctx->tgt_hi.reserve(ntg, st, false), "allocate target hi");
   KS_CUDA(ctx->tgt_lo.reserve(ntg, st, false), "allocate target lo");
   KS_CUDA(ctx->nb.reserve((size_t)n_pad, st, false), "allocate target norms");
-  KS_CUDA(ks::launch_prep_tc_targets(beta, N, n_pad, ctx->K, k_pad, ctx->mu.p, ctx->c, ctx->tc_aug, ctx->tgt_hi.p,
-                                     ctx->tgt_lo.p, ctx->nb.p, st),
-          "target prep (TC)");
+  KS_CUDA(ctx->tsc.reserve((size_t)n_pad, st, false), "allocate target scales");
+  if (f16) {
+    KS_CUDA(ks::launch_prep_f16_targets(beta, N, n_pad, ctx->K, k_pad, ctx->mu.p, ctx->c, ctx->amax.p,
+                                        ctx->tgt_hi.p, ctx->tgt_lo.p, ctx->nb.p, ctx->tsc.p, st),
+            "target prep (TC, FP16)");
+  } else {
+    KS_CUDA(ks::launch_prep_tc_targets(beta, N, n_pad, ctx->K, k_pad, ctx->mu.p, ctx->c, ctx->tc_aug,
+                                       ctx->tgt_hi.p, ctx->tgt_lo.p, ctx->nb.p, ctx->tsc.p, st),
+            "target prep (TC)");
+  }
   ctx->launches += 1;
   CUtensorMap maps[6];
-  ks_status s = encode_2d_sw64(&maps[0], ctx->tgt_hi.p, k_pad, n_pad, ks::kTcTileT);
+  ks_status s = encode_2d_sw64(&maps[0], ctx->tgt_hi.p, k_pad, n_pad, ks::kTcTileT, f16);
   if (s != KS_OK) return s;
-  s = encode_2d_sw64(&maps[1], ctx->tgt_lo.p, k_pad, n_pad, ks::kTcTileT);
+  s = encode_2d_sw64(&maps[1], ctx->tgt_lo.p, k_pad, n_pad, ks::kTcTileT, f16);
   if (s != KS_OK) return s;
   maps[2] = ctx->tmB_hi;
   maps[3] = ctx->tmB_lo;
@@ -381,8 +410,10 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
 
   ks::TcArgs a;
   a.N = N;
-  a.k_pad = k_pad;
+  a.k_pad = f16 ? k_pad / 2 : k_pad;  // in FP32 units: 64-byte chunks = k_pad / kTcKC
   a.R = ctx->R;
+  a.f16 = f16 ? 1 : 0;
+  a.tsc = ctx->tsc.p;
   a.three = (ctx->prec_eff == KS_PREC_TF32) ? 0 : 1;
   a.aug = ctx->tc_aug;
   a.wv = ctx->wv.p;
@@ -497,8 +528,9 @@ ks_status ks_destroy(ks_ctx* ctx) {
   cudaStreamSynchronize(ctx->stream);
   ctx->src.release();
   for (DBuf<float>* bptr : {&ctx->src_hi, &ctx->src_lo, &ctx->na, &ctx->wt_hi, &ctx->wt_lo, &ctx->wv, &ctx->tgt_hi,
-                            &ctx->tgt_lo, &ctx->nb})
+                            &ctx->tgt_lo, &ctx->nb, &ctx->tsc})
     bptr->release();
+  ctx->amax.release();
   ctx->mu.release();
   ctx->mean_part.release();
   ctx->partial.release();
@@ -515,7 +547,7 @@ ks_status ks_destroy(ks_ctx* ctx) {
 
 ks_status ks_set_precision(ks_ctx* ctx, ks_precision p) {
   if (check_ctx(ctx)) return KS_EINVAL;
-  if (p != KS_PREC_AUTO && p != KS_PREC_FP32 && p != KS_PREC_3XTF32 && p != KS_PREC_TF32)
+  if (p != KS_PREC_AUTO && p != KS_PREC_FP32 && p != KS_PREC_3XTF32 && p != KS_PREC_TF32 && p != KS_PREC_3XF16)
     return fail(KS_EINVAL, "unknown precision %d", (int)p);
   ctx->prec_req = p;
   return KS_OK;
@@ -540,7 +572,7 @@ ks_status ks_set_sources(ks_ctx* ctx, const float* alpha, const float* W, int64_
     // every configuration except tiny source sets (M <= 4096, K <= 32, R == 1),
     // where the FP32 kernel's lower fixed cost wins.
     path = (ctx->K <= 32 && R == 1 && M <= 4096) ? KS_PATH_FP32 : KS_PATH_TC;
-    prec = (path == KS_PATH_FP32) ? KS_PREC_FP32 : KS_PREC_3XTF32;
+    prec = (path == KS_PATH_FP32) ? KS_PREC_FP32 : KS_PREC_3XF16;
   } else if (prec == KS_PREC_FP32) {
     if (ctx->K > 32 || R != 1)
       return fail(KS_EUNSUPPORTED, "FP32 path needs K <= 32 and R == 1 (K=%d, R=%d)", ctx->K, R);

@@ -27,6 +27,7 @@
 //            last-arriver fix-up (no atomics on V).
 // The M x N kernel matrix exists only as 128x128 TMEM tiles.
 #include "ks_internal.h"
+#include <cuda_fp16.h>
 #include "ks_ptx.cuh"
 
 #include <cstdlib>
@@ -203,6 +204,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       tma_prefetch_desc(&mB_hi);
       tma_prefetch_desc(&mW_hi);
     }
+    const int kcw = args.f16 ? 2 * kTcKC : kTcKC;  // elements per 64-byte chunk
     int it = 0;
     UnitIt cu = unit_begin(sc);
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
@@ -233,10 +235,11 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
         if (leader) {
           mbar_arrive_expect_tx(&full[s], kStageBytes);
-          tma_load_2d(sp, &mA_hi, kc * kTcKC, tt * kTcTileT, &full[s]);
-          tma_load_2d(sp + kChunkA, &mA_lo, kc * kTcKC, tt * kTcTileT, &full[s]);
-          tma_load_2d(sp + 2 * kChunkA, &mB_hi, kc * kTcKC, st * TS, &full[s]);
-          tma_load_2d(sp + 2 * kChunkA + kChunkB, &mB_lo, kc * kTcKC, st * TS, &full[s]);
+          const int k0 = kc * kcw;  // element coordinate of the 64-byte chunk
+          tma_load_2d(sp, &mA_hi, k0, tt * kTcTileT, &full[s]);
+          tma_load_2d(sp + kChunkA, &mA_lo, k0, tt * kTcTileT, &full[s]);
+          tma_load_2d(sp + 2 * kChunkA, &mB_hi, k0, st * TS, &full[s]);
+          tma_load_2d(sp + 2 * kChunkA + kChunkB, &mB_lo, k0, st * TS, &full[s]);
         }
         __syncwarp();
       }
@@ -244,7 +247,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   } else if (warp == 1) {
     // ================= MMA issuer (whole warp converged; one elected lane issues)
     const bool leader = elect_one();
-    const uint32_t idS = idesc_tf32(128, TS);
+    const uint32_t idS = args.f16 ? idesc_f16(128, TS) : idesc_tf32(128, TS);
     const uint32_t idV = idesc_tf32(128, RC);
     const int nprod = args.three ? 3 : 1;
     const bool skip_v = args.dbg_skip_v != 0;
@@ -308,8 +311,16 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           const uint64_t bH = d0 + (uint64_t)((2 * kChunkA + ks * 32) >> 4);
           const uint64_t bL = d0 + (uint64_t)((2 * kChunkA + kChunkB + ks * 32) >> 4);
           const uint32_t acc0 = (kc > 0 || ks > 0) ? 1u : 0u;
-          if (leader) {
-            if (args.three) {
+          if (leader) {  // products lo.hi, hi.lo, hi.hi (small terms first)
+            if (args.f16) {  // K = 16 halves = 32 bytes per instruction, as K = 8 TF32
+              if (args.three) {
+                mma_f16_ss(dS, aL, bH, idS, acc0);
+                mma_f16_ss(dS, aH, bL, idS, 1u);
+                mma_f16_ss(dS, aH, bH, idS, 1u);
+              } else {
+                mma_f16_ss(dS, aH, bH, idS, acc0);
+              }
+            } else if (args.three) {
               mma_tf32_ss(dS, aL, bH, idS, acc0);
               mma_tf32_ss(dS, aH, bL, idS, 1u);
               mma_tf32_ss(dS, aH, bH, idS, 1u);
@@ -355,7 +366,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     for (int r = 0; r < RVA; ++r) { vacc[r] = 0.0; vblk[r] = 0.f; }
     f2_t vacc2[2] = {0ull, 0ull};         // RV == 1: FFMA2 partial sums (4 lanes)
     int nblk = 0;
-    float nbj = 0.f;
+    float nbj = 0.f, rjs = 1.f;
     int seg_q = 0, seg_st0 = 0;
     UnitIt cu = unit_begin(sc);
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
@@ -364,6 +375,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       if (q == seg_q) {
         seg_st0 = cu.st;
         nbj = __ldg(args.nb + cu.tt * kTcTileT + row);  // 0 when args.aug
+        rjs = __ldg(args.tsc + cu.tt * kTcTileT + row);  // S scale (1 in TF32 modes)
       }
       mbar_wait(&wfull[q % WS], (uint32_t)((q / WS) & 1));
       mbar_wait(&sfull[bq], use & 1);
@@ -390,7 +402,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           // two elements per FADD2/FFMA2; PP of every 16 pairs take 2^t on the
           // FMA pipe (exp2_poly2) instead of MUFU.EX2 -- the MUFU rate is the
           // epilogue's bound (SS6)
-          const f2_t nb2 = f2_bcast(nbj);
+          const f2_t nb2 = f2_bcast(nbj), rj2 = f2_bcast(rjs);
 #pragma unroll
           for (int i = 0; i < BC; i += 4) {
             const ulonglong2 na2 = lds_pairs(nas + c0 + i);
@@ -399,8 +411,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
             for (int u = 0; u < 2; ++u) {
               const int k = (i >> 1) + u;  // pair index within the batch
               float t0, t1;
-              f2_unpack(fadd2(f2_pack(__uint_as_float(sv[i + 2 * u]), __uint_as_float(sv[i + 2 * u + 1])),
-                              fadd2(u ? na2.y : na2.x, nb2)),
+              // t = S rj + (na_i + nb_j)
+              f2_unpack(ffma2f(f2_pack(__uint_as_float(sv[i + 2 * u]), __uint_as_float(sv[i + 2 * u + 1])), rj2,
+                               fadd2(u ? na2.y : na2.x, nb2)),
                         t0, t1);
               t0 = fminf(t0, 0.f);  // clamp d^2 >= 0
               t1 = fminf(t1, 0.f);
@@ -420,7 +433,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
             const float nav[4] = {na4.x + nbj, na4.y + nbj, na4.z + nbj, na4.w + nbj};
 #pragma unroll
             for (int e = 0; e < 4; ++e) {
-              const float t = fminf(__uint_as_float(sv[i + e]) + nav[e], 0.f);  // clamp d^2 >= 0
+              const float t = fminf(fmaf(__uint_as_float(sv[i + e]), rjs, nav[e]), 0.f);  // clamp d^2 >= 0
               const float pk = ex2_approx(t);
               const float* wrow = wvs + (c0 + i + e) * RVA;
 #pragma unroll
@@ -515,7 +528,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     double vacc[HC];
 #pragma unroll
     for (int r = 0; r < HC; ++r) vacc[r] = 0.0;
-    float nbj = 0.f;
+    float nbj = 0.f, rjs = 1.f;
     int seg_q = 0;                        // first local unit of the current segment
     int seg_st0 = 0;                      // its source tile
 
@@ -602,6 +615,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       if (q == seg_q) {  // new segment: this target tile's norms
         seg_st0 = cu.st;
         nbj = __ldg(args.nb + cu.tt * kTcTileT + row);  // 0 when args.aug
+        rjs = __ldg(args.tsc + cu.tt * kTcTileT + row);
       }
       const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC) +
                                                        TcSmem::na_off(RC));
@@ -619,15 +633,12 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         uint32_t hi[CB], lo[CB];
 #pragma unroll
         for (int i = 0; i < CB; i += 4) {
-          float nav[4] = {0.f, 0.f, 0.f, 0.f};
-          if (!args.aug) {
-            const float4 na4 = *reinterpret_cast<const float4*>(nas + c0 + i);
-            nav[0] = na4.x + nbj; nav[1] = na4.y + nbj; nav[2] = na4.z + nbj; nav[3] = na4.w + nbj;
-          }
+          const float4 na4 = *reinterpret_cast<const float4*>(nas + c0 + i);
+          const float nav[4] = {na4.x + nbj, na4.y + nbj, na4.z + nbj, na4.w + nbj};
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
-            // t = S + na_i + nb_j (norms already inside S when args.aug), clamp d^2 >= 0
-            const float t = fminf(__uint_as_float(sv[i + e]) + nav[e], 0.f);
+            // t = S rj + na_i + nb_j (na, nb = 0 when the norms ride in S, args.aug), clamp d^2 >= 0
+            const float t = fminf(fmaf(__uint_as_float(sv[i + e]), rjs, nav[e]), 0.f);
             const float p = ex2_approx(t);                                    // in [0, 1]
             const uint32_t hb = (__float_as_uint(p) + 0x1000u) & 0xFFFFE000u;  // TF32 round-to-nearest
             hi[i + e] = hb;
@@ -672,10 +683,27 @@ __device__ __forceinline__ double warp_sum_fixed(double v) {
   return __shfl_sync(0xffffffffu, v, 0);
 }
 
+// Exponent s such that amax * 2^s lies in [2^12, 2^13) (FP16 mode operand
+// scaling; clamped so that 2^-(sA + sB) stays a normal FP32 number).
+__device__ __forceinline__ int f16_scale_exp(float amax) {
+  if (!(amax > 0.f)) return 0;
+  int e;
+  frexpf(amax, &e);  // amax = m 2^e, m in [0.5, 1)
+  const int s = 13 - e;
+  return s < -60 ? -60 : (s > 60 ? 60 : s);
+}
+
+__device__ __forceinline__ void split_f16(float x, __half& hi, __half& lo) {
+  hi = __float2half_rn(x);
+  lo = __float2half_rn(x - __half2float(hi));  // x - hi is exact in FP32
+}
+
+template <bool F16>
 __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const float* __restrict__ W, int64_t M,
                                        int64_t m_pad, int K, int k_pad, int R, int r_pad,
-                                       const float* __restrict__ mu, double c, int aug, float* __restrict__ src_hi,
-                                       float* __restrict__ src_lo, float* __restrict__ na,
+                                       const float* __restrict__ mu, double c, int aug,
+                                       const unsigned* __restrict__ amax, void* __restrict__ src_hi,
+                                       void* __restrict__ src_lo, float* __restrict__ na,
                                        float* __restrict__ wt_hi, float* __restrict__ wt_lo,
                                        float* __restrict__ wv, int rv) {
   const int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -690,19 +718,28 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
   n = warp_sum_fixed(n);
   const float nai = live ? (float)(-c * n) : 0.f;
   const double c2 = 2.0 * c;
+  float sA = 1.f;
+  if constexpr (F16) sA = ldexpf(1.f, f16_scale_exp((float)(c2 * (double)__uint_as_float(*amax))));
   for (int d = lane; d < k_pad; d += 32) {
     float a = 0.f;
     if (d < K) {
       const float x = live ? alpha[i * K + d] - mu[d] : 0.f;
       a = (float)(c2 * (double)x);
-    } else if (aug && d == K) {
+    } else if (!F16 && aug && d == K) {
       a = 1.f;   // multiplies nb_j of the target
-    } else if (aug && d == K + 1) {
+    } else if (!F16 && aug && d == K + 1) {
       a = nai;   // times 1 on the target side
     }
-    const float ah = to_tf32(a);
-    src_hi[i * k_pad + d] = ah;
-    src_lo[i * k_pad + d] = to_tf32(a - ah);
+    if constexpr (F16) {
+      __half h, l;
+      split_f16(a * sA, h, l);  // exact power-of-2 scaling
+      static_cast<__half*>(src_hi)[i * k_pad + d] = h;
+      static_cast<__half*>(src_lo)[i * k_pad + d] = l;
+    } else {
+      const float ah = to_tf32(a);
+      static_cast<float*>(src_hi)[i * k_pad + d] = ah;
+      static_cast<float*>(src_lo)[i * k_pad + d] = to_tf32(a - ah);
+    }
   }
   if (lane == 0) na[i] = aug ? 0.f : nai;  // aug: the norms ride in the contraction, the epilogue adds 0
   for (int r = lane; r < rv; r += 32) wv[i * rv + r] = (live && r < R) ? W[i * R + r] : 0.f;
@@ -714,30 +751,76 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
   }
 }
 
+template <bool F16>
 __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N, int64_t n_pad, int K, int k_pad,
-                                       const float* __restrict__ mu, double c, int aug, float* __restrict__ tgt_hi,
-                                       float* __restrict__ tgt_lo, float* __restrict__ nb) {
+                                       const float* __restrict__ mu, double c, int aug,
+                                       const unsigned* __restrict__ amax, void* __restrict__ tgt_hi,
+                                       void* __restrict__ tgt_lo, float* __restrict__ nb,
+                                       float* __restrict__ tsc) {
   const int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   if (j >= n_pad) return;
   const bool live = j < N;
   double n = 0.0;
+  float bmax = 0.f;
   for (int d = lane; d < K; d += 32) {
     const float x = live ? beta[j * K + d] - mu[d] : 0.f;
     n += (double)x * (double)x;
+    bmax = fmaxf(bmax, fabsf(x));
   }
   n = warp_sum_fixed(n);
   const float nbj = live ? (float)(-c * n) : 0.f;
+  float sB = 1.f, rj = 1.f;
+  if constexpr (F16) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) bmax = fmaxf(bmax, __shfl_xor_sync(0xffffffffu, bmax, o));
+    const int eA = f16_scale_exp((float)(2.0 * c * (double)__uint_as_float(*amax)));
+    const int eB = f16_scale_exp(bmax);
+    sB = ldexpf(1.f, eB);
+    rj = ldexpf(1.f, -(eA + eB));
+  }
   for (int d = lane; d < k_pad; d += 32) {
     float x = 0.f;
     if (d < K) x = live ? beta[j * K + d] - mu[d] : 0.f;
-    else if (aug && d == K) x = nbj;
-    else if (aug && d == K + 1) x = 1.f;
-    const float xh = to_tf32(x);
-    tgt_hi[j * k_pad + d] = xh;
-    tgt_lo[j * k_pad + d] = to_tf32(x - xh);
+    else if (!F16 && aug && d == K) x = nbj;
+    else if (!F16 && aug && d == K + 1) x = 1.f;
+    if constexpr (F16) {
+      __half h, l;
+      split_f16(x * sB, h, l);
+      static_cast<__half*>(tgt_hi)[j * k_pad + d] = h;
+      static_cast<__half*>(tgt_lo)[j * k_pad + d] = l;
+    } else {
+      const float xh = to_tf32(x);
+      static_cast<float*>(tgt_hi)[j * k_pad + d] = xh;
+      static_cast<float*>(tgt_lo)[j * k_pad + d] = to_tf32(x - xh);
+    }
   }
-  if (lane == 0) nb[j] = aug ? 0.f : nbj;
+  if (lane == 0) {
+    nb[j] = aug ? 0.f : nbj;
+    tsc[j] = rj;
+  }
+}
+
+// max_i,d |alpha[i][d] - mu[d]| as FP32 bits (non-negative floats order as unsigned ints).
+__global__ void source_absmax_kernel(const float* __restrict__ alpha, int64_t total, int K,
+                                     const float* __restrict__ mu, unsigned* __restrict__ amax) {
+  float m = 0.f;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x)
+    m = fmaxf(m, fabsf(alpha[e] - mu[e % K]));
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+  if ((threadIdx.x & 31) == 0) atomicMax(amax, __float_as_uint(m));
+}
+
+cudaError_t launch_source_absmax(const float* alpha, int64_t M, int K, const float* mu, unsigned* amax,
+                                 cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(amax, 0, sizeof(unsigned), st);
+  if (e != cudaSuccess || M == 0) return e;
+  const int64_t total = M * K;
+  int64_t blocks = (total + 255) / 256;
+  if (blocks > 4 * 148) blocks = 4 * 148;
+  source_absmax_kernel<<<(unsigned)blocks, 256, 0, st>>>(alpha, total, K, mu, amax);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
@@ -746,17 +829,39 @@ cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M
                                    cudaStream_t st) {
   if (m_pad == 0) return cudaSuccess;
   const int bs = 256;  // 8 points per block
-  prep_tc_sources_kernel<<<(unsigned)((m_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
-      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv);
+  prep_tc_sources_kernel<false><<<(unsigned)((m_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
+      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, nullptr, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_prep_f16_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
+                                    int R, int r_pad, const float* mu, double c, const unsigned* amax, void* src_hi,
+                                    void* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv, int rv,
+                                    cudaStream_t st) {
+  if (m_pad == 0) return cudaSuccess;
+  const int bs = 256;
+  prep_tc_sources_kernel<true><<<(unsigned)((m_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
+      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, 0, amax, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv);
   return cudaGetLastError();
 }
 
 cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
-                                   double c, int aug, float* tgt_hi, float* tgt_lo, float* nb, cudaStream_t st) {
+                                   double c, int aug, float* tgt_hi, float* tgt_lo, float* nb, float* tsc,
+                                   cudaStream_t st) {
   if (n_pad == 0) return cudaSuccess;
   const int bs = 256;
-  prep_tc_targets_kernel<<<(unsigned)((n_pad * 32 + bs - 1) / bs), bs, 0, st>>>(beta, N, n_pad, K, k_pad, mu, c, aug,
-                                                                                tgt_hi, tgt_lo, nb);
+  prep_tc_targets_kernel<false><<<(unsigned)((n_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
+      beta, N, n_pad, K, k_pad, mu, c, aug, nullptr, tgt_hi, tgt_lo, nb, tsc);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_prep_f16_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
+                                    double c, const unsigned* amax, void* tgt_hi, void* tgt_lo, float* nb,
+                                    float* tsc, cudaStream_t st) {
+  if (n_pad == 0) return cudaSuccess;
+  const int bs = 256;
+  prep_tc_targets_kernel<true><<<(unsigned)((n_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
+      beta, N, n_pad, K, k_pad, mu, c, 0, amax, tgt_hi, tgt_lo, nb, tsc);
   return cudaGetLastError();
 }
 

@@ -70,7 +70,9 @@ struct TcArgs {
   int r_valid;          // valid columns among them
   int r_off;            // first weight column of this launch
   int R;                // row stride of V
-  int three;            // 1: 3xTF32 (hi.hi + hi.lo + lo.hi), 0: plain TF32 (hi.hi)
+  int three;            // 1: three split products (hi.hi + hi.lo + lo.hi), 0: plain TF32 (hi.hi)
+  int f16;              // 1: operands are the FP16 split of power-of-2 scaled values (kind::f16 MMA)
+  const float* tsc;     // [n_pad] per-target factor on S: 1 (TF32 modes) or 2^-(eA+eB_j) (FP16 mode)
   int aug;              // 1: norms folded into the contraction (2 extra K columns), epilogue adds nothing
   int vcc;              // RV > 0: weighted sum on CUDA cores over RV padded columns (no W^T tiles, no V MMA)
   const float* wv;      // [m_pad][RV] weights, zero padded (vcc)
@@ -95,7 +97,24 @@ cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M
 // targets: tgt_hi/lo [n_pad][k_pad] = TF32 split of (beta - mu), nb [n_pad]
 // aug: columns K, K+1 hold (nb_j, 1)
 cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
-                                   double c, int aug, float* tgt_hi, float* tgt_lo, float* nb, cudaStream_t st);
+                                   double c, int aug, float* tgt_hi, float* tgt_lo, float* nb, float* tsc,
+                                   cudaStream_t st);
+// FP16 mode (KS_PREC_3XF16).  k_pad is a multiple of 2*kTcKC halves (one
+// 64-byte row chunk per stage, as in TF32 mode).  amax = max |alpha - mu|
+// (FP32 bits, atomicMax; must be zeroed first).  Sources are scaled by
+// sA = 2^(13 - e), e = exponent of RN(2c * amax) (frexp convention), targets
+// per row by sB_j = 2^(13 - e_j) from max_k |beta_jk - mu_k|; each scaled
+// value x is split x = hi + lo, hi = RN_f16(x), lo = RN_f16(x - hi);
+// tsc[j] = 2^-(log2 sA + log2 sB_j) undoes the scaling on S.
+cudaError_t launch_source_absmax(const float* alpha, int64_t M, int K, const float* mu, unsigned* amax,
+                                 cudaStream_t st);
+cudaError_t launch_prep_f16_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
+                                    int R, int r_pad, const float* mu, double c, const unsigned* amax, void* src_hi,
+                                    void* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv, int rv,
+                                    cudaStream_t st);
+cudaError_t launch_prep_f16_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
+                                    double c, const unsigned* amax, void* tgt_hi, void* tgt_lo, float* nb,
+                                    float* tsc, cudaStream_t st);
 // maps: A_hi, A_lo (targets), B_hi, B_lo (sources), W_hi, W_lo (weights^T)
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st);
 int fused_tc_stages();

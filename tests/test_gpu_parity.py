@@ -27,7 +27,7 @@ import paper_conf_icppw_wangkbgj16_b200 as ks  # noqa: E402
 _PREC = {"p": "fp32"}
 
 
-@pytest.fixture(autouse=True, params=["fp32", "3xtf32"])
+@pytest.fixture(autouse=True, params=["fp32", "3xtf32", "3xf16"])
 def precision(request):
     _PREC["p"] = request.param
     yield request.param
@@ -253,8 +253,8 @@ def test_info_reports_path():
 
 
 def test_auto_policy():
-    """AUTO: FP32 kernel for tiny source sets, tcgen05 3xTF32 otherwise (SS7)."""
-    for M, want in ((1024, ks.KS_PATH_FP32), (8192, ks.KS_PATH_TC)):
+    """AUTO: FP32 kernel for tiny source sets, tcgen05 split-FP16 otherwise (SS7)."""
+    for M, want, prec in ((1024, ks.KS_PATH_FP32, ks.KS_PREC_FP32), (8192, ks.KS_PATH_TC, ks.KS_PREC_3XF16)):
         with ks.KernelSum(32, 1.0, "auto") as plan:
             plan.set_sources(torch.rand((M, 32), device="cuda"), torch.rand((M, 1), device="cuda"))
-            assert plan.info()["path"] == want
+            assert plan.info()["path"] == want and plan.info()["precision"] == prec

@@ -1,6 +1,6 @@
 """GPU parity of the tensor-core (tcgen05 / TMEM, 3xTF32) path against the
 FP64 oracle.  The path serves K > 32 or R > 1 by default (KS_PREC_AUTO) and
-any (K, R) on request ("3xtf32" / "tf32").  Bars (BASELINE.json north_star,
+any (K, R) on request ("3xf16" / "3xtf32" / "tf32").  Bars (BASELINE.json north_star,
 DESIGN.md SS4): e_norm <= 1e-5 for 3xTF32, <= 2e-3 for plain TF32."""
 import numpy as np
 import pytest
@@ -17,7 +17,20 @@ if not torch.cuda.is_available():
 import paper_conf_icppw_wangkbgj16_b200 as ks  # noqa: E402
 
 
-def gpu_eval(alpha, W, beta, h, precision="auto"):
+_PREC = {"p": "auto"}
+
+
+@pytest.fixture(autouse=True, params=["3xf16", "3xtf32"])
+def _split_precision(request):
+    """Every test below runs on both split-operand MMA kinds (kind::f16 with
+    power-of-2 scaled FP16 hi/lo operands -- the KS_PREC_AUTO choice -- and
+    kind::tf32 with TF32 hi/lo), unless it names a precision itself."""
+    _PREC["p"] = request.param
+    yield
+
+
+def gpu_eval(alpha, W, beta, h, precision=None):
+    precision = precision or _PREC["p"]
     W = np.asarray(W, np.float32)
     if W.ndim == 1:
         W = W[:, None]
@@ -30,7 +43,7 @@ def gpu_eval(alpha, W, beta, h, precision="auto"):
     return V.cpu().numpy().astype(np.float64), info
 
 
-def check(oracle_mod, a, W, b, h, precision="auto", tol=TOL_3XTF32, J=None):
+def check(oracle_mod, a, W, b, h, precision=None, tol=TOL_3XTF32, J=None):
     V, info = gpu_eval(a, W, b, h, precision)
     assert info["path"] == ks.KS_PATH_TC
     Vr = oracle_mod.oracle_eval(a, W, b, float(h), J=J)
@@ -50,7 +63,7 @@ def test_cfg4_tight_cluster_separates_tf32(oracle_mod):
     reported against its own 2e-3 bar and is measurably worse."""
     c = workloads.Config(4, 3000, 500, 256, 16, 2.0, "gm", sigma=0.05)
     a, W, b, h = workloads.make(c, wkind="pos")
-    e3 = check(oracle_mod, a, W, b, h, "3xtf32", TOL_3XTF32)
+    e3 = check(oracle_mod, a, W, b, h, None, TOL_3XTF32)
     e1 = check(oracle_mod, a, W, b, h, "tf32", TOL_TF32)
     assert e1 > 10 * e3
 
@@ -68,7 +81,7 @@ def test_tensor_core_path_for_low_k(oracle_mod, K):
     """NEXT-3: the tcgen05 path on request for K <= 32, R = 1."""
     c = workloads.Config(3, 4000, 900, K, 1, 1.0, "gm", sigma=0.1)
     a, W, b, h = workloads.make(c, wkind="pos")
-    check(oracle_mod, a, W, b, h, "3xtf32")
+    check(oracle_mod, a, W, b, h)
 
 
 @pytest.mark.parametrize("M,N", [(1, 1), (1, 129), (129, 1), (128, 128), (257, 255)])
