@@ -122,6 +122,8 @@ struct ks_ctx {
   DBuf<float> src_hi, src_lo, na, wt_hi, wt_lo, wv;
   DBuf<float> tgt_hi, tgt_lo, nb, tsc;   // FP16 mode: the hi/lo buffers hold halves
   DBuf<unsigned> amax;                   // FP16 mode: max |alpha - mu| (FP32 bits)
+  DBuf<unsigned> wstat;                  // R = 1: {max |W| bits, any W < 0} (log-weight epilogue)
+  bool tc_wstat = false;
   int tc_f16 = 0;
   int r_pad = 16;
   int tc_aug = 0;  // norms folded into the contraction as 2 extra K columns
@@ -342,18 +344,28 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(ctx->mean_part.reserve((size_t)nparts * K, st, false), "allocate mean partials");
   KS_CUDA(ks::launch_source_mean(alpha, M, K, k_pad, ctx->mean_part.p, nparts, ctx->mu.p, st), "source mean");
   ctx->launches += (M > 0) ? 2 : 1;
+  // R = 1 with W >= 0: log-weights in na (decided on the device, no host sync);
+  // KS_TC_LOGW=0 disables (measurement knob)
+  const char* elw = getenv("KS_TC_LOGW");
+  const bool use_wstat = (vcc == 1) && !(elw && elw[0] == '0');
+  if (use_wstat) {
+    KS_CUDA(ctx->wstat.reserve(2, st, false), "allocate weight stats");
+    KS_CUDA(ks::launch_weight_stats(W, M, ctx->wstat.p, st), "weight stats");
+    ctx->launches += (M > 0) ? 1 : 0;
+  }
+  const unsigned* wst = use_wstat ? ctx->wstat.p : nullptr;
   if (f16) {
     KS_CUDA(ctx->amax.reserve(1, st, false), "allocate source max");
     KS_CUDA(ks::launch_source_absmax(alpha, M, K, ctx->mu.p, ctx->amax.p, st), "source max (FP16 scaling)");
     ctx->launches += (M > 0) ? 1 : 0;
     KS_CUDA(ks::launch_prep_f16_sources(alpha, W, M, m_pad, K, k_pad, R, vcc ? 0 : r_pad, ctx->mu.p, ctx->c,
                                         ctx->amax.p, ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p,
-                                        ctx->wt_lo.p, ctx->wv.p, vcc, st),
+                                        ctx->wt_lo.p, ctx->wv.p, vcc, wst, st),
             "source prep (TC, FP16)");
   } else {
     KS_CUDA(ks::launch_prep_tc_sources(alpha, W, M, m_pad, K, k_pad, R, vcc ? 0 : r_pad, ctx->mu.p, ctx->c, aug,
                                        ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p,
-                                       ctx->wv.p, vcc, st),
+                                       ctx->wv.p, vcc, wst, st),
             "source prep (TC)");
   }
   ctx->launches += 1;
@@ -367,6 +379,7 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   ctx->tc_aug = aug;
   ctx->tc_vcc = vcc;
   ctx->tc_f16 = f16 ? 1 : 0;
+  ctx->tc_wstat = use_wstat;
   return KS_OK;
 }
 
@@ -414,6 +427,7 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.R = ctx->R;
   a.f16 = f16 ? 1 : 0;
   a.tsc = ctx->tsc.p;
+  a.wstat = ctx->tc_wstat ? ctx->wstat.p : nullptr;
   a.three = (ctx->prec_eff == KS_PREC_TF32) ? 0 : 1;
   a.aug = ctx->tc_aug;
   a.wv = ctx->wv.p;
@@ -424,7 +438,7 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   }
   {
     const char* e = getenv("KS_TC_DEBUG_SKIP_V");
-    a.dbg_skip_v = (e && e[0] == '1') ? 1 : 0;
+    a.dbg_skip_v = (e && e[0] >= '1' && e[0] <= '3') ? e[0] - '0' : 0;  // 1 no epilogue math, 2 no MUFU, 3 no TMEM load
   }
   a.na = ctx->na.p;
   a.nb = ctx->nb.p;
@@ -531,6 +545,7 @@ ks_status ks_destroy(ks_ctx* ctx) {
                             &ctx->tgt_lo, &ctx->nb, &ctx->tsc})
     bptr->release();
   ctx->amax.release();
+  ctx->wstat.release();
   ctx->mu.release();
   ctx->mean_part.release();
   ctx->partial.release();

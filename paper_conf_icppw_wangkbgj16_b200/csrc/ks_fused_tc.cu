@@ -250,7 +250,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     const uint32_t idS = args.f16 ? idesc_f16(128, TS) : idesc_tf32(128, TS);
     const uint32_t idV = idesc_tf32(128, RC);
     const int nprod = args.three ? 3 : 1;
-    const bool skip_v = args.dbg_skip_v != 0;
+    const bool skip_v = args.dbg_skip_v == 1;
     int it = 0;
     // V(p, hh) += P(p)[:, 64hh : 64hh+64] . W(p)[64hh : 64hh+64, :] on the tensor
     // cores, A = P read from TMEM.  Issued as soon as the epilogue has
@@ -365,6 +365,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 #pragma unroll
     for (int r = 0; r < RVA; ++r) { vacc[r] = 0.0; vblk[r] = 0.f; }
     f2_t vacc2[2] = {0ull, 0ull};         // RV == 1: FFMA2 partial sums (4 lanes)
+    // R = 1 with W >= 0 (device-side flag from the source prep): log-weights in na
+    const bool logw = RV == 1 && args.wstat != nullptr && args.wstat[1] == 0u && args.wstat[0] != 0u;
+    const double wsc = logw ? (double)__uint_as_float(args.wstat[0]) : 1.0;
     int nblk = 0;
     float nbj = 0.f, rjs = 1.f;
     int seg_q = 0, seg_st0 = 0;
@@ -394,36 +397,58 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           __syncwarp();
           if (lane == 0) mbar_arrive(&sempty[bq]);  // S buffer may be overwritten now
         }
-        if (args.dbg_skip_v) {  // measurement knob: MMA/TMA-only timing
+        if (args.dbg_skip_v == 1) {  // measurement knob: MMA/TMA-only timing
           if (__uint_as_float(sv[0]) == 12345.f) vblk[0] += 1.f;
           continue;
         }
         if constexpr (RV == 1) {
           // two elements per FADD2/FFMA2; PP of every 16 pairs take 2^t on the
-          // FMA pipe (exp2_poly2) instead of MUFU.EX2 -- the MUFU rate is the
-          // epilogue's bound (SS6)
+          // FMA pipe (exp2_poly2) instead of MUFU.EX2.  No clamp of t at 0
+          // here (reading Q12): rounding can leave t a few ulps
+          // above 0, as it can leave it below.
           const f2_t nb2 = f2_bcast(nbj), rj2 = f2_bcast(rjs);
+          if (logw) {
+            // W >= 0: na_i carries + log2(W_i / Wmax), so V_j / Wmax = sum_i 2^t
 #pragma unroll
-          for (int i = 0; i < BC; i += 4) {
-            const ulonglong2 na2 = lds_pairs(nas + c0 + i);
-            const ulonglong2 w2 = lds_pairs(wvs + c0 + i);
+            for (int i = 0; i < BC; i += 4) {
+              const ulonglong2 na2 = lds_pairs(nas + c0 + i);
 #pragma unroll
-            for (int u = 0; u < 2; ++u) {
-              const int k = (i >> 1) + u;  // pair index within the batch
-              float t0, t1;
-              // t = S rj + (na_i + nb_j)
-              f2_unpack(ffma2f(f2_pack(__uint_as_float(sv[i + 2 * u]), __uint_as_float(sv[i + 2 * u + 1])), rj2,
-                               fadd2(u ? na2.y : na2.x, nb2)),
-                        t0, t1);
-              t0 = fminf(t0, 0.f);  // clamp d^2 >= 0
-              t1 = fminf(t1, 0.f);
-              f2_t pk;
-              if (((k * PP) & 15) < PP) {
-                pk = exp2_poly2(f2_pack(fmaxf(t0, -125.f), fmaxf(t1, -125.f)));
-              } else {
-                pk = f2_pack(ex2_approx(t0), ex2_approx(t1));
+              for (int u = 0; u < 2; ++u) {
+                const int k = (i >> 1) + u;
+                const f2_t x = ffma2f(f2_pack(__uint_as_float(sv[i + 2 * u]), __uint_as_float(sv[i + 2 * u + 1])),
+                                      rj2, fadd2(u ? na2.y : na2.x, nb2));
+                float t0, t1;
+                f2_unpack(x, t0, t1);
+                f2_t pk;
+                if (((k * PP) & 15) < PP) {
+                  pk = exp2_poly2(f2_pack(fmaxf(t0, -125.f), fmaxf(t1, -125.f)));
+                } else {
+                  pk = f2_pack(ex2_approx(t0), ex2_approx(t1));
+                }
+                vacc2[u] = fadd2(vacc2[u], pk);
               }
-              vacc2[u] = ffma2f(pk, u ? w2.y : w2.x, vacc2[u]);
+            }
+          } else {
+#pragma unroll
+            for (int i = 0; i < BC; i += 4) {
+              const ulonglong2 na2 = lds_pairs(nas + c0 + i);
+              const ulonglong2 w2 = lds_pairs(wvs + c0 + i);
+#pragma unroll
+              for (int u = 0; u < 2; ++u) {
+                const int k = (i >> 1) + u;  // pair index within the batch
+                // t = S rj + (na_i + nb_j)
+                const f2_t x = ffma2f(f2_pack(__uint_as_float(sv[i + 2 * u]), __uint_as_float(sv[i + 2 * u + 1])),
+                                      rj2, fadd2(u ? na2.y : na2.x, nb2));
+                float t0, t1;
+                f2_unpack(x, t0, t1);
+                f2_t pk;
+                if (((k * PP) & 15) < PP) {
+                  pk = exp2_poly2(f2_pack(fmaxf(t0, -125.f), fmaxf(t1, -125.f)));
+                } else {
+                  pk = f2_pack(ex2_approx(t0), ex2_approx(t1));
+                }
+                vacc2[u] = ffma2f(pk, u ? w2.y : w2.x, vacc2[u]);
+              }
             }
           }
         } else {
@@ -460,7 +485,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           vacc2[0] = vacc2[1] = 0ull;
         }
 #pragma unroll
-        for (int r = 0; r < RVA; ++r) { vacc[r] += (double)vblk[r]; vblk[r] = 0.f; }
+        for (int r = 0; r < RVA; ++r) { vacc[r] += (double)vblk[r] * wsc; vblk[r] = 0.f; }
         nblk = 0;
       }
       if (seg_end) {
@@ -705,7 +730,7 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
                                        const unsigned* __restrict__ amax, void* __restrict__ src_hi,
                                        void* __restrict__ src_lo, float* __restrict__ na,
                                        float* __restrict__ wt_hi, float* __restrict__ wt_lo,
-                                       float* __restrict__ wv, int rv) {
+                                       float* __restrict__ wv, int rv, const unsigned* __restrict__ wstat) {
   const int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   if (i >= m_pad) return;
@@ -741,7 +766,15 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
       static_cast<float*>(src_lo)[i * k_pad + d] = to_tf32(a - ah);
     }
   }
-  if (lane == 0) na[i] = aug ? 0.f : nai;  // aug: the norms ride in the contraction, the epilogue adds 0
+  if (lane == 0) {
+    if (wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u) {
+      // R = 1, W >= 0: fold the weight into the exponent, na_i + log2(W_i / Wmax) (-inf for W_i = 0)
+      const double wl = live ? log2((double)W[i]) - log2((double)__uint_as_float(wstat[0])) : -INFINITY;
+      na[i] = (float)((aug ? 0.0 : -c * n) + wl);
+    } else {
+      na[i] = aug ? 0.f : nai;  // aug: the norms ride in the contraction, the epilogue adds 0
+    }
+  }
   for (int r = lane; r < rv; r += 32) wv[i * rv + r] = (live && r < R) ? W[i * R + r] : 0.f;
   for (int r = lane; r < r_pad; r += 32) {
     const float w = (live && r < R) ? W[i * R + r] : 0.f;
@@ -812,6 +845,34 @@ __global__ void source_absmax_kernel(const float* __restrict__ alpha, int64_t to
   if ((threadIdx.x & 31) == 0) atomicMax(amax, __float_as_uint(m));
 }
 
+__global__ void weight_stats_kernel(const float* __restrict__ W, int64_t M, unsigned* __restrict__ wstat) {
+  float m = 0.f;
+  unsigned neg = 0u;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < M; e += (int64_t)gridDim.x * blockDim.x) {
+    const float w = W[e];
+    m = fmaxf(m, fabsf(w));
+    neg |= (w < 0.f || w != w) ? 1u : 0u;  // NaN weights take the general path
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    neg |= __shfl_xor_sync(0xffffffffu, neg, o);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    atomicMax(&wstat[0], __float_as_uint(m));
+    if (neg) atomicOr(&wstat[1], 1u);
+  }
+}
+
+cudaError_t launch_weight_stats(const float* W, int64_t M, unsigned* wstat, cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(wstat, 0, 2 * sizeof(unsigned), st);
+  if (e != cudaSuccess || M == 0) return e;
+  int64_t blocks = (M + 255) / 256;
+  if (blocks > 4 * 148) blocks = 4 * 148;
+  weight_stats_kernel<<<(unsigned)blocks, 256, 0, st>>>(W, M, wstat);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_source_absmax(const float* alpha, int64_t M, int K, const float* mu, unsigned* amax,
                                  cudaStream_t st) {
   cudaError_t e = cudaMemsetAsync(amax, 0, sizeof(unsigned), st);
@@ -826,22 +887,22 @@ cudaError_t launch_source_absmax(const float* alpha, int64_t M, int K, const flo
 cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
                                    int R, int r_pad, const float* mu, double c, int aug, float* src_hi,
                                    float* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv, int rv,
-                                   cudaStream_t st) {
+                                   const unsigned* wstat, cudaStream_t st) {
   if (m_pad == 0) return cudaSuccess;
   const int bs = 256;  // 8 points per block
   prep_tc_sources_kernel<false><<<(unsigned)((m_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
-      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, nullptr, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv);
+      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, nullptr, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv, wstat);
   return cudaGetLastError();
 }
 
 cudaError_t launch_prep_f16_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
                                     int R, int r_pad, const float* mu, double c, const unsigned* amax, void* src_hi,
                                     void* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv, int rv,
-                                    cudaStream_t st) {
+                                    const unsigned* wstat, cudaStream_t st) {
   if (m_pad == 0) return cudaSuccess;
   const int bs = 256;
   prep_tc_sources_kernel<true><<<(unsigned)((m_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
-      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, 0, amax, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv);
+      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, 0, amax, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv, wstat);
   return cudaGetLastError();
 }
 

@@ -73,6 +73,7 @@ struct TcArgs {
   int three;            // 1: three split products (hi.hi + hi.lo + lo.hi), 0: plain TF32 (hi.hi)
   int f16;              // 1: operands are the FP16 split of power-of-2 scaled values (kind::f16 MMA)
   const float* tsc;     // [n_pad] per-target factor on S: 1 (TF32 modes) or 2^-(eA+eB_j) (FP16 mode)
+  const unsigned* wstat;  // R = 1: {bits of max |W|, any W < 0}; na holds log-weights when W >= 0; else nullptr
   int aug;              // 1: norms folded into the contraction (2 extra K columns), epilogue adds nothing
   int vcc;              // RV > 0: weighted sum on CUDA cores over RV padded columns (no W^T tiles, no V MMA)
   const float* wv;      // [m_pad][RV] weights, zero padded (vcc)
@@ -93,7 +94,7 @@ struct TcArgs {
 cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
                                    int R, int r_pad, const float* mu, double c, int aug, float* src_hi,
                                    float* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv, int rv,
-                                   cudaStream_t st);
+                                   const unsigned* wstat, cudaStream_t st);
 // targets: tgt_hi/lo [n_pad][k_pad] = TF32 split of (beta - mu), nb [n_pad]
 // aug: columns K, K+1 hold (nb_j, 1)
 cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
@@ -106,12 +107,16 @@ cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, 
 // per row by sB_j = 2^(13 - e_j) from max_k |beta_jk - mu_k|; each scaled
 // value x is split x = hi + lo, hi = RN_f16(x), lo = RN_f16(x - hi);
 // tsc[j] = 2^-(log2 sA + log2 sB_j) undoes the scaling on S.
+// R = 1 weight statistics: wstat[0] = FP32 bits of max |W_i|, wstat[1] = 1 if any W_i < 0.
+// With W >= 0 and max > 0 the source prep stores na_i + log2(W_i / max) in na
+// (-inf for W_i = 0) and the fused kernel sums 2^t, scaling by max at the end.
+cudaError_t launch_weight_stats(const float* W, int64_t M, unsigned* wstat, cudaStream_t st);
 cudaError_t launch_source_absmax(const float* alpha, int64_t M, int K, const float* mu, unsigned* amax,
                                  cudaStream_t st);
 cudaError_t launch_prep_f16_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
                                     int R, int r_pad, const float* mu, double c, const unsigned* amax, void* src_hi,
                                     void* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv, int rv,
-                                    cudaStream_t st);
+                                    const unsigned* wstat, cudaStream_t st);
 cudaError_t launch_prep_f16_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
                                     double c, const unsigned* amax, void* tgt_hi, void* tgt_lo, float* nb,
                                     float* tsc, cudaStream_t st);

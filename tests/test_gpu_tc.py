@@ -133,3 +133,38 @@ def test_tensor_core_v_path(oracle_mod, monkeypatch, R):
     monkeypatch.setenv("KS_TC_VCC", "0")
     a, W, b, h = workloads.custom(2100, 333, 64, R, 3.0, seed=11 + R, wkind="signed")
     check(oracle_mod, a, W, b, h)
+
+
+@pytest.mark.parametrize("wcase", ["zeros", "all_zero", "one_negative", "tiny", "huge"])
+def test_r1_weight_modes(oracle_mod, wcase):
+    """R = 1: W >= 0 takes the log-weight epilogue (log2 W_i folded into the
+    exponent, -inf for W_i = 0, scaled back by max W); any negative weight
+    takes the general multiply path.  Both must meet the same bar."""
+    a, W, b, h = workloads.make(3, M=3000, N=700, wkind="pos")
+    W = W.copy()
+    if wcase == "zeros":
+        W[::3] = 0.0
+    elif wcase == "all_zero":
+        W[:] = 0.0
+    elif wcase == "one_negative":
+        W[17] = -0.5
+    elif wcase == "tiny":
+        W *= np.float32(1e-30)
+    elif wcase == "huge":
+        W *= np.float32(1e30)
+    V, info = gpu_eval(a, W, b, h)
+    Vr = oracle_mod.oracle_eval(a, W, b, float(h))
+    if wcase == "all_zero":
+        assert np.all(V == 0.0)
+        return
+    assert e_norm(V, Vr, W) <= TOL_3XTF32
+
+
+def test_r1_log_weights_match_general_path(oracle_mod, monkeypatch):
+    a, W, b, h = workloads.make(3, M=5000, N=900, wkind="pos")
+    V1, _ = gpu_eval(a, W, b, h)
+    monkeypatch.setenv("KS_TC_LOGW", "0")
+    V0, _ = gpu_eval(a, W, b, h)
+    Vr = oracle_mod.oracle_eval(a, W, b, float(h))
+    assert e_norm(V1, Vr, W) <= TOL_3XTF32 and e_norm(V0, Vr, W) <= TOL_3XTF32
+    assert np.max(np.abs(V1 - V0)) / np.abs(W).sum() <= 2 * TOL_3XTF32
