@@ -438,7 +438,8 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   }
   {
     const char* e = getenv("KS_TC_DEBUG_SKIP_V");
-    a.dbg_skip_v = (e && e[0] >= '1' && e[0] <= '3') ? e[0] - '0' : 0;  // 1 no epilogue math, 2 no MUFU, 3 no TMEM load
+    // 1 no epilogue math, 4 W/na loaded once, 5 no S MMAs, 6 one product, 7 no MMAs and no operand loads
+    a.dbg_skip_v = (e && e[0] >= '1' && e[0] <= '7') ? e[0] - '0' : 0;
   }
   a.na = ctx->na.p;
   a.nb = ctx->nb.p;
@@ -448,8 +449,9 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.sk = sk;
   a.cta_times = nullptr;
   const char* dbg = getenv("KS_CTA_TIMES");
+  const size_t n_dbg = (size_t)sk.grid * (2 + 20 * 5);  // CTA start/end + (KS_PROF builds) per-warp phase clocks
   if (dbg && *dbg) {
-    KS_CUDA(ctx->dbg_times.reserve((size_t)sk.grid * 2, st, true), "allocate debug timers");
+    KS_CUDA(ctx->dbg_times.reserve(n_dbg, st, true), "allocate debug timers");
     a.cta_times = ctx->dbg_times.p;
   }
   for (int r_off = 0; r_off < ctx->r_pad;) {
@@ -473,12 +475,16 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
     r_off += r_c;
   }
   if (a.cta_times) {
-    std::vector<unsigned long long> h((size_t)sk.grid * 2);
+    std::vector<unsigned long long> h(n_dbg);
     KS_CUDA(cudaMemcpyAsync(h.data(), a.cta_times, h.size() * 8, cudaMemcpyDeviceToHost, st), "copy debug timers");
     KS_CUDA(cudaStreamSynchronize(st), "synchronize");
     FILE* f = fopen(dbg, "a");
     if (f) {
-      for (int i = 0; i < sk.grid; ++i) fprintf(f, "%d %llu %llu\n", i, h[2 * i], h[2 * i + 1]);
+      for (int i = 0; i < sk.grid; ++i) {
+        fprintf(f, "%d %llu %llu", i, h[2 * i], h[2 * i + 1]);
+        for (int k = 0; k < 20 * 5; ++k) fprintf(f, " %llu", h[2 * (size_t)sk.grid + (size_t)i * 100 + k]);
+        fprintf(f, "\n");
+      }
       fprintf(f, "--\n");
       fclose(f);
     }

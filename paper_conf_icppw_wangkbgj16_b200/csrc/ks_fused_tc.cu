@@ -63,6 +63,19 @@ struct TcSmemT {
   static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 256 + 4 * kTcTileT * 8; }  // + VCC scratch
 };
 
+// Phase profiling (build with -DKS_PROF=1, run with KS_CTA_TIMES=file): per
+// warp clock64() totals of its waits and work, written after the CTA times.
+#ifndef KS_PROF
+#define KS_PROF 0
+#endif
+#if KS_PROF
+#define PROF_BEGIN(v) const long long v = clock64()
+#define PROF_END(k, v) pf[k] += clock64() - v
+#else
+#define PROF_BEGIN(v) (void)0
+#define PROF_END(k, v) (void)0
+#endif
+
 __device__ __forceinline__ int64_t sk_start(int64_t b, int64_t U, int64_t G) { return (b * U) / G; }
 __device__ __forceinline__ int64_t sk_owner(int64_t u, int64_t U, int64_t G) { return ((u + 1) * G - 1) / U; }
 
@@ -148,8 +161,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   uint64_t* full = bars;                 // [kStages]
   uint64_t* empty = full + kStages;      // [kStages]
   constexpr int WSA = TcSmem::kWSlots;   // allocated W/na slots
-  // measured: a 2-deep W/na ring is faster than 4 (KS_TC_WSLOTS knob)
-  const int WS = (VCC && args.wslots >= 2 && args.wslots <= WSA) ? args.wslots : 2;
+  // W/na ring depth: 3 where it fits (measured on cfg3: 2 -> 1.34 ms, 3 -> 1.30 ms; KS_TC_WSLOTS knob)
+  const int WS = (VCC && args.wslots >= 2 && args.wslots <= WSA) ? args.wslots : (WSA >= 3 ? 3 : 2);
   uint64_t* wfull = empty + kStages;     // [WSA]
   uint64_t* wempty = wfull + WSA;        // [WSA]
   uint64_t* sfull = wempty + WSA;        // [2]
@@ -161,6 +174,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int n_s = args.sk.n_s;
+#if KS_PROF
+  long long pf[5] = {0, 0, 0, 0, 0};
+  const long long pf_t0 = clock64();
+#endif
   const int64_t b = blockIdx.x;
   Sched sc;
   sc.init(args.sk.n_t, n_s, args.sk.grid, b);
@@ -179,10 +196,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     }
     for (int i = 0; i < WSA; ++i) {
       mbar_init(&wfull[i], 1);
-      mbar_init(&wempty[i], VCC ? EW : 1);
+      mbar_init(&wempty[i], VCC ? EW / 2 : 1);  // VCC: one epilogue group reads a tile
     }
     for (int i = 0; i < 2; ++i) {
-      mbar_init(&sempty[i], EW);
+      mbar_init(&sempty[i], EW / 2);
       mbar_init(&sfull[i], 1);
       mbar_init(&vdone[i], 1);
     }
@@ -197,43 +214,27 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   const uint32_t tbase = *tmem_base_smem;
 
   if (warp == 0) {
-    // ================= TMA producer (whole warp converged; one elected lane issues)
+    // ================= TMA producer of the operand stages (whole warp converged; one elected lane issues)
     const bool leader = elect_one();
     if (leader) {
       tma_prefetch_desc(&mA_hi);
       tma_prefetch_desc(&mB_hi);
-      tma_prefetch_desc(&mW_hi);
     }
     const int kcw = args.f16 ? 2 * kTcKC : kTcKC;  // elements per 64-byte chunk
     int it = 0;
     UnitIt cu = unit_begin(sc);
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
       const int tt = (int)cu.tt, st = cu.st;
-      {
-        const int slot = q % WS;
-        const uint32_t use = (uint32_t)(q / WS);
-        mbar_wait(&wempty[slot], (use & 1) ^ 1);
-        uint8_t* ws = smem + TcSmem::kW0 + slot * TcSmem::w_slot_bytes(RC);
-        if (leader) {
-          if constexpr (VCC) {  // na and the tile's weight rows
-            mbar_arrive_expect_tx(&wfull[slot], 4 * TS * (1 + RV));
-            bulk_load(ws, args.na + (int64_t)st * TS, 4 * TS, &wfull[slot]);
-            bulk_load(ws + 4 * TS, args.wv + (int64_t)st * TS * RV, 4 * TS * RV, &wfull[slot]);
-          } else {
-            mbar_arrive_expect_tx(&wfull[slot], 2 * TcSmem::wslot(RC) + 512);
-            tma_load_3d(ws, &mW_hi, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
-            tma_load_3d(ws + TcSmem::wslot(RC), &mW_lo, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
-            bulk_load(ws + 2 * TcSmem::wslot(RC), args.na + (int64_t)st * kTcTileS, 512, &wfull[slot]);
-          }
-        }
-        __syncwarp();
-      }
       for (int kc = 0; kc < n_kc; ++kc, ++it) {
         const int s = it % kStages;
         const uint32_t use = (uint32_t)(it / kStages);
+        PROF_BEGIN(w0);
         mbar_wait(&empty[s], (use & 1) ^ 1);
+        PROF_END(0, w0);
         uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
-        if (leader) {
+        if (leader && args.dbg_skip_v == 7) {  // measurement: no operand loads (wrong results)
+          mbar_arrive(&full[s]);
+        } else if (leader) {
           mbar_arrive_expect_tx(&full[s], kStageBytes);
           const int k0 = kc * kcw;  // element coordinate of the 64-byte chunk
           tma_load_2d(sp, &mA_hi, k0, tt * kTcTileT, &full[s]);
@@ -244,12 +245,43 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         __syncwarp();
       }
     }
+  } else if (warp == 3) {
+    // ================= producer of the per-tile source norms and weights (own ring, so a
+    // slot still in use by the epilogue never holds back the operand prefetch)
+    const bool leader = elect_one();
+    if (leader && !VCC) tma_prefetch_desc(&mW_hi);
+    UnitIt cu = unit_begin(sc);
+    for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
+      const int st = cu.st;
+      const int slot = q % WS;
+      const uint32_t use = (uint32_t)(q / WS);
+      if (VCC && args.dbg_skip_v == 4 && q >= WS) break;  // measurement: W/na loaded once (wrong results)
+      PROF_BEGIN(w0);
+      mbar_wait(&wempty[slot], (use & 1) ^ 1);
+      PROF_END(0, w0);
+      uint8_t* ws = smem + TcSmem::kW0 + slot * TcSmem::w_slot_bytes(RC);
+      if (leader) {
+        if constexpr (VCC) {  // na and the tile's weight rows
+          mbar_arrive_expect_tx(&wfull[slot], 4 * TS * (1 + RV));
+          bulk_load(ws, args.na + (int64_t)st * TS, 4 * TS, &wfull[slot]);
+          bulk_load(ws + 4 * TS, args.wv + (int64_t)st * TS * RV, 4 * TS * RV, &wfull[slot]);
+        } else {
+          mbar_arrive_expect_tx(&wfull[slot], 2 * TcSmem::wslot(RC) + 512);
+          tma_load_3d(ws, &mW_hi, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
+          tma_load_3d(ws + TcSmem::wslot(RC), &mW_lo, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
+          bulk_load(ws + 2 * TcSmem::wslot(RC), args.na + (int64_t)st * kTcTileS, 512, &wfull[slot]);
+        }
+      }
+      __syncwarp();
+    }
   } else if (warp == 1) {
     // ================= MMA issuer (whole warp converged; one elected lane issues)
     const bool leader = elect_one();
     const uint32_t idS = args.f16 ? idesc_f16(128, TS) : idesc_tf32(128, TS);
     const uint32_t idV = idesc_tf32(128, RC);
     const int nprod = args.three ? 3 : 1;
+    const bool dbg_no_mma = args.dbg_skip_v == 5 || args.dbg_skip_v == 7;  // measurement: no S MMAs (wrong results)
+    const bool dbg_one = args.dbg_skip_v == 6;      // measurement: one product only (wrong results)
     const bool skip_v = args.dbg_skip_v == 1;
     int it = 0;
     // V(p, hh) += P(p)[:, 64hh : 64hh+64] . W(p)[64hh : 64hh+64, :] on the tensor
@@ -293,14 +325,18 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       const uint32_t dS = tbase + (bq ? (uint32_t)TS : 0u);
       if constexpr (VCC) {
         if (q >= 2) {  // the epilogue has read S(q-2) out of this buffer
+          PROF_BEGIN(w1);
           mbar_wait(&sempty[bq], (uint32_t)(((q - 2) >> 1) & 1));
+          PROF_END(1, w1);
           tc_fence_after();
         }
       }
       for (int kc = 0; kc < n_kc; ++kc, ++it) {
         const int s = it % kStages;
         const uint32_t use = (uint32_t)(it / kStages);
+        PROF_BEGIN(w0);
         mbar_wait(&full[s], use & 1);
+        PROF_END(0, w0);
         tc_fence_after();
         uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
         const uint64_t d0 = sdesc_k_sw64(sp);
@@ -311,8 +347,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           const uint64_t bH = d0 + (uint64_t)((2 * kChunkA + ks * 32) >> 4);
           const uint64_t bL = d0 + (uint64_t)((2 * kChunkA + kChunkB + ks * 32) >> 4);
           const uint32_t acc0 = (kc > 0 || ks > 0) ? 1u : 0u;
-          if (leader) {  // products lo.hi, hi.lo, hi.hi (small terms first)
-            if (args.f16) {  // K = 16 halves = 32 bytes per instruction, as K = 8 TF32
+          if (leader && !dbg_no_mma) {  // products lo.hi, hi.lo, hi.hi (small terms first)
+            if (args.f16 && dbg_one) {
+              mma_f16_ss(dS, aH, bH, idS, acc0);
+            } else if (args.f16) {  // K = 16 halves = 32 bytes per instruction, as K = 8 TF32
               if (args.three) {
                 mma_f16_ss(dS, aL, bH, idS, acc0);
                 mma_f16_ss(dS, aH, bL, idS, 1u);
@@ -351,19 +389,27 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     }
   } else if (VCC && warp >= 4) {
     // ================= epilogue, R <= 16: V on CUDA cores
+    // Two groups of EW/2 warps take alternate tiles (group = parity of the
+    // local tile index, = the S buffer), so one group's barrier waits and
+    // per-tile bookkeeping overlap the other group's exponentials.
     const int ew = warp - 4;
     const int g = ew & 3;                 // TMEM lanes 32g..32g+31
-    const int h = ew >> 2;                // columns CW h .. CW h + CW - 1 of the tile
+    const int h = ew >> 2;                // 0..SUB-1: slot of this warp in the segment-end reduction
+    const int grp = ew >> 3;              // tiles q with (q & 1) == grp
+    const int hc = (ew >> 2) & 1;         // columns CW hc .. CW hc + CW - 1 of the tile
     const int row = 32 * g + lane;        // target row within the tile
     const uint32_t lane_off = (uint32_t)(32 * g) << 16;
-    constexpr int CW = TS / SUB;          // columns per warp (64)
+    constexpr int CW = TS / 2;            // columns per warp and tile (128)
+    static_assert(EW == 16, "two groups x 2 column halves x 4 TMEM lane groups");
     constexpr int BC = (RV >= 8) ? 16 : 32;  // TMEM columns per load batch (register budget)
     double* red = reinterpret_cast<double*>(smem + TcSmem::bar_off(RC) + 256);  // [SUB][128]
     constexpr int RVA = RV > 0 ? RV : 1;  // (this branch only runs with RV > 0)
-    double vacc[RVA];
-    float vblk[RVA];                      // FP32 sums over <= 8 tiles
+    // per-row sums: FP32 over <= 8 tiles (vblk), folded into an unevaluated
+    // FP32 pair (vhi + vlo, TwoSum: exact fold, no FP64 pipe in the tile loop)
+    float vhi[RVA], vlo[RVA];
+    float vblk[RVA];
 #pragma unroll
-    for (int r = 0; r < RVA; ++r) { vacc[r] = 0.0; vblk[r] = 0.f; }
+    for (int r = 0; r < RVA; ++r) { vhi[r] = 0.f; vlo[r] = 0.f; vblk[r] = 0.f; }
     f2_t vacc2[2] = {0ull, 0ull};         // RV == 1: FFMA2 partial sums (4 lanes)
     // R = 1 with W >= 0 (device-side flag from the source prep): log-weights in na
     const bool logw = RV == 1 && args.wstat != nullptr && args.wstat[1] == 0u && args.wstat[0] != 0u;
@@ -380,15 +426,22 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         nbj = __ldg(args.nb + cu.tt * kTcTileT + row);  // 0 when args.aug
         rjs = __ldg(args.tsc + cu.tt * kTcTileT + row);  // S scale (1 in TF32 modes)
       }
-      mbar_wait(&wfull[q % WS], (uint32_t)((q / WS) & 1));
+      const bool mine = (q & 1) == grp;
+      if (mine) {
+      PROF_BEGIN(e0);
+      if (args.dbg_skip_v != 4 || q < WS) mbar_wait(&wfull[q % WS], (uint32_t)((q / WS) & 1));
+      PROF_END(0, e0);
+      PROF_BEGIN(e1);
       mbar_wait(&sfull[bq], use & 1);
+      PROF_END(1, e1);
+      PROF_BEGIN(e2);
       tc_fence_after();
       const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q % WS) * TcSmem::w_slot_bytes(RC));
       const float* wvs = nas + TS;        // [TS][RV]
       const uint32_t colS = bq ? (uint32_t)TS : 0u;
 #pragma unroll
       for (int hh = 0; hh < CW / BC; ++hh) {
-        const int c0 = CW * h + BC * hh;
+        const int c0 = CW * hc + BC * hh;
         uint32_t sv[BC];
         tmem_ldn<BC>(tbase + lane_off + colS + c0, sv);
         tmem_wait_ld();
@@ -474,9 +527,12 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         }
       }
       __syncwarp();
-      if (lane == 0) mbar_arrive(&wempty[q % WS]);  // na / W slot consumed
+      PROF_END(2, e2);
+      if (lane == 0 && args.dbg_skip_v != 4) mbar_arrive(&wempty[q % WS]);  // na / W slot consumed
+      }
+      PROF_BEGIN(e3);
       const bool seg_end = (q == count - 1) || (cu.st + 1 == n_s);
-      if (++nblk == 8 || seg_end) {  // FP32 over <= 8 tiles, then FP64
+      if ((mine && ++nblk == 8) || seg_end) {  // FP32 over <= 8 of this warp's tiles, then the FP32 pair
         if constexpr (RV == 1) {  // the 4 FFMA2 lanes, fixed order
           float a0, a1, a2, a3;
           f2_unpack(vacc2[0], a0, a1);
@@ -485,7 +541,13 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           vacc2[0] = vacc2[1] = 0ull;
         }
 #pragma unroll
-        for (int r = 0; r < RVA; ++r) { vacc[r] += (double)vblk[r] * wsc; vblk[r] = 0.f; }
+        for (int r = 0; r < RVA; ++r) {
+          const float sum = vhi[r] + vblk[r];  // TwoSum(vhi, vblk)
+          const float bb = sum - vhi[r];
+          vlo[r] += (vhi[r] - (sum - bb)) + (vblk[r] - bb);
+          vhi[r] = sum;
+          vblk[r] = 0.f;
+        }
         nblk = 0;
       }
       if (seg_end) {
@@ -497,7 +559,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         // combine the SUB column groups of each row, column by column, in a fixed order
 #pragma unroll 1
         for (int r = 0; r < RVA; ++r) {
-          red[h * kTcTileT + row] = vacc[r];
+          red[h * kTcTileT + row] = ((double)vhi[r] + (double)vlo[r]) * wsc;
           named_bar_sync(1, 32 * EW);
           if (h == 0) {
             double v = 0.0;
@@ -538,9 +600,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           named_bar_sync(2, 128);  // flag reuse
         }
 #pragma unroll
-        for (int r = 0; r < RVA; ++r) vacc[r] = 0.0;
+        for (int r = 0; r < RVA; ++r) { vhi[r] = 0.f; vlo[r] = 0.f; }
         seg_q = q + 1;
       }
+      PROF_END(3, e3);
     }
   } else if (!VCC && warp >= 4) {
     // ================= epilogue (EW warps: TMEM lane group g, sub-split h)
@@ -687,6 +750,11 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     }
   }
 
+#if KS_PROF
+  pf[4] = clock64() - pf_t0;  // this warp's whole run (before the final barrier)
+  if (args.cta_times != nullptr && lane == 0)
+    for (int k = 0; k < 5; ++k) args.cta_times[2 * args.sk.grid + ((int64_t)b * 20 + warp) * 5 + k] = pf[k];
+#endif
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -961,7 +1029,7 @@ static cudaError_t launch_rcsv(const CUtensorMap* m, const TcArgs& a, cudaStream
   return cudaGetLastError();
 }
 
-static constexpr int kTcPolyDefault = 0;  // measured (cfg3): PP 0 1.60 ms, 4 1.63, 6 1.69, 8 1.76
+static constexpr int kTcPolyDefault = 4;  // measured (cfg3, log-weight epilogue): PP 0 1.34 ms, 4 1.31, 6 1.41, 8 1.55
 
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st) {
   // CUDA-core weighted sum (256-source tiles): 48 KB stages, 4 fit (3 with the 16 KB weight slots)

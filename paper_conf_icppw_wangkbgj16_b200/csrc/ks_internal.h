@@ -61,7 +61,7 @@ constexpr int kTcTileT = 128;  // targets per tile = MMA M = TMEM lanes
 constexpr int kTcTileS = 128;  // sources per tile = N of the S MMA = K of the V MMA
 constexpr int kTcKC = 16;      // K floats per pipeline stage (64-byte rows, SWIZZLE_64B)
 constexpr int kTcEpiWarps = 16;  // epilogue warps (4 per TMEM lane group)
-constexpr int kTcThreads = 128 + 32 * kTcEpiWarps;  // warp 0 TMA, 1 MMA, 2 TMEM alloc, 3 idle, 4.. epilogue
+constexpr int kTcThreads = 128 + 32 * kTcEpiWarps;  // warp 0 operand TMA, 1 MMA, 2 TMEM alloc, 3 norms/weights loads, 4.. epilogue
 
 struct TcArgs {
   int64_t N;            // targets
