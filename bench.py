@@ -336,16 +336,22 @@ def run_ours(args):
             deriv = ("MEASURED_PEAKS bf16_tflops (burst) %.1f x 0.5 (nominal TF32/BF16 = 1.1/2.25 "
                      "PFLOP/s)" % bf16) if bf16 else "fallback nominal dense TF32 1.1 PFLOP/s"
         achieved = pairs_launch * flops_pair / (kms / 1e3) / 1e12
-        roof = {"bound": "tensor", "kernel": "ks_fused_tc_kernel", "achieved": achieved, "peak": peak,
-                "unit": unit, "frac": achieved / peak,
-                "traffic": load_traffic(args.cfg, args.precision), "peak_derivation": deriv}
-        # co-bound: one MUFU ex2 per pair, 16 / clk / SM
+        tensor = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": unit, "frac": achieved / peak,
+                  "peak_derivation": deriv}
+        # the exponential: one 2^t per pair on MUFU.EX2 (16 / clk / SM), except the
+        # R = 1 epilogue's 4 of 16 that run as a polynomial on the FMA pipe
         sfu_peak = 16 * sms * max_mhz * 1e6
-        roof["sfu"] = {"achieved_ex2_per_s": pairs_launch / (kms / 1e3), "peak_ex2_per_s": sfu_peak,
-                       "frac": pairs_launch / (kms / 1e3) / sfu_peak,
-                       "peak_derivation": f"16 ex2/clk/SM x {sms} SMs x {max_mhz} MHz"}
+        ex2_rate = pairs_launch / (kms / 1e3)
+        sfu = {"bound": "alu", "achieved": ex2_rate / 1e9, "peak": sfu_peak / 1e9, "frac": ex2_rate / sfu_peak,
+               "unit": "G exponentials/s (MUFU.EX2 peak; R = 1 computes 1/4 of them on the FMA pipe)",
+               "peak_derivation": f"16 ex2/clk/SM x {sms} SMs x {max_mhz} MHz (sm_max)"}
+        # the binding resource is the primary roofline, the other the co-bound
+        prim, co = (sfu, tensor) if sfu["frac"] >= tensor["frac"] else (tensor, sfu)
+        roof = dict(prim)
+        roof.update({"kernel": "ks_fused_tc_kernel", "traffic": load_traffic(args.cfg, args.precision),
+                     "co_bound": co})
         if vcc:
-            # co-bound: CUDA-core epilogue, R FFMA (weighted sum) + 1 FADD (exponent) per pair
+            # CUDA-core epilogue, R FFMA (weighted sum) + 1 FADD (exponent) per pair
             ops = pairs_launch * (R + 1) / (kms / 1e3) / 1e12
             roof["fp32_epilogue"] = {"achieved": ops, "peak": 128 * sms * max_mhz * 1e6 / 1e12,
                                      "unit": "Top/s FP32-pipe lane ops (R+1 per pair)",

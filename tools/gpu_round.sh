@@ -7,6 +7,7 @@ python -c "import __graft_entry__ as g; g.build(); g.smoke()" > $OUT/smoke.log 2
 timeout 1200 python -m pytest tests -m gpu -x -q > $OUT/pytest_gpu.log 2>&1
 timeout 600 python bench.py > $OUT/bench.json 2> $OUT/bench.err
 timeout 600 python bench.py --precision fp32 --no-cpu-baseline > $OUT/bench_cfg3_fp32.json 2>&1
+timeout 600 python bench.py --precision 3xtf32 --no-cpu-baseline > $OUT/bench_cfg3_3xtf32.json 2>&1
 for c in 2 5; do timeout 900 python bench.py --cfg $c --steps 5 --no-cpu-baseline > $OUT/bench_cfg$c.json 2>&1; done
 for c in 2 5; do timeout 900 python bench.py --cfg $c --steps 5 --precision fp32 --no-cpu-baseline > $OUT/bench_cfg${c}_fp32.json 2>&1; done
 timeout 900 python bench.py --cfg 4 --steps 5 --warmup 2 --no-cpu-baseline > $OUT/bench_cfg4.json 2>&1
