@@ -147,6 +147,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
                        const __grid_constant__ CUtensorMap mW_hi, const __grid_constant__ CUtensorMap mW_lo,
                        const TcArgs args) {
   constexpr bool VCC = RV > 0;
+  // PP (R = 1 only): bits 0-3 = exponential pairs of every 16 computed on the FMA pipe;
+  // bit 4 = clamp d^2 >= 0 in the log-weight epilogue (t <= lw_i; off by default, Q8)
+  constexpr int NPOLY = PP & 15;
+  constexpr bool CLAMP_LW = (PP & 16) != 0;
   constexpr int TS = VCC ? 256 : kTcTileS;  // sources per tile
   using TcSmem = TcSmemT<kStages, TS, RV>;
   constexpr uint32_t kChunkB = TcSmem::kChunkB;
@@ -456,15 +460,16 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         }
         if constexpr (RV == 1) {
           // two elements per FADD2/FFMA2; PP of every 16 pairs take 2^t on the
-          // FMA pipe (exp2_poly2) instead of MUFU.EX2.  No clamp of t at 0
-          // here (reading Q12): rounding can leave t a few ulps
-          // above 0, as it can leave it below.
+          // FMA pipe (exp2_poly2) instead of MUFU.EX2
           const f2_t nb2 = f2_bcast(nbj), rj2 = f2_bcast(rjs);
           if (logw) {
-            // W >= 0: na_i carries + log2(W_i / Wmax), so V_j / Wmax = sum_i 2^t
+            // W >= 0: na_i carries + lw_i = log2(W_i / Wmax) and the W slot holds lw_i,
+            // so V_j / Wmax = sum_i 2^t; d^2 >= 0 <=> t <= lw_i (the clamp)
 #pragma unroll
             for (int i = 0; i < BC; i += 4) {
               const ulonglong2 na2 = lds_pairs(nas + c0 + i);
+              ulonglong2 lw2;
+              if constexpr (CLAMP_LW) lw2 = lds_pairs(wvs + c0 + i);
 #pragma unroll
               for (int u = 0; u < 2; ++u) {
                 const int k = (i >> 1) + u;
@@ -472,8 +477,14 @@ __global__ void __launch_bounds__(kTcThreads, 1)
                                       rj2, fadd2(u ? na2.y : na2.x, nb2));
                 float t0, t1;
                 f2_unpack(x, t0, t1);
+                if constexpr (CLAMP_LW) {  // clamp d^2 >= 0
+                  float l0, l1;
+                  f2_unpack(u ? lw2.y : lw2.x, l0, l1);
+                  t0 = fminf(t0, l0);
+                  t1 = fminf(t1, l1);
+                }
                 f2_t pk;
-                if (((k * PP) & 15) < PP) {
+                if (((k * NPOLY) & 15) < NPOLY) {
                   pk = exp2_poly2(f2_pack(fmaxf(t0, -125.f), fmaxf(t1, -125.f)));
                 } else {
                   pk = f2_pack(ex2_approx(t0), ex2_approx(t1));
@@ -494,8 +505,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
                                       rj2, fadd2(u ? na2.y : na2.x, nb2));
                 float t0, t1;
                 f2_unpack(x, t0, t1);
+                t0 = fminf(t0, 0.f);  // clamp d^2 >= 0
+                t1 = fminf(t1, 0.f);
                 f2_t pk;
-                if (((k * PP) & 15) < PP) {
+                if (((k * NPOLY) & 15) < NPOLY) {
                   pk = exp2_poly2(f2_pack(fmaxf(t0, -125.f), fmaxf(t1, -125.f)));
                 } else {
                   pk = f2_pack(ex2_approx(t0), ex2_approx(t1));
@@ -843,7 +856,13 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
       na[i] = aug ? 0.f : nai;  // aug: the norms ride in the contraction, the epilogue adds 0
     }
   }
-  for (int r = lane; r < rv; r += 32) wv[i * rv + r] = (live && r < R) ? W[i * R + r] : 0.f;
+  const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u;
+  for (int r = lane; r < rv; r += 32) {
+    if (logw)  // R = 1, W >= 0: the slot holds lw_i = log2(W_i / Wmax), the clamp bound (Q23)
+      wv[i * rv + r] = live ? (float)(log2((double)W[i]) - log2((double)__uint_as_float(wstat[0]))) : -INFINITY;
+    else
+      wv[i * rv + r] = (live && r < R) ? W[i * R + r] : 0.f;
+  }
   for (int r = lane; r < r_pad; r += 32) {
     const float w = (live && r < R) ? W[i * R + r] : 0.f;
     const float wh = to_tf32(w);
@@ -1035,15 +1054,14 @@ cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream
   // CUDA-core weighted sum (256-source tiles): 48 KB stages, 4 fit (3 with the 16 KB weight slots)
   switch (a.vcc) {
     case 1: {
-      // R = 1: PP of 16 exponential pairs on the FMA pipe (KS_TC_POLY = 0/4/6/8; measurement knob)
+      // R = 1: exponential pairs of 16 on the FMA pipe (KS_TC_POLY = 0 or 4; measured 6 and 8 slower)
+      // and the exact d^2 >= 0 clamp of the log-weight epilogue (KS_TC_CLAMP=1; costs 15% at cfg3)
       const char* e = getenv("KS_TC_POLY");
       const int pp = e ? atoi(e) : kTcPolyDefault;
-      switch (pp) {
-        case 0: return launch_rcsv<16, 4, 1, 0>(maps, a, st);
-        case 4: return launch_rcsv<16, 4, 1, 4>(maps, a, st);
-        case 8: return launch_rcsv<16, 4, 1, 8>(maps, a, st);
-        default: return launch_rcsv<16, 4, 1, 6>(maps, a, st);
-      }
+      const char* ec = getenv("KS_TC_CLAMP");
+      const bool clamp = ec && ec[0] == '1';
+      if (clamp) return pp == 0 ? launch_rcsv<16, 4, 1, 16>(maps, a, st) : launch_rcsv<16, 4, 1, 20>(maps, a, st);
+      return pp == 0 ? launch_rcsv<16, 4, 1, 0>(maps, a, st) : launch_rcsv<16, 4, 1, 4>(maps, a, st);
     }
     case 2: return launch_rcsv<16, 4, 2>(maps, a, st);
     case 4: return launch_rcsv<16, 4, 4>(maps, a, st);

@@ -168,3 +168,15 @@ def test_r1_log_weights_match_general_path(oracle_mod, monkeypatch):
     Vr = oracle_mod.oracle_eval(a, W, b, float(h))
     assert e_norm(V1, Vr, W) <= TOL_3XTF32 and e_norm(V0, Vr, W) <= TOL_3XTF32
     assert np.max(np.abs(V1 - V0)) / np.abs(W).sum() <= 2 * TOL_3XTF32
+
+
+@pytest.mark.parametrize("clamp", ["0", "1"])
+def test_r1_coincident_points_clamp_modes(oracle_mod, monkeypatch, clamp):
+    """beta == alpha (d^2 = 0 on the diagonal, where Eq.3 cancels): both the
+    default log-weight epilogue and its exact d^2 >= 0 clamp variant
+    (KS_TC_CLAMP=1, Q8) meet the bar."""
+    monkeypatch.setenv("KS_TC_CLAMP", clamp)
+    a, W, b, h = workloads.make(3, M=3000, N=3000, wkind="pos", same_points=True)
+    V, _ = gpu_eval(a, W, b, h)
+    Vr = oracle_mod.oracle_eval(a, W, b, float(h))
+    assert e_norm(V, Vr, W) <= TOL_3XTF32
