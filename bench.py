@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """bench.py -- Gaussian pair-interactions/s of the fused kernel summation on B200.
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--cfg 3] [--impl ours|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--cfg 3] [--impl ours|reference|unfused]
 
 One STEP is one pass of the whole hot path
 over one batch of synthetic input: ks_set_sources (a1: centre, norms,
@@ -26,6 +26,12 @@ launches in the timed region.
 
 --impl reference: the oracle itself (oracle/, plain FP64 CPU loop) timed on
 this host's cores, each step a bounded target sample of the same workload.
+--impl unfused: the paper's cuBLAS-Unfused design on this GPU (NEXT-1): SGEMM
+into HBM, elementwise kernel evaluation, GEMM with W (tools/unfused.py).
+
+"energy" (NEXT-4): board energy from NVML's total-energy counter over a loop
+of whole steps lasting --energy-seconds after the timed region (the counter
+updates too coarsely for a 20-step window): J per step and pairs per joule.
 """
 from __future__ import annotations
 
@@ -54,7 +60,10 @@ def parse():
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--cfg", type=int, default=3, help="BASELINE config id (1-based, SURVEY SS8(a))")
-    p.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    p.add_argument("--impl", choices=["ours", "reference", "unfused"], default="ours",
+                   help="unfused: the paper's cuBLAS-Unfused comparison (NEXT-1, tools/unfused.py)")
+    p.add_argument("--energy-seconds", type=float, default=1.0,
+                   help="length of the NVML energy loop after the timed region (0: skip)")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
     p.add_argument("--no-flush", action="store_true")
@@ -127,6 +136,35 @@ class ClockSampler:
         return {"sm_mhz": float(statistics.median(self.samples)), "sm_max_mhz": self.max_mhz,
                 "reasons": names, "samples": len(self.samples),
                 "sm_mhz_min": float(min(self.samples))}
+
+
+def energy_per_step(step, dev_index: int, seconds: float, sync):
+    """NEXT-4: NVML board energy (mJ counter) over >= `seconds` of whole steps."""
+    if seconds <= 0:
+        return None
+    try:
+        import pynvml
+        pynvml.nvmlInit()
+        hdl = pynvml.nvmlDeviceGetHandleByIndex(dev_index)
+        sync()
+        e0 = pynvml.nvmlDeviceGetTotalEnergyConsumption(hdl)
+        t0 = time.perf_counter()
+        n = 0
+        while True:
+            step()
+            n += 1
+            if n % 8 == 0:
+                sync()
+                if time.perf_counter() - t0 >= seconds:
+                    break
+        sync()
+        dt = time.perf_counter() - t0
+        e1 = pynvml.nvmlDeviceGetTotalEnergyConsumption(hdl)
+        j = (e1 - e0) / 1e3
+        return {"j_per_step": j / n, "avg_power_w": j / dt, "steps": n, "seconds": dt,
+                "source": "nvmlDeviceGetTotalEnergyConsumption (board, mJ), whole steps incl. L2 flush-free loop"}
+    except Exception as e:  # pragma: no cover - no NVML
+        return {"unavailable": str(e)}
 
 
 # ---------------------------------------------------------------- CPU baseline (the oracle)
@@ -317,7 +355,11 @@ def run_ours(args):
         # R <= 16 (256-source tiles): the weighted sum runs on CUDA cores and the
         # tensor work is the 2K contraction; R > 16: a second MMA adds 2R per pair
         vcc = info1["tile_s"] == 256
-        bf16 = load_peaks().get("bf16_tflops")
+        # burst peak for a kernel timed alone; the sustained (power-capped) one inside a long step
+        long_step = ms_per_step >= 20.0
+        pk = load_peaks()
+        bf16 = pk.get("bf16_tflops_sustained" if long_step else "bf16_tflops") or pk.get("bf16_tflops")
+        peak_kind = "sustained" if long_step and pk.get("bf16_tflops_sustained") else "burst"
         if f16:
             # S contraction on kind::f16 (BF16/FP16 rate); the R > 16 V-MMA stays TF32 and is
             # counted at twice its FLOPs (TF32 runs at half the FP16 rate): FP16-equivalent FLOPs
@@ -326,15 +368,15 @@ def run_ours(args):
             formula = ("%d products x 2K per pair" % nprod) if vcc else \
                       ("%d products x 2(K+2R) per pair, FP16-equivalent" % nprod)
             unit = "TFLOP/s (FP16 tensor; %s)" % formula
-            deriv = ("MEASURED_PEAKS bf16_tflops (burst) %.1f (kind::f16 = BF16 rate)" % bf16) if bf16 else \
+            deriv = ("MEASURED_PEAKS bf16 (%s) %.1f (kind::f16 = BF16 rate)" % (peak_kind, bf16)) if bf16 else \
                     "fallback nominal dense FP16 2.25 PFLOP/s"
         else:
             flops_pair = nprod * 2 * (K + (0 if vcc else R))
             peak = (bf16 * 0.5) if bf16 else 1100.0
             formula = ("%d products x 2K per pair" % nprod) if vcc else ("%d products x 2(K+R) per pair" % nprod)
             unit = "TFLOP/s (TF32 tensor; %s)" % formula
-            deriv = ("MEASURED_PEAKS bf16_tflops (burst) %.1f x 0.5 (nominal TF32/BF16 = 1.1/2.25 "
-                     "PFLOP/s)" % bf16) if bf16 else "fallback nominal dense TF32 1.1 PFLOP/s"
+            deriv = ("MEASURED_PEAKS bf16 (%s) %.1f x 0.5 (nominal TF32/BF16 = 1.1/2.25 "
+                     "PFLOP/s)" % (peak_kind, bf16)) if bf16 else "fallback nominal dense TF32 1.1 PFLOP/s"
         achieved = pairs_launch * flops_pair / (kms / 1e3) / 1e12
         tensor = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": unit, "frac": achieved / peak,
                   "peak_derivation": deriv}
@@ -370,6 +412,13 @@ def run_ours(args):
     roof.update({"kernel_ms": kms, "kernel_launches_per_step": kern_n / args.steps,
                  "kernel_share_of_step": kms / ms_per_step if ms_per_step else None,
                  "pairs_per_step": pairs_launch})
+
+    # ---- NEXT-4: board energy per step (NVML), world == 1 only
+    energy = None
+    if world == 1:
+        energy = energy_per_step(step, local, args.energy_seconds, torch.cuda.synchronize)
+        if energy and "j_per_step" in energy:
+            energy["pairs_per_joule"] = pairs_per_step / energy["j_per_step"]
 
     # ---- e2e through the C-ABI host entry points (pinned buffers, copies timed)
     ha = torch.from_numpy(a).pin_memory()
@@ -428,6 +477,8 @@ def run_ours(args):
                       "stages": info1["stages"]},
            "roofline": roof, "e2e": e2e, "clocks": clk_sum, "gpu_launches": launches,
            "gpu": torch.cuda.get_device_name(dev)}
+    if energy is not None:
+        out["energy"] = energy
 
     # ---- CPU baseline (oracle) on rank 0 at N=1 only; also a parity spot-check of the timed V
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -443,10 +494,77 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
+def run_unfused(args):
+    """NEXT-1: the paper's cuBLAS-Unfused comparison on this GPU,
+    same workload, same step (a1 prep + evaluation), same JSON line."""
+    import torch
+    sys.path.insert(0, os.path.join(ROOT, "tools"))
+    from unfused import hbm_bytes_per_pair, unfused_eval
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if rank != 0:
+        return
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    c = workloads.CONFIGS[args.cfg]
+    a, W, b, h = workloads.make(c)
+    M, N, K, R = c.M, c.N, c.K, c.R
+    ta, tw, tb = (torch.from_numpy(x).to(dev) for x in (a, W, b))
+    flush = None if args.no_flush else torch.empty(64 * 1024 * 1024, dtype=torch.float32, device=dev)
+    out_v = {}
+
+    def step():
+        out_v["V"] = unfused_eval(ta, tw, tb, float(h))
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    ev0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ev1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    with ClockSampler(local) as clk:
+        for i in range(args.steps):
+            if flush is not None:
+                l2_flush(flush)
+            ev0[i].record()
+            step()
+            ev1[i].record()
+        torch.cuda.synchronize()
+    ms = sum(s.elapsed_time(e) for s, e in zip(ev0, ev1)) / args.steps
+    pairs = M * N
+    energy = energy_per_step(step, local, args.energy_seconds, torch.cuda.synchronize)
+    if energy and "j_per_step" in energy:
+        energy["pairs_per_joule"] = pairs / energy["j_per_step"]
+    bpp = hbm_bytes_per_pair(R)
+    out = {"impl": "unfused", "metric": METRIC, "value": pairs / (ms / 1e3), "unit": UNIT, "n_gpus": 1,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+           "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+           "config": {"workload": workload_desc(c),
+                      "design": "cuBLAS SGEMM (FP32, TF32 off) of the centred, 2c-prescaled targets x sources "
+                                "into HBM, norm add + clamp + exp2 as PyTorch elementwise passes, cuBLAS GEMM "
+                                "with W; targets chunked to an 8 GiB intermediate (tools/unfused.py)",
+                      "l2": "flushed before every step"},
+           "hbm_bytes_per_pair": bpp,
+           "hbm_bound_ms": {k: v * pairs / (load_peaks().get("hbm_gbs", 6545.9) * 1e9) * 1e3 for k, v in bpp.items()},
+           "clocks": clk.summary(), "gpu": torch.cuda.get_device_name(dev)}
+    if energy is not None:
+        out["energy"] = energy
+    if not args.no_cpu_baseline:
+        import oracle
+        oracle.build()
+        J = workloads.sample_targets(N, 64, 7)
+        Vr = oracle.oracle_eval(a, W, b, float(h), J=J)
+        Vg = out_v["V"].cpu().numpy().astype(np.float64)[J]
+        out["parity_sampled"] = {"e_norm": float(np.max(np.abs(Vg - Vr).max(axis=0) / np.abs(W).sum(axis=0))),
+                                 "targets": int(len(J))}
+    print(json.dumps(out), flush=True)
+
+
 def main():
     args = parse()
     if args.impl == "reference":
         run_reference(args)
+    elif args.impl == "unfused":
+        run_unfused(args)
     else:
         run_ours(args)
 

@@ -1,0 +1,130 @@
+"""NEXT-2 + NEXT-4: the paper's workload grid (K in {32, 64, 128,
+256}, N = 1,024 targets, M from 1,024 to 524,288 sources) on one B200, fused
+(libks.so, AUTO) against the unfused cuBLAS design (tools/unfused.py; the
+paper's cuBLAS-Unfused), with NVML board energy per evaluation -- the B200
+analog of the paper's Fig. 6 (speedup) and Table III (energy saving).
+
+    python tools/grid.py [out_dir]     (GPU; writes grid.json and grid.md)
+
+Inputs: uniform points in [0,1]^K, W ~ U[0,1], h = sqrt(K)/4 (the paper does
+not state h; this keeps ||a-b||^2 / 2h^2 ~ 1.3 on average), seeds from
+workloads.custom.  One timed evaluation = set_sources + eval (both designs
+recompute the norms), CUDA events, median of repeats; energy = NVML total
+energy over >= 0.5 s of repeated evaluations.
+"""
+from __future__ import annotations
+
+import json
+import math
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+sys.path.insert(0, os.path.join(ROOT, "tools"))
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import oracle  # noqa: E402
+import paper_conf_icppw_wangkbgj16_b200 as ks  # noqa: E402
+import workloads  # noqa: E402
+from unfused import unfused_eval  # noqa: E402
+
+KS = (32, 64, 128, 256)
+MS = (1024, 8192, 131072, 524288)
+N = 1024
+
+
+def timed(fn, reps=None, min_s=0.2):
+    fn()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    fn()
+    torch.cuda.synchronize()
+    one = time.perf_counter() - t0
+    reps = reps or max(3, min(200, int(min_s / max(one, 1e-5))))
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+    for s, e in ev:
+        s.record()
+        fn()
+        e.record()
+    torch.cuda.synchronize()
+    return float(np.median([s.elapsed_time(e) for s, e in ev]))
+
+
+def energy(fn, hdl, seconds=0.5):
+    import pynvml
+    torch.cuda.synchronize()
+    e0 = pynvml.nvmlDeviceGetTotalEnergyConsumption(hdl)
+    t0 = time.perf_counter()
+    n = 0
+    while time.perf_counter() - t0 < seconds:
+        for _ in range(4):
+            fn()
+        n += 4
+        torch.cuda.synchronize()
+    e1 = pynvml.nvmlDeviceGetTotalEnergyConsumption(hdl)
+    return (e1 - e0) / 1e3 / n
+
+
+def main():
+    out_dir = sys.argv[1] if len(sys.argv) > 1 else os.path.join(ROOT, "profiles", "r01")
+    os.makedirs(out_dir, exist_ok=True)
+    import pynvml
+    pynvml.nvmlInit()
+    hdl = pynvml.nvmlDeviceGetHandleByIndex(0)
+    oracle.build()
+    dev = torch.device("cuda", 0)
+    rows = []
+    for K in KS:
+        for M in MS:
+            h = math.sqrt(K) / 4.0
+            a, W, b, h = workloads.custom(M, N, K, 1, h, dist="uniform", wkind="pos", seed=1000 * K + M % 997)
+            ta, tw, tb = (torch.from_numpy(x).to(dev) for x in (a, W, b))
+            plan = ks.KernelSum(K, float(h), "auto")
+            V = torch.empty((N, 1), device=dev)
+
+            def fused():
+                plan.set_sources(ta, tw)
+                plan.eval(tb, out=V)
+
+            def unf():
+                return unfused_eval(ta, tw, tb, float(h))
+
+            t_f = timed(fused)
+            t_u = timed(unf)
+            e_f = energy(fused, hdl)
+            e_u = energy(unf, hdl)
+            J = workloads.sample_targets(N, 16, K + M)
+            Vr = oracle.oracle_eval(a, W, b, float(h), J=J)
+            fused()
+            Vf = V.cpu().numpy().astype(np.float64)[J]
+            Vu = unf().cpu().numpy().astype(np.float64)[J]
+            sw = np.abs(W).sum()
+            info = plan.info()
+            plan.close()
+            r = {"K": K, "M": M, "N": N, "h": float(h), "fused_ms": t_f, "unfused_ms": t_u, "speedup": t_u / t_f,
+                 "fused_j": e_f, "unfused_j": e_u, "energy_saving": 1.0 - e_f / e_u,
+                 "fused_pairs_per_s": M * N / (t_f / 1e3),
+                 "fused_path": {1: "fp32", 2: "tcgen05"}.get(info["path"]),
+                 "e_norm_fused": float(np.max(np.abs(Vf - Vr)) / sw),
+                 "e_norm_unfused": float(np.max(np.abs(Vu - Vr)) / sw)}
+            rows.append(r)
+            print(json.dumps(r), flush=True)
+            del ta, tw, tb, V
+            torch.cuda.empty_cache()
+    json.dump(rows, open(os.path.join(out_dir, "grid.json"), "w"), indent=1)
+    lines = ["| K | M (N = 1,024) | fused ms | unfused ms | speedup | fused mJ | unfused mJ | energy saved | "
+             "fused e_norm | unfused e_norm |", "|---|---|---|---|---|---|---|---|---|---|"]
+    for r in rows:
+        lines.append(f"| {r['K']} | {r['M']:,} | {r['fused_ms']:.4f} | {r['unfused_ms']:.4f} | {r['speedup']:.2f}x | "
+                     f"{1e3 * r['fused_j']:.2f} | {1e3 * r['unfused_j']:.2f} | {100 * r['energy_saving']:.0f}% | "
+                     f"{r['e_norm_fused']:.1e} | {r['e_norm_unfused']:.1e} |")
+    open(os.path.join(out_dir, "grid.md"), "w").write("\n".join(lines) + "\n")
+    print("\n".join(lines))
+
+
+if __name__ == "__main__":
+    main()
