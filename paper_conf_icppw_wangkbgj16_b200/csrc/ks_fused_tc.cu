@@ -420,6 +420,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     const double wsc = logw ? (double)__uint_as_float(args.wstat[0]) : 1.0;
     int nblk = 0;
     float nbj = 0.f, rjs = 1.f;
+    const bool can_nbf = RV == 1 && logw && !CLAMP_LW;
+    bool nbfast = false;                  // this segment's rows take 2^nb_j out of the sum
+    double rowsc = 1.0;
     int seg_q = 0, seg_st0 = 0;
     UnitIt cu = unit_begin(sc);
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
@@ -429,6 +432,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         seg_st0 = cu.st;
         nbj = __ldg(args.nb + cu.tt * kTcTileT + row);  // 0 when args.aug
         rjs = __ldg(args.tsc + cu.tt * kTcTileT + row);  // S scale (1 in TF32 modes)
+        // factor 2^nb_j out of the row sum when 2^(t - nb_j) <= 2^64 cannot overflow (whole warp)
+        nbfast = can_nbf && __all_sync(0xffffffffu, nbj >= -64.f);
+        rowsc = nbfast ? exp2((double)nbj) : 1.0;
       }
       const bool mine = (q & 1) == grp;
       if (mine) {
@@ -462,7 +468,29 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           // two elements per FADD2/FFMA2; PP of every 16 pairs take 2^t on the
           // FMA pipe (exp2_poly2) instead of MUFU.EX2
           const f2_t nb2 = f2_bcast(nbj), rj2 = f2_bcast(rjs);
-          if (logw) {
+          if (logw && !CLAMP_LW && nbfast) {
+            // W >= 0 and nb_j factored out of the row (sig_j = nb_j >= -64 for the whole warp):
+            // V_j = Wmax 2^nb_j sum_i 2^(S rj + na_i + lw_i) -- one FFMA2 + exp2 + FADD2 per pair
+#pragma unroll
+            for (int i = 0; i < BC; i += 4) {
+              const ulonglong2 na2 = lds_pairs(nas + c0 + i);
+#pragma unroll
+              for (int u = 0; u < 2; ++u) {
+                const int k = (i >> 1) + u;
+                const f2_t x = ffma2f(f2_pack(__uint_as_float(sv[i + 2 * u]), __uint_as_float(sv[i + 2 * u + 1])),
+                                      rj2, u ? na2.y : na2.x);
+                float t0, t1;
+                f2_unpack(x, t0, t1);
+                f2_t pk;
+                if (((k * NPOLY) & 15) < NPOLY) {
+                  pk = exp2_poly2(f2_pack(fmaxf(t0, -125.f), fmaxf(t1, -125.f)));
+                } else {
+                  pk = f2_pack(ex2_approx(t0), ex2_approx(t1));
+                }
+                vacc2[u] = fadd2(vacc2[u], pk);
+              }
+            }
+          } else if (logw) {
             // W >= 0: na_i carries + lw_i = log2(W_i / Wmax) and the W slot holds lw_i,
             // so V_j / Wmax = sum_i 2^t; d^2 >= 0 <=> t <= lw_i (the clamp)
 #pragma unroll
@@ -572,7 +600,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         // combine the SUB column groups of each row, column by column, in a fixed order
 #pragma unroll 1
         for (int r = 0; r < RVA; ++r) {
-          red[h * kTcTileT + row] = ((double)vhi[r] + (double)vlo[r]) * wsc;
+          red[h * kTcTileT + row] = ((double)vhi[r] + (double)vlo[r]) * wsc * rowsc;
           named_bar_sync(1, 32 * EW);
           if (h == 0) {
             double v = 0.0;

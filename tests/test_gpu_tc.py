@@ -180,3 +180,14 @@ def test_r1_coincident_points_clamp_modes(oracle_mod, monkeypatch, clamp):
     V, _ = gpu_eval(a, W, b, h)
     Vr = oracle_mod.oracle_eval(a, W, b, float(h))
     assert e_norm(V, Vr, W) <= TOL_3XTF32
+
+
+@pytest.mark.parametrize("h", [0.15, 0.6])
+def test_r1_row_factor_paths(oracle_mod, h):
+    """R = 1, W >= 0: 2^nb_j is factored out of a row's sum when nb_j >= -64 for
+    the whole warp (h = 0.6: every row); otherwise the warp keeps nb_j inside
+    the exponent (h = 0.15 at K = 32: c ||beta_hat||^2 > 64 for most rows)."""
+    a, W, b, _ = workloads.custom(2500, 2500, 32, 1, h, wkind="pos", seed=77, same_points=True)
+    V, _ = gpu_eval(a, W, b, np.float32(h))
+    Vr = oracle_mod.oracle_eval(a, W, b, float(np.float32(h)))
+    assert e_norm(V, Vr, W) <= TOL_3XTF32
