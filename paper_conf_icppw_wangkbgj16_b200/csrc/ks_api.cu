@@ -127,6 +127,8 @@ struct ks_ctx {
   int tc_f16 = 0;
   int r_pad = 16;
   int tc_aug = 0;  // norms folded into the contraction as 2 extra K columns
+  int tc_fold = 0;  // FP16 R = 1 folded layout (6 extra hi-plane K columns)
+  int tc_kcols = 0, tc_kdims = 0;  // live operand columns / columns needing every split product
   int tc_vcc = 0;  // RV: weighted sum on CUDA cores over RV padded columns (0: tensor-core V path)
   CUtensorMap tmB_hi, tmB_lo;
   DBuf<float> mu;         // [k_pad]
@@ -320,12 +322,20 @@ int tc_k_pad(int K) { return (int)round_up(K + 2 * tc_aug(K), ks::kTcKC); }
 ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M, int R) {
   const int K = ctx->K;
   const bool f16 = ctx->prec_eff == KS_PREC_3XF16;
-  // k_pad in elements: one 64-byte row chunk per pipeline stage = 16 FP32 or 32 FP16
-  const int k_pad = f16 ? (int)round_up(K, 2 * ks::kTcKC) : tc_k_pad(K);
-  const int aug = f16 ? 0 : tc_aug(K);  // FP16 mode: norms stay in FP32 in the epilogue
   // R == 1: weighted sum on CUDA cores (KS_TC_VCC=0 forces the tensor-core V path; measurement knob)
   const char* ev = getenv("KS_TC_VCC");
   const int vcc = (ev && ev[0] == '0') ? 0 : ks::fused_tc_rv(R);
+  // R = 1 with W >= 0: log-weights in na (decided on the device, no host sync);
+  // KS_TC_LOGW=0 disables (measurement knob)
+  const char* elw = getenv("KS_TC_LOGW");
+  const bool use_wstat = (vcc == 1) && !(elw && elw[0] == '0');
+  // FP16, R = 1: folded layout (norms + log-weights as 6 extra hi-plane K columns, reading
+  // Q26; active on the device when c K amax^2 <= 2^12).  KS_TC_FOLD=0 disables (measurement knob)
+  const char* efo = getenv("KS_TC_FOLD");
+  const int fold = (f16 && use_wstat && !(efo && efo[0] == '0')) ? 1 : 0;
+  // k_pad in elements: one 64-byte row chunk per pipeline stage = 16 FP32 or 32 FP16
+  const int k_pad = f16 ? (int)round_up(K + 6 * fold, 2 * ks::kTcKC) : tc_k_pad(K);
+  const int aug = f16 ? 0 : tc_aug(K);  // FP16 mode: norms stay in FP32 in the epilogue (or fold)
   const int tile_s = ks::fused_tc_tile_s(vcc);
   const int64_t m_pad = round_up(M > 0 ? M : 1, tile_s);
   const int r_pad = (int)round_up(R, 16);
@@ -344,10 +354,6 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(ctx->mean_part.reserve((size_t)nparts * K, st, false), "allocate mean partials");
   KS_CUDA(ks::launch_source_mean(alpha, M, K, k_pad, ctx->mean_part.p, nparts, ctx->mu.p, st), "source mean");
   ctx->launches += (M > 0) ? 2 : 1;
-  // R = 1 with W >= 0: log-weights in na (decided on the device, no host sync);
-  // KS_TC_LOGW=0 disables (measurement knob)
-  const char* elw = getenv("KS_TC_LOGW");
-  const bool use_wstat = (vcc == 1) && !(elw && elw[0] == '0');
   if (use_wstat) {
     KS_CUDA(ctx->wstat.reserve(2, st, false), "allocate weight stats");
     KS_CUDA(ks::launch_weight_stats(W, M, ctx->wstat.p, st), "weight stats");
@@ -359,7 +365,7 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
     KS_CUDA(ks::launch_source_absmax(alpha, M, K, ctx->mu.p, ctx->amax.p, st), "source max (FP16 scaling)");
     ctx->launches += (M > 0) ? 1 : 0;
     KS_CUDA(ks::launch_prep_f16_sources(alpha, W, M, m_pad, K, k_pad, R, vcc ? 0 : r_pad, ctx->mu.p, ctx->c,
-                                        ctx->amax.p, ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p,
+                                        ctx->amax.p, fold, ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p,
                                         ctx->wt_lo.p, ctx->wv.p, vcc, wst, st),
             "source prep (TC, FP16)");
   } else {
@@ -377,6 +383,9 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   ctx->m_pad = m_pad;
   ctx->r_pad = r_pad;
   ctx->tc_aug = aug;
+  ctx->tc_fold = fold;
+  ctx->tc_kcols = f16 ? K + 6 * fold : K + 2 * aug;
+  ctx->tc_kdims = f16 ? K : K + 2 * aug;
   ctx->tc_vcc = vcc;
   ctx->tc_f16 = f16 ? 1 : 0;
   ctx->tc_wstat = use_wstat;
@@ -395,7 +404,7 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   KS_CUDA(ctx->tsc.reserve((size_t)n_pad, st, false), "allocate target scales");
   if (f16) {
     KS_CUDA(ks::launch_prep_f16_targets(beta, N, n_pad, ctx->K, k_pad, ctx->mu.p, ctx->c, ctx->amax.p,
-                                        ctx->tgt_hi.p, ctx->tgt_lo.p, ctx->nb.p, ctx->tsc.p, st),
+                                        ctx->tc_fold, ctx->tgt_hi.p, ctx->tgt_lo.p, ctx->nb.p, ctx->tsc.p, st),
             "target prep (TC, FP16)");
   } else {
     KS_CUDA(ks::launch_prep_tc_targets(beta, N, n_pad, ctx->K, k_pad, ctx->mu.p, ctx->c, ctx->tc_aug,
@@ -430,6 +439,12 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.wstat = ctx->tc_wstat ? ctx->wstat.p : nullptr;
   a.three = (ctx->prec_eff == KS_PREC_TF32) ? 0 : 1;
   a.aug = ctx->tc_aug;
+  a.kcols = ctx->tc_kcols;
+  a.kdims = ctx->tc_kdims;
+  a.fold = ctx->tc_fold;
+  a.amax = f16 ? ctx->amax.p : nullptr;
+  a.c = ctx->c;
+  a.K = ctx->K;
   a.wv = ctx->wv.p;
   a.vcc = ctx->tc_vcc;
   {

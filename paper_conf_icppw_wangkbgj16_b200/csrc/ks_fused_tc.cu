@@ -76,6 +76,35 @@ struct TcSmemT {
 #define PROF_END(k, v) (void)0
 #endif
 
+// ---- folded layout (FP16 split, R = 1; reading Q26 in DESIGN.md).  The
+// source norm (with the log-weight) and the target norm ride in the
+// contraction as three FP16 pieces each, so the accumulator already holds
+// t = -log2(e) ||alpha - beta||^2 / 2h^2 (+ log2 W_i / Wmax) and the epilogue
+// is exp2 + sum.  Columns K..K+2: A = (n1, n2, n3) of na_i, B = (1, 1, 1);
+// columns K+3..K+5: A = (1, 1, 1), B = (m1, m2, m3) of nb_j; hi planes only.
+// Operands are scaled by 2^eF (sources) and 2^-eF (targets), so S needs no
+// per-row factor.  Valid when c K amax^2 <= 2^12 (every |na_i| and every
+// kept |nb_j| < 2^15, FP16 range); evaluated identically by both prep kernels
+// and the fused kernel from amax, so no flag travels between them.
+__device__ __forceinline__ bool f16_fold_ok(const unsigned* amax, double c, int K) {
+  const double a = (double)__uint_as_float(*amax);
+  return c * (double)K * a * a <= 4096.0;
+}
+// balanced scaling: |2c x 2^eF| ~ |x 2^-eF| for coordinates of equal spread
+__device__ __forceinline__ int f16_fold_exp(double c) {
+  const int e = (int)rint(-0.5 * log2(2.0 * c));
+  return e < -60 ? -60 : (e > 60 ? 60 : e);
+}
+// x = p1 + p2 + p3 (FP16 pieces; |x| < 2^15): error <= max(2^-33 |x|, 2^-25)
+__device__ __forceinline__ void split3_f16(double x, __half* p) {
+  p[0] = __double2half(x);
+  const double r1 = x - (double)__half2float(p[0]);
+  p[1] = __double2half(r1);
+  p[2] = __double2half(r1 - (double)__half2float(p[1]));
+}
+constexpr double kFoldFar = 16384.0;   // c ||beta_hat_j||^2 above this: every kernel value of row j is < 2^-4096
+constexpr float kFoldNegInf = -32768.f;  // stands for -inf in FP16 operands (no inf * 0 in the MMA)
+
 __device__ __forceinline__ int64_t sk_start(int64_t b, int64_t U, int64_t G) { return (b * U) / G; }
 __device__ __forceinline__ int64_t sk_owner(int64_t u, int64_t U, int64_t G) { return ((u + 1) * G - 1) / U; }
 
@@ -149,7 +178,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   constexpr bool VCC = RV > 0;
   // PP (R = 1 only): bits 0-3 = exponential pairs of every 16 computed on the FMA pipe;
   // bit 4 = clamp d^2 >= 0 in the log-weight epilogue (t <= lw_i; off by default, Q8)
-  constexpr int NPOLY = PP & 15;
+  constexpr int NPOLY = PP & 15;                    // folded epilogue (exp2 + sum)
+  constexpr int NPOLY_U = NPOLY > 4 ? 4 : NPOLY;    // unfolded epilogues (more FMA-pipe work per pair)
   constexpr bool CLAMP_LW = (PP & 16) != 0;
   constexpr int TS = VCC ? 256 : kTcTileS;  // sources per tile
   using TcSmem = TcSmemT<kStages, TS, RV>;
@@ -182,6 +212,11 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   long long pf[5] = {0, 0, 0, 0, 0};
   const long long pf_t0 = clock64();
 #endif
+  // R = 1: W >= 0 (log-weights) and the folded layout active -> the epilogue is exp2 + sum
+  // of the raw accumulator and needs no per-tile norms or weights (no W/na ring)
+  const bool logw_k = RV == 1 && args.wstat != nullptr && args.wstat[1] == 0u && args.wstat[0] != 0u;
+  const bool fold_k = RV == 1 && args.fold && f16_fold_ok(args.amax, args.c, args.K);
+  const bool ring = !(logw_k && fold_k && !CLAMP_LW);
   const int64_t b = blockIdx.x;
   Sched sc;
   sc.init(args.sk.n_t, n_s, args.sk.grid, b);
@@ -239,12 +274,13 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         if (leader && args.dbg_skip_v == 7) {  // measurement: no operand loads (wrong results)
           mbar_arrive(&full[s]);
         } else if (leader) {
-          mbar_arrive_expect_tx(&full[s], kStageBytes);
           const int k0 = kc * kcw;  // element coordinate of the 64-byte chunk
+          const bool lo = k0 < args.kdims;  // chunks holding only folded norm columns: hi planes only
+          mbar_arrive_expect_tx(&full[s], lo ? kStageBytes : kChunkA + kChunkB);
           tma_load_2d(sp, &mA_hi, k0, tt * kTcTileT, &full[s]);
-          tma_load_2d(sp + kChunkA, &mA_lo, k0, tt * kTcTileT, &full[s]);
+          if (lo) tma_load_2d(sp + kChunkA, &mA_lo, k0, tt * kTcTileT, &full[s]);
           tma_load_2d(sp + 2 * kChunkA, &mB_hi, k0, st * TS, &full[s]);
-          tma_load_2d(sp + 2 * kChunkA + kChunkB, &mB_lo, k0, st * TS, &full[s]);
+          if (lo) tma_load_2d(sp + 2 * kChunkA + kChunkB, &mB_lo, k0, st * TS, &full[s]);
         }
         __syncwarp();
       }
@@ -255,7 +291,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     const bool leader = elect_one();
     if (leader && !VCC) tma_prefetch_desc(&mW_hi);
     UnitIt cu = unit_begin(sc);
-    for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
+    for (int q = 0; q < (ring ? count : 0); ++q, unit_next(sc, cu)) {
       const int st = cu.st;
       const int slot = q % WS;
       const uint32_t use = (uint32_t)(q / WS);
@@ -284,6 +320,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     const uint32_t idS = args.f16 ? idesc_f16(128, TS) : idesc_tf32(128, TS);
     const uint32_t idV = idesc_tf32(128, RC);
     const int nprod = args.three ? 3 : 1;
+    const int kcw = args.f16 ? 2 * kTcKC : kTcKC;  // elements per 64-byte chunk
     const bool dbg_no_mma = args.dbg_skip_v == 5 || args.dbg_skip_v == 7;  // measurement: no S MMAs (wrong results)
     const bool dbg_one = args.dbg_skip_v == 6;      // measurement: one product only (wrong results)
     const bool skip_v = args.dbg_skip_v == 1;
@@ -351,8 +388,14 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           const uint64_t bH = d0 + (uint64_t)((2 * kChunkA + ks * 32) >> 4);
           const uint64_t bL = d0 + (uint64_t)((2 * kChunkA + kChunkB + ks * 32) >> 4);
           const uint32_t acc0 = (kc > 0 || ks > 0) ? 1u : 0u;
+          const int col0 = kc * kcw + ks * (kcw / 2);  // first element column of this K step
+          if (col0 >= args.kcols) continue;            // all-zero padding step
+          const bool hh_only = col0 >= args.kdims;     // folded norm columns only: hi planes
           if (leader && !dbg_no_mma) {  // products lo.hi, hi.lo, hi.hi (small terms first)
-            if (args.f16 && dbg_one) {
+            if (hh_only) {
+              if (args.f16) mma_f16_ss(dS, aH, bH, idS, acc0);
+              else mma_tf32_ss(dS, aH, bH, idS, acc0);
+            } else if (args.f16 && dbg_one) {
               mma_f16_ss(dS, aH, bH, idS, acc0);
             } else if (args.f16) {  // K = 16 halves = 32 bytes per instruction, as K = 8 TF32
               if (args.three) {
@@ -439,7 +482,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       const bool mine = (q & 1) == grp;
       if (mine) {
       PROF_BEGIN(e0);
-      if (args.dbg_skip_v != 4 || q < WS) mbar_wait(&wfull[q % WS], (uint32_t)((q / WS) & 1));
+      if (ring && (args.dbg_skip_v != 4 || q < WS)) mbar_wait(&wfull[q % WS], (uint32_t)((q / WS) & 1));
       PROF_END(0, e0);
       PROF_BEGIN(e1);
       mbar_wait(&sfull[bq], use & 1);
@@ -468,7 +511,21 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           // two elements per FADD2/FFMA2; PP of every 16 pairs take 2^t on the
           // FMA pipe (exp2_poly2) instead of MUFU.EX2
           const f2_t nb2 = f2_bcast(nbj), rj2 = f2_bcast(rjs);
-          if (logw && !CLAMP_LW && nbfast) {
+          if (!ring) {
+            // folded layout, W >= 0: S = t already (norms and log2 W_i / Wmax in the
+            // contraction, reading Q26): V_j = Wmax sum_i 2^S -- exp2 + FADD2 per pair
+#pragma unroll
+            for (int i = 0; i < BC; i += 2) {
+              const int k = i >> 1;
+              f2_t pk;
+              if (((k * NPOLY) & 15) < NPOLY) {
+                pk = exp2_poly2(f2_pack(fmaxf(__uint_as_float(sv[i]), -125.f), fmaxf(__uint_as_float(sv[i + 1]), -125.f)));
+              } else {
+                pk = f2_pack(ex2_approx(__uint_as_float(sv[i])), ex2_approx(__uint_as_float(sv[i + 1])));
+              }
+              vacc2[k & 1] = fadd2(vacc2[k & 1], pk);
+            }
+          } else if (logw && !CLAMP_LW && nbfast) {
             // W >= 0 and nb_j factored out of the row (sig_j = nb_j >= -64 for the whole warp):
             // V_j = Wmax 2^nb_j sum_i 2^(S rj + na_i + lw_i) -- one FFMA2 + exp2 + FADD2 per pair
 #pragma unroll
@@ -482,7 +539,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
                 float t0, t1;
                 f2_unpack(x, t0, t1);
                 f2_t pk;
-                if (((k * NPOLY) & 15) < NPOLY) {
+                if (((k * NPOLY_U) & 15) < NPOLY_U) {
                   pk = exp2_poly2(f2_pack(fmaxf(t0, -125.f), fmaxf(t1, -125.f)));
                 } else {
                   pk = f2_pack(ex2_approx(t0), ex2_approx(t1));
@@ -512,7 +569,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
                   t1 = fminf(t1, l1);
                 }
                 f2_t pk;
-                if (((k * NPOLY) & 15) < NPOLY) {
+                if (((k * NPOLY_U) & 15) < NPOLY_U) {
                   pk = exp2_poly2(f2_pack(fmaxf(t0, -125.f), fmaxf(t1, -125.f)));
                 } else {
                   pk = f2_pack(ex2_approx(t0), ex2_approx(t1));
@@ -536,7 +593,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
                 t0 = fminf(t0, 0.f);  // clamp d^2 >= 0
                 t1 = fminf(t1, 0.f);
                 f2_t pk;
-                if (((k * NPOLY) & 15) < NPOLY) {
+                if (((k * NPOLY_U) & 15) < NPOLY_U) {
                   pk = exp2_poly2(f2_pack(fmaxf(t0, -125.f), fmaxf(t1, -125.f)));
                 } else {
                   pk = f2_pack(ex2_approx(t0), ex2_approx(t1));
@@ -569,7 +626,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       }
       __syncwarp();
       PROF_END(2, e2);
-      if (lane == 0 && args.dbg_skip_v != 4) mbar_arrive(&wempty[q % WS]);  // na / W slot consumed
+      if (ring && lane == 0 && args.dbg_skip_v != 4) mbar_arrive(&wempty[q % WS]);  // na / W slot consumed
       }
       PROF_BEGIN(e3);
       const bool seg_end = (q == count - 1) || (cu.st + 1 == n_s);
@@ -832,6 +889,7 @@ __device__ __forceinline__ void split_f16(float x, __half& hi, __half& lo) {
   lo = __float2half_rn(x - __half2float(hi));  // x - hi is exact in FP32
 }
 
+
 template <bool F16>
 __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const float* __restrict__ W, int64_t M,
                                        int64_t m_pad, int K, int k_pad, int R, int r_pad,
@@ -852,8 +910,23 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
   n = warp_sum_fixed(n);
   const float nai = live ? (float)(-c * n) : 0.f;
   const double c2 = 2.0 * c;
+  const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u;
+  // log2(W_i / Wmax) (R = 1, W >= 0; -inf for W_i = 0 and padding)
+  const double wl = !logw ? 0.0 : live ? log2((double)W[i]) - log2((double)__uint_as_float(wstat[0])) : -INFINITY;
   float sA = 1.f;
-  if constexpr (F16) sA = ldexpf(1.f, f16_scale_exp((float)(c2 * (double)__uint_as_float(*amax))));
+  bool fa = false;  // folded layout active
+  __half np[3] = {__float2half(0.f), __float2half(0.f), __float2half(0.f)};
+  if constexpr (F16) {
+    fa = aug && f16_fold_ok(amax, c, K);
+    if (fa) {
+      sA = ldexpf(1.f, f16_fold_exp(c));
+      const double nf = -c * n + wl;  // finite unless W_i = 0: then the FP16 stand-in for -inf
+      if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
+      else split3_f16(nf, np);
+    } else {
+      sA = ldexpf(1.f, f16_scale_exp((float)(c2 * (double)__uint_as_float(*amax))));
+    }
+  }
   for (int d = lane; d < k_pad; d += 32) {
     float a = 0.f;
     if (d < K) {
@@ -867,6 +940,10 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
     if constexpr (F16) {
       __half h, l;
       split_f16(a * sA, h, l);  // exact power-of-2 scaling
+      if (fa && d >= K && d < K + 6) {  // folded norm columns: hi planes only
+        h = d < K + 3 ? np[d - K] : __float2half(1.f);
+        l = __float2half(0.f);
+      }
       static_cast<__half*>(src_hi)[i * k_pad + d] = h;
       static_cast<__half*>(src_lo)[i * k_pad + d] = l;
     } else {
@@ -876,15 +953,15 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
     }
   }
   if (lane == 0) {
-    if (wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u) {
+    if (fa) {
+      na[i] = 0.f;  // folded: the norm and log-weight ride in the contraction
+    } else if (logw) {
       // R = 1, W >= 0: fold the weight into the exponent, na_i + log2(W_i / Wmax) (-inf for W_i = 0)
-      const double wl = live ? log2((double)W[i]) - log2((double)__uint_as_float(wstat[0])) : -INFINITY;
-      na[i] = (float)((aug ? 0.0 : -c * n) + wl);
+      na[i] = (float)((aug && !F16 ? 0.0 : -c * n) + wl);
     } else {
-      na[i] = aug ? 0.f : nai;  // aug: the norms ride in the contraction, the epilogue adds 0
+      na[i] = aug && !F16 ? 0.f : nai;  // aug: the norms ride in the contraction, the epilogue adds 0
     }
   }
-  const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u;
   for (int r = lane; r < rv; r += 32) {
     if (logw)  // R = 1, W >= 0: the slot holds lw_i = log2(W_i / Wmax), the clamp bound (Q23)
       wv[i * rv + r] = live ? (float)(log2((double)W[i]) - log2((double)__uint_as_float(wstat[0]))) : -INFINITY;
@@ -919,22 +996,36 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
   n = warp_sum_fixed(n);
   const float nbj = live ? (float)(-c * n) : 0.f;
   float sB = 1.f, rj = 1.f;
+  bool fa = false, far = false;  // folded layout active; row beyond every source (kernel row 0)
+  __half mp[3] = {__float2half(0.f), __float2half(0.f), __float2half(0.f)};
   if constexpr (F16) {
+    fa = aug && f16_fold_ok(amax, c, K);
+    if (fa) {
+      sB = ldexpf(1.f, -f16_fold_exp(c));
+      far = c * n > kFoldFar;
+      if (far) mp[0] = __float2half(kFoldNegInf);
+      else split3_f16(-c * n, mp);
+    } else {
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) bmax = fmaxf(bmax, __shfl_xor_sync(0xffffffffu, bmax, o));
-    const int eA = f16_scale_exp((float)(2.0 * c * (double)__uint_as_float(*amax)));
-    const int eB = f16_scale_exp(bmax);
-    sB = ldexpf(1.f, eB);
-    rj = ldexpf(1.f, -(eA + eB));
+      for (int o = 16; o > 0; o >>= 1) bmax = fmaxf(bmax, __shfl_xor_sync(0xffffffffu, bmax, o));
+      const int eA = f16_scale_exp((float)(2.0 * c * (double)__uint_as_float(*amax)));
+      const int eB = f16_scale_exp(bmax);
+      sB = ldexpf(1.f, eB);
+      rj = ldexpf(1.f, -(eA + eB));
+    }
   }
   for (int d = lane; d < k_pad; d += 32) {
     float x = 0.f;
-    if (d < K) x = live ? beta[j * K + d] - mu[d] : 0.f;
+    if (d < K) x = (live && !far) ? beta[j * K + d] - mu[d] : 0.f;
     else if (!F16 && aug && d == K) x = nbj;
     else if (!F16 && aug && d == K + 1) x = 1.f;
     if constexpr (F16) {
       __half h, l;
       split_f16(x * sB, h, l);
+      if (fa && d >= K && d < K + 6) {  // folded norm columns: hi planes only
+        h = d < K + 3 ? __float2half(1.f) : mp[d - K - 3];
+        l = __float2half(0.f);
+      }
       static_cast<__half*>(tgt_hi)[j * k_pad + d] = h;
       static_cast<__half*>(tgt_lo)[j * k_pad + d] = l;
     } else {
@@ -944,7 +1035,7 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
     }
   }
   if (lane == 0) {
-    nb[j] = aug ? 0.f : nbj;
+    nb[j] = aug ? 0.f : nbj;  // aug (TF32) / folded (FP16): the norm rides in the contraction
     tsc[j] = rj;
   }
 }
@@ -1011,13 +1102,13 @@ cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M
 }
 
 cudaError_t launch_prep_f16_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
-                                    int R, int r_pad, const float* mu, double c, const unsigned* amax, void* src_hi,
-                                    void* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv, int rv,
-                                    const unsigned* wstat, cudaStream_t st) {
+                                    int R, int r_pad, const float* mu, double c, const unsigned* amax, int fold,
+                                    void* src_hi, void* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv,
+                                    int rv, const unsigned* wstat, cudaStream_t st) {
   if (m_pad == 0) return cudaSuccess;
   const int bs = 256;
   prep_tc_sources_kernel<true><<<(unsigned)((m_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
-      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, 0, amax, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv, wstat);
+      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, fold, amax, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv, wstat);
   return cudaGetLastError();
 }
 
@@ -1032,12 +1123,12 @@ cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, 
 }
 
 cudaError_t launch_prep_f16_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
-                                    double c, const unsigned* amax, void* tgt_hi, void* tgt_lo, float* nb,
+                                    double c, const unsigned* amax, int fold, void* tgt_hi, void* tgt_lo, float* nb,
                                     float* tsc, cudaStream_t st) {
   if (n_pad == 0) return cudaSuccess;
   const int bs = 256;
   prep_tc_targets_kernel<true><<<(unsigned)((n_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
-      beta, N, n_pad, K, k_pad, mu, c, 0, amax, tgt_hi, tgt_lo, nb, tsc);
+      beta, N, n_pad, K, k_pad, mu, c, fold, amax, tgt_hi, tgt_lo, nb, tsc);
   return cudaGetLastError();
 }
 
@@ -1076,20 +1167,28 @@ static cudaError_t launch_rcsv(const CUtensorMap* m, const TcArgs& a, cudaStream
   return cudaGetLastError();
 }
 
-static constexpr int kTcPolyDefault = 4;  // measured (cfg3, log-weight epilogue): PP 0 1.34 ms, 4 1.31, 6 1.41, 8 1.55
+// exponential pairs of 16 on the FMA pipe, measured (kernel ms): unfolded log-weight epilogue cfg3
+// PP 0 1.34, 4 1.31, 6 1.41, 8 1.55; folded layout cfg3 PP 0 1.135, 4 1.057, 6 1.046, 8 1.150,
+// cfg5 301.0 / 270.2 / 254.7 / 284.7, cfg2 0.091 / 0.085 / 0.081 / 0.089
+static constexpr int kTcPolyDefault = 6;
 
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st) {
   // CUDA-core weighted sum (256-source tiles): 48 KB stages, 4 fit (3 with the 16 KB weight slots)
   switch (a.vcc) {
     case 1: {
-      // R = 1: exponential pairs of 16 on the FMA pipe (KS_TC_POLY = 0 or 4; measured 6 and 8 slower)
+      // R = 1: exponential pairs of 16 on the FMA pipe (KS_TC_POLY = 0, 4, 6 or 8)
       // and the exact d^2 >= 0 clamp of the log-weight epilogue (KS_TC_CLAMP=1; costs 15% at cfg3)
       const char* e = getenv("KS_TC_POLY");
       const int pp = e ? atoi(e) : kTcPolyDefault;
       const char* ec = getenv("KS_TC_CLAMP");
       const bool clamp = ec && ec[0] == '1';
       if (clamp) return pp == 0 ? launch_rcsv<16, 4, 1, 16>(maps, a, st) : launch_rcsv<16, 4, 1, 20>(maps, a, st);
-      return pp == 0 ? launch_rcsv<16, 4, 1, 0>(maps, a, st) : launch_rcsv<16, 4, 1, 4>(maps, a, st);
+      switch (pp) {
+        case 0: return launch_rcsv<16, 4, 1, 0>(maps, a, st);
+        case 4: return launch_rcsv<16, 4, 1, 4>(maps, a, st);
+        case 8: return launch_rcsv<16, 4, 1, 8>(maps, a, st);
+        default: return launch_rcsv<16, 4, 1, 6>(maps, a, st);
+      }
     }
     case 2: return launch_rcsv<16, 4, 2>(maps, a, st);
     case 4: return launch_rcsv<16, 4, 4>(maps, a, st);

@@ -75,6 +75,13 @@ struct TcArgs {
   const float* tsc;     // [n_pad] per-target factor on S: 1 (TF32 modes) or 2^-(eA+eB_j) (FP16 mode)
   const unsigned* wstat;  // R = 1: {bits of max |W|, any W < 0}; na holds log-weights when W >= 0; else nullptr
   int aug;              // 1: norms folded into the contraction (2 extra K columns), epilogue adds nothing
+  int kcols;            // operand columns (elements) that can be nonzero: MMA K steps at or past it are skipped
+  int kdims;            // columns that need every split product; steps holding only [kdims, kcols) run hi.hi
+  int fold;             // FP16, R = 1: folded layout (norms + log-weight in 6 hi-plane columns); active on the
+                        // device iff f16_fold_ok(amax, c, K) (prep and kernel evaluate the same test)
+  const unsigned* amax; // FP16: bits of max |alpha - mu|
+  double c;             // log2(e) / (2 h^2)
+  int K;
   int vcc;              // RV > 0: weighted sum on CUDA cores over RV padded columns (no W^T tiles, no V MMA)
   const float* wv;      // [m_pad][RV] weights, zero padded (vcc)
   int wslots;           // VCC W/na ring depth (2..4; 0 = default)
@@ -113,12 +120,15 @@ cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, 
 cudaError_t launch_weight_stats(const float* W, int64_t M, unsigned* wstat, cudaStream_t st);
 cudaError_t launch_source_absmax(const float* alpha, int64_t M, int K, const float* mu, unsigned* amax,
                                  cudaStream_t st);
+// fold = 1 (R = 1): folded layout, k_pad >= K + 6 -- columns K..K+5 carry the
+// norms (and log-weights) as FP16 pieces when c K amax^2 <= 2^12 (checked on
+// the device); operands are then scaled by 2^eF / 2^-eF and tsc = 1, nb = na = 0.
 cudaError_t launch_prep_f16_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
-                                    int R, int r_pad, const float* mu, double c, const unsigned* amax, void* src_hi,
-                                    void* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv, int rv,
-                                    const unsigned* wstat, cudaStream_t st);
+                                    int R, int r_pad, const float* mu, double c, const unsigned* amax, int fold,
+                                    void* src_hi, void* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv,
+                                    int rv, const unsigned* wstat, cudaStream_t st);
 cudaError_t launch_prep_f16_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
-                                    double c, const unsigned* amax, void* tgt_hi, void* tgt_lo, float* nb,
+                                    double c, const unsigned* amax, int fold, void* tgt_hi, void* tgt_lo, float* nb,
                                     float* tsc, cudaStream_t st);
 // maps: A_hi, A_lo (targets), B_hi, B_lo (sources), W_hi, W_lo (weights^T)
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st);

@@ -191,3 +191,49 @@ def test_r1_row_factor_paths(oracle_mod, h):
     V, _ = gpu_eval(a, W, b, np.float32(h))
     Vr = oracle_mod.oracle_eval(a, W, b, float(np.float32(h)))
     assert e_norm(V, Vr, W) <= TOL_3XTF32
+
+
+def test_r1_folded_layout_matches_unfolded(oracle_mod, monkeypatch):
+    """FP16, R = 1, W >= 0: the norms and log-weights ride in the contraction
+    (six hi-plane K columns, DESIGN.md Q26) and the epilogue is exp2 + sum;
+    KS_TC_FOLD=0 keeps them in FP32 in the epilogue.  Both meet the bar and
+    agree with each other (cfg3 distribution, K = 32: the norm columns take a
+    K step of their own)."""
+    a, W, b, h = workloads.make(3, M=4100, N=900, wkind="pos")
+    V1, _ = gpu_eval(a, W, b, h)
+    monkeypatch.setenv("KS_TC_FOLD", "0")
+    V0, _ = gpu_eval(a, W, b, h)
+    Vr = oracle_mod.oracle_eval(a, W, b, float(h))
+    assert e_norm(V1, Vr, W) <= TOL_3XTF32 and e_norm(V0, Vr, W) <= TOL_3XTF32
+    assert np.max(np.abs(V1 - V0)) / np.abs(W).sum() <= 2 * TOL_3XTF32
+
+
+@pytest.mark.parametrize("K", [1, 8, 10, 11, 16, 26, 27, 33])
+def test_r1_folded_norm_columns_placement(oracle_mod, K):
+    """The six norm columns share the last dimension K step when K % 16 <= 10,
+    else take (part of) a step of their own; every placement meets the bar."""
+    a, W, b, h = workloads.custom(1500, 700, K, 1, 0.25 * np.sqrt(K) + 0.1, dist="gm", sigma=0.05,
+                                  wkind="pos", seed=90 + K)
+    check(oracle_mod, a, W, b, h)
+
+
+def test_r1_fold_inactive_for_wide_spread(oracle_mod):
+    """c K amax^2 > 2^12 (h = 0.01 on the unit cube, K = 4): the folded layout
+    is switched off on the device (the FP16 norm pieces would not hold the
+    norms) and the epilogue adds them in FP32; same bar."""
+    a, W, b, h = workloads.custom(2000, 600, 4, 1, 0.01, wkind="pos", seed=5, same_points=True)
+    check(oracle_mod, a, W, b, h)
+
+
+def test_r1_fold_far_targets_are_zero(oracle_mod):
+    """Targets far outside the sources (c ||beta_hat||^2 > 2^14: every kernel
+    value < 2^-4096) get zero coordinates and a -2^15 norm in the folded
+    layout: V = 0 there up to the FMA-pipe exp2's floor of 2^-125 per term
+    (Q23), the other rows unaffected."""
+    a, W, b, h = workloads.make(3, M=2000, N=600, wkind="pos")
+    b = b.copy()
+    b[::7] += np.float32(40.0)
+    V, _ = gpu_eval(a, W, b, h)
+    Vr = oracle_mod.oracle_eval(a, W, b, float(h))
+    assert np.all(np.abs(V[::7]) <= 2.0**-120 * np.abs(W).sum())
+    assert e_norm(V, Vr, W) <= TOL_3XTF32
