@@ -448,6 +448,10 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.wv = ctx->wv.p;
   a.vcc = ctx->tc_vcc;
   {
+    const char* e = getenv("KS_TC_ARES");  // measurement knob: 0 = reload the target operand per unit
+    a.ares = (e && e[0] == '0') ? 0 : 1;
+  }
+  {
     const char* e = getenv("KS_TC_WSLOTS");  // measurement knob
     a.wslots = (e && e[0] >= '2' && e[0] <= '4') ? (e[0] - '0') : 0;
   }

@@ -45,14 +45,20 @@ constexpr uint32_t kColS0 = 0, kColS1 = 128, kColPlo = 256, kColV = 384;
 // Shared-memory layout (bytes from a 1 KB-aligned base).  TS = sources per
 // tile (128 with the tensor-core V path, 256 when the weighted sum runs on CUDA
 // cores, RV = padded weight columns of that mode, 0 = tensor-core V path).
-template <int kStages, int TS, int RV>
+template <int kStages, int TS, int RV, bool AR = false>
 struct TcSmemT {
   static constexpr bool VCC = RV > 0;
   static constexpr uint32_t kChunkB = TS * kTcKC * 4;                 // one hi or lo source chunk
-  static constexpr uint32_t kStageBytes = 2 * kChunkA + 2 * kChunkB;  // A_hi, A_lo, B_hi, B_lo
+  // AR (target operand resident): stages hold B_hi, B_lo only; A lives in 2 buffers x
+  // 2 chunks x (hi, lo) loaded once per target tile; else stages hold A_hi, A_lo, B_hi, B_lo
+  static constexpr uint32_t kStageBytes = AR ? 2 * kChunkB : 2 * kChunkA + 2 * kChunkB;
   static constexpr uint32_t kStage0 = 0;
+  static constexpr uint32_t kA0 = kStages * kStageBytes;
+  static constexpr uint32_t a_chunk(int buf, int kc, int plane) {
+    return kA0 + (uint32_t)((buf * 2 + kc) * 2 + plane) * kChunkA;
+  }
   static constexpr uint32_t wslot(int r_c) { return (uint32_t)r_c * 512u; }  // one of W^T hi/lo: 8 chunks x r_c x 64 B
-  static constexpr uint32_t kW0 = kStages * kStageBytes;
+  static constexpr uint32_t kW0 = kA0 + (AR ? 8 * kChunkA : 0u);
   // VCC: na[TS] | W[TS][RV];  else W^T hi | W^T lo | na[128].  Slots 1 KB aligned (SWIZZLE_64B atoms).
   static constexpr uint32_t w_slot_bytes(int r_c) {
     return VCC ? ((uint32_t)(4 * TS * (1 + RV)) + 1023u) & ~1023u : (2 * wslot(r_c) + 512 + 1023) & ~1023u;
@@ -60,7 +66,7 @@ struct TcSmemT {
   static constexpr uint32_t na_off(int r_c) { return VCC ? 0u : 2 * wslot(r_c); }
   static constexpr int kWSlots = VCC && RV < 8 ? 4 : 2;  // W/na ring depth (RV >= 8: 2 to fit 4 stages)
   static constexpr uint32_t bar_off(int r_c) { return kW0 + kWSlots * w_slot_bytes(r_c); }
-  static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 256 + 4 * kTcTileT * 8; }  // + VCC scratch
+  static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 512 + 4 * kTcTileT * 8; }  // + VCC scratch
 };
 
 // Phase profiling (build with -DKS_PROF=1, run with KS_CTA_TIMES=file): per
@@ -181,8 +187,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   constexpr int NPOLY = PP & 15;                    // folded epilogue (exp2 + sum)
   constexpr int NPOLY_U = NPOLY > 4 ? 4 : NPOLY;    // unfolded epilogues (more FMA-pipe work per pair)
   constexpr bool CLAMP_LW = (PP & 16) != 0;
+  constexpr bool AR = (PP & 32) != 0;  // target operand resident per target tile (VCC, <= 2 chunks)
   constexpr int TS = VCC ? 256 : kTcTileS;  // sources per tile
-  using TcSmem = TcSmemT<kStages, TS, RV>;
+  using TcSmem = TcSmemT<kStages, TS, RV, AR>;
   constexpr uint32_t kChunkB = TcSmem::kChunkB;
   constexpr uint32_t kStageBytes = TcSmem::kStageBytes;
   constexpr int EW = kTcEpiWarps;        // epilogue warps
@@ -203,7 +210,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   uint64_t* pready = sfull + 2;          // [2 S buffers][2 source halves]
   uint64_t* vdone = pready + 4;          // [2 source halves]
   uint64_t* sempty = vdone + 2;          // [2] (VCC: epilogue has read the S buffer)
-  uint32_t* tmem_base_smem = reinterpret_cast<uint32_t*>(sempty + 2);
+  uint64_t* afull = sempty + 2;          // [2] AR: target operand buffer loaded
+  uint64_t* aempty = afull + 2;          // [2] AR: MMAs done with the target operand buffer
+  uint32_t* tmem_base_smem = reinterpret_cast<uint32_t*>(aempty + 2);
   int* flag = reinterpret_cast<int*>(tmem_base_smem + 1);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -241,6 +250,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       mbar_init(&sempty[i], EW / 2);
       mbar_init(&sfull[i], 1);
       mbar_init(&vdone[i], 1);
+      mbar_init(&afull[i], 1);
+      mbar_init(&aempty[i], 1);
     }
     for (int i = 0; i < 4; ++i) mbar_init(&pready[i], EW);  // one arrival per epilogue warp
     fence_mbar_init();
@@ -261,9 +272,28 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     }
     const int kcw = args.f16 ? 2 * kTcKC : kTcKC;  // elements per 64-byte chunk
     int it = 0;
+    int seg = -1;
+    int64_t cur_tt = -1;
     UnitIt cu = unit_begin(sc);
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
       const int tt = (int)cu.tt, st = cu.st;
+      if (AR && cu.tt != cur_tt) {  // new target tile: its operand into buffer seg & 1, once
+        ++seg;
+        cur_tt = cu.tt;
+        const int ab = seg & 1;
+        mbar_wait(&aempty[ab], (uint32_t)(((seg >> 1) & 1) ^ 1));
+        if (leader) {
+          uint32_t bytes = 0;
+          for (int kc = 0; kc < n_kc; ++kc) bytes += (kc * kcw < args.kdims ? 2u : 1u) * kChunkA;
+          mbar_arrive_expect_tx(&afull[ab], bytes);
+          for (int kc = 0; kc < n_kc; ++kc) {
+            tma_load_2d(smem + TcSmem::a_chunk(ab, kc, 0), &mA_hi, kc * kcw, tt * kTcTileT, &afull[ab]);
+            if (kc * kcw < args.kdims)
+              tma_load_2d(smem + TcSmem::a_chunk(ab, kc, 1), &mA_lo, kc * kcw, tt * kTcTileT, &afull[ab]);
+          }
+        }
+        __syncwarp();
+      }
       for (int kc = 0; kc < n_kc; ++kc, ++it) {
         const int s = it % kStages;
         const uint32_t use = (uint32_t)(it / kStages);
@@ -276,11 +306,17 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         } else if (leader) {
           const int k0 = kc * kcw;  // element coordinate of the 64-byte chunk
           const bool lo = k0 < args.kdims;  // chunks holding only folded norm columns: hi planes only
-          mbar_arrive_expect_tx(&full[s], lo ? kStageBytes : kChunkA + kChunkB);
-          tma_load_2d(sp, &mA_hi, k0, tt * kTcTileT, &full[s]);
-          if (lo) tma_load_2d(sp + kChunkA, &mA_lo, k0, tt * kTcTileT, &full[s]);
-          tma_load_2d(sp + 2 * kChunkA, &mB_hi, k0, st * TS, &full[s]);
-          if (lo) tma_load_2d(sp + 2 * kChunkA + kChunkB, &mB_lo, k0, st * TS, &full[s]);
+          if constexpr (AR) {
+            mbar_arrive_expect_tx(&full[s], lo ? 2 * kChunkB : kChunkB);
+            tma_load_2d(sp, &mB_hi, k0, st * TS, &full[s]);
+            if (lo) tma_load_2d(sp + kChunkB, &mB_lo, k0, st * TS, &full[s]);
+          } else {
+            mbar_arrive_expect_tx(&full[s], lo ? kStageBytes : kChunkA + kChunkB);
+            tma_load_2d(sp, &mA_hi, k0, tt * kTcTileT, &full[s]);
+            if (lo) tma_load_2d(sp + kChunkA, &mA_lo, k0, tt * kTcTileT, &full[s]);
+            tma_load_2d(sp + 2 * kChunkA, &mB_hi, k0, st * TS, &full[s]);
+            if (lo) tma_load_2d(sp + 2 * kChunkA + kChunkB, &mB_lo, k0, st * TS, &full[s]);
+          }
         }
         __syncwarp();
       }
@@ -361,9 +397,19 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     };
     UnitIt cu = unit_begin(sc);
     int prev_st = 0;
+    int seg = -1;
+    int64_t cur_tt = -1;
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
       const int bq = q & 1;
       const uint32_t dS = tbase + (bq ? (uint32_t)TS : 0u);
+      if (AR && cu.tt != cur_tt) {  // new target tile: release the previous operand buffer, wait for this one
+        if (seg >= 0 && leader) tc_commit(&aempty[seg & 1]);
+        __syncwarp();
+        ++seg;
+        cur_tt = cu.tt;
+        mbar_wait(&afull[seg & 1], (uint32_t)((seg >> 1) & 1));
+        tc_fence_after();
+      }
       if constexpr (VCC) {
         if (q >= 2) {  // the epilogue has read S(q-2) out of this buffer
           PROF_BEGIN(w1);
@@ -380,13 +426,17 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         PROF_END(0, w0);
         tc_fence_after();
         uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
-        const uint64_t d0 = sdesc_k_sw64(sp);
+        // operand descriptors: A (targets) from the stage or the resident buffer, B from the stage
+        const uint64_t dAh = AR ? sdesc_k_sw64(smem + TcSmem::a_chunk(seg & 1, kc, 0)) : sdesc_k_sw64(sp);
+        const uint64_t dAl = AR ? sdesc_k_sw64(smem + TcSmem::a_chunk(seg & 1, kc, 1)) : sdesc_k_sw64(sp + kChunkA);
+        const uint64_t dBh = sdesc_k_sw64(sp + (AR ? 0u : 2 * kChunkA));
+        const uint64_t dBl = sdesc_k_sw64(sp + (AR ? 0u : 2 * kChunkA) + kChunkB);
 #pragma unroll
         for (int ks = 0; ks < kTcKC / 8; ++ks) {
-          const uint64_t aH = d0 + (uint64_t)((ks * 32) >> 4);
-          const uint64_t aL = d0 + (uint64_t)((kChunkA + ks * 32) >> 4);
-          const uint64_t bH = d0 + (uint64_t)((2 * kChunkA + ks * 32) >> 4);
-          const uint64_t bL = d0 + (uint64_t)((2 * kChunkA + kChunkB + ks * 32) >> 4);
+          const uint64_t aH = dAh + (uint64_t)((ks * 32) >> 4);
+          const uint64_t aL = dAl + (uint64_t)((ks * 32) >> 4);
+          const uint64_t bH = dBh + (uint64_t)((ks * 32) >> 4);
+          const uint64_t bL = dBl + (uint64_t)((ks * 32) >> 4);
           const uint32_t acc0 = (kc > 0 || ks > 0) ? 1u : 0u;
           const int col0 = kc * kcw + ks * (kcw / 2);  // first element column of this K step
           if (col0 >= args.kcols) continue;            // all-zero padding step
@@ -449,7 +499,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     constexpr int CW = TS / 2;            // columns per warp and tile (128)
     static_assert(EW == 16, "two groups x 2 column halves x 4 TMEM lane groups");
     constexpr int BC = (RV >= 8) ? 16 : 32;  // TMEM columns per load batch (register budget)
-    double* red = reinterpret_cast<double*>(smem + TcSmem::bar_off(RC) + 256);  // [SUB][128]
+    double* red = reinterpret_cast<double*>(smem + TcSmem::bar_off(RC) + 512);  // [SUB][128]
     constexpr int RVA = RV > 0 ? RV : 1;  // (this branch only runs with RV > 0)
     // per-row sums: FP32 over <= 8 tiles (vblk), folded into an unevaluated
     // FP32 pair (vhi + vlo, TwoSum: exact fold, no FP64 pipe in the tile loop)
@@ -1155,8 +1205,9 @@ int fused_tc_rv(int R) { return R <= 1 ? 1 : R <= 2 ? 2 : R <= 4 ? 4 : R <= 8 ? 
 template <int RC, int NS, int RV, int PP = 0>
 static cudaError_t launch_rcsv(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
   static bool attr_done = false;
-  const size_t smem = TcSmemT<NS, RV ? 256 : kTcTileS, RV>::total(RC);
-  static_assert(TcSmemT<NS, RV ? 256 : kTcTileS, RV>::total(RC) <= 232448, "exceeds 227 KB of shared memory");
+  using Sm = TcSmemT<NS, RV ? 256 : kTcTileS, RV, (PP & 32) != 0>;
+  const size_t smem = Sm::total(RC);
+  static_assert(Sm::total(RC) <= 232448, "exceeds 227 KB of shared memory");
   if (!attr_done) {
     cudaError_t e = cudaFuncSetAttribute(ks_fused_tc_kernel<RC, NS, RV, PP>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -1183,6 +1234,13 @@ cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream
       const char* ec = getenv("KS_TC_CLAMP");
       const bool clamp = ec && ec[0] == '1';
       if (clamp) return pp == 0 ? launch_rcsv<16, 4, 1, 16>(maps, a, st) : launch_rcsv<16, 4, 1, 20>(maps, a, st);
+      if (a.ares && a.k_pad <= 2 * kTcKC) {  // target operand resident (<= 2 chunks)
+        switch (pp) {
+          case 0: return launch_rcsv<16, 4, 1, 32>(maps, a, st);
+          case 4: return launch_rcsv<16, 4, 1, 36>(maps, a, st);
+          default: return launch_rcsv<16, 4, 1, 38>(maps, a, st);
+        }
+      }
       switch (pp) {
         case 0: return launch_rcsv<16, 4, 1, 0>(maps, a, st);
         case 4: return launch_rcsv<16, 4, 1, 4>(maps, a, st);

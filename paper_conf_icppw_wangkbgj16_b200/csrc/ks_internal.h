@@ -85,6 +85,7 @@ struct TcArgs {
   int vcc;              // RV > 0: weighted sum on CUDA cores over RV padded columns (no W^T tiles, no V MMA)
   const float* wv;      // [m_pad][RV] weights, zero padded (vcc)
   int wslots;           // VCC W/na ring depth (2..4; 0 = default)
+  int ares;             // R = 1, <= 2 operand chunks: target operand resident per target tile (no reload per unit)
   int dbg_skip_v;       // measurement only (KS_TC_DEBUG_SKIP_V=1): do not issue the V MMAs (wrong results)
   const float* na;      // [m_pad]  -c ||alpha_hat||^2
   const float* nb;      // [n_pad]  -c ||beta_hat||^2

@@ -1,0 +1,89 @@
+// mma_microbench.cu -- tcgen05.mma kind::f16 (M = 128, FP32 accumulate in
+// TMEM) issue rate from shared-memory operands on B200, one CTA per SM, one
+// issuing thread: SWIZZLE_64B (64-byte K-major rows, the fused kernel's
+// layout) vs SWIZZLE_128B rows, N = 256 and 128.  Prints SM cycles per MMA
+// instruction at 1965 MHz; the dense FP16 rate would be M N K 2 / 8192.
+#include <cstdio>
+#include <cuda_runtime.h>
+#include "../paper_conf_icppw_wangkbgj16_b200/csrc/ks_ptx.cuh"
+using namespace ks;
+#define NMMA 8192
+
+__device__ __forceinline__ uint64_t sdesc_sw(const void* p, int sw) {
+  const uint64_t a = (uint64_t)((smem_u32(p) >> 4) & 0x3FFF);
+  const uint64_t sbo = (uint64_t)((8 * sw) >> 4);  // 8-row atoms
+  const uint64_t layout = sw == 128 ? 2ull : sw == 64 ? 4ull : 6ull;
+  return a | (1ull << 16) | (sbo << 32) | (1ull << 46) | (layout << 61);
+}
+
+template <int SW, int N>
+__global__ void __launch_bounds__(128, 1) k(float* out) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ uint32_t tb;
+  __shared__ __align__(8) uint64_t bar;
+  const int tid = threadIdx.x, warp = tid >> 5;
+  // A: 128 rows x SW bytes, B: 256 rows x SW bytes (one 'chunk' each), zero
+  for (int i = tid; i < (128 + 256) * SW / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(smem)[i] = 0u;
+  if (tid == 0) { mbar_init(&bar, 1); fence_mbar_init(); }
+  if (warp == 0) tmem_alloc(&tb, 512);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = tb;
+  if (warp == 0) {
+    const bool leader = elect_one();
+    const uint64_t dA = sdesc_sw(smem, SW), dB = sdesc_sw(smem + 128 * SW, SW);
+    const uint32_t id = idesc_f16(128, N);
+    const int steps = SW / 32;  // K = 16 halves = 32 bytes per MMA
+    for (int i = 0; i < NMMA; ++i) {
+      const int ks = i % steps;
+      const uint32_t d = tbase + (uint32_t)(((i / steps) & 1) * 256);
+      if (leader) mma_f16_ss(d, dA + (uint64_t)((ks * 32) >> 4), dB + (uint64_t)((ks * 32) >> 4), id, ks ? 1u : 0u);
+      __syncwarp();
+    }
+    if (leader) tc_commit(&bar);
+    __syncwarp();
+    mbar_wait(&bar, 0);
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) tmem_dealloc(tbase, 512);
+  if (tid == 0 && out[0] == 1234.5f) out[1] = 1.f;
+}
+
+template <int SW, int N>
+void run(float* out, int G) {
+  const int smem = (128 + 256) * SW + 1024;
+  cudaFuncSetAttribute(k<SW, N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  float best = 1e9;
+  for (int r = 0; r < 5; ++r) {
+    cudaEventRecord(e0);
+    k<SW, N><<<G, 128, smem>>>(out);
+    cudaEventRecord(e1);
+    cudaEventSynchronize(e1);
+    float ms;
+    cudaEventElapsedTime(&ms, e0, e1);
+    if (ms < best) best = ms;
+  }
+  const double cyc = best * 1e-3 * 1.965e9 / NMMA;
+  printf("SWIZZLE_%dB N=%d: %.3f ms  %.1f cycles/MMA (dense rate %d)  %.0f TFLOP/s chip\n", SW, N, best, cyc,
+         128 * N * 16 * 2 / 8192, 128.0 * N * 16 * 2 * NMMA * G / (best * 1e-3) / 1e12);
+}
+int main() {
+  cudaDeviceProp p;
+  cudaGetDeviceProperties(&p, 0);
+  float* out;
+  cudaMalloc(&out, 8);
+  cudaMemset(out, 0, 8);
+  const int G = p.multiProcessorCount;
+  run<64, 256>(out, G);
+  run<128, 256>(out, G);
+  run<32, 256>(out, G);
+  run<64, 128>(out, G);
+  run<128, 128>(out, G);
+  printf("%s\n", cudaGetErrorString(cudaDeviceSynchronize()));
+}
