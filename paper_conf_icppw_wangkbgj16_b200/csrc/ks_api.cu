@@ -457,8 +457,10 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   }
   {
     const char* e = getenv("KS_TC_DEBUG_SKIP_V");
-    // 1 no epilogue math, 4 W/na loaded once, 5 no S MMAs, 6 one product, 7 no MMAs and no operand loads
-    a.dbg_skip_v = (e && e[0] >= '1' && e[0] <= '7') ? e[0] - '0' : 0;
+    // 1 no epilogue math, 4 W/na loaded once, 5 no S MMAs, 6 one product, 7 no MMAs and no operand
+    // loads, 8 = 1 + 5, 9 = 1 + no operand loads, 10 = 1 + 7 (measurement only: wrong results)
+    a.dbg_skip_v = e ? atoi(e) : 0;
+    if (a.dbg_skip_v < 0 || a.dbg_skip_v > 10) a.dbg_skip_v = 0;
   }
   a.na = ctx->na.p;
   a.nb = ctx->nb.p;

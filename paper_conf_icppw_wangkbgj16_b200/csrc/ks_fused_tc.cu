@@ -226,6 +226,12 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   const bool logw_k = RV == 1 && args.wstat != nullptr && args.wstat[1] == 0u && args.wstat[0] != 0u;
   const bool fold_k = RV == 1 && args.fold && f16_fold_ok(args.amax, args.c, args.K);
   const bool ring = !(logw_k && fold_k && !CLAMP_LW);
+  // measurement knobs (KS_TC_DEBUG_SKIP_V, wrong results): 1 no epilogue math, 4 W/na loaded once,
+  // 5 no S MMAs, 6 one product, 7 no MMAs and no operand loads, 8 = 1 + 5, 9 = 1 + no operand
+  // loads, 10 = 1 + 7
+  const int dv = args.dbg_skip_v;
+  const bool dbg_noepi = dv == 1 || dv >= 8;
+  const bool dbg_noload = dv == 7 || dv == 9 || dv == 10;
   const int64_t b = blockIdx.x;
   Sched sc;
   sc.init(args.sk.n_t, n_s, args.sk.grid, b);
@@ -282,7 +288,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         cur_tt = cu.tt;
         const int ab = seg & 1;
         mbar_wait(&aempty[ab], (uint32_t)(((seg >> 1) & 1) ^ 1));
-        if (leader) {
+        if (leader && dbg_noload) {
+          mbar_arrive(&afull[ab]);
+        } else if (leader) {
           uint32_t bytes = 0;
           for (int kc = 0; kc < n_kc; ++kc) bytes += (kc * kcw < args.kdims ? 2u : 1u) * kChunkA;
           mbar_arrive_expect_tx(&afull[ab], bytes);
@@ -301,7 +309,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         mbar_wait(&empty[s], (use & 1) ^ 1);
         PROF_END(0, w0);
         uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
-        if (leader && args.dbg_skip_v == 7) {  // measurement: no operand loads (wrong results)
+        if (leader && dbg_noload) {  // measurement: no operand loads (wrong results)
           mbar_arrive(&full[s]);
         } else if (leader) {
           const int k0 = kc * kcw;  // element coordinate of the 64-byte chunk
@@ -357,7 +365,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     const uint32_t idV = idesc_tf32(128, RC);
     const int nprod = args.three ? 3 : 1;
     const int kcw = args.f16 ? 2 * kTcKC : kTcKC;  // elements per 64-byte chunk
-    const bool dbg_no_mma = args.dbg_skip_v == 5 || args.dbg_skip_v == 7;  // measurement: no S MMAs (wrong results)
+    const bool dbg_no_mma = dv == 5 || dv == 7 || dv == 8 || dv == 10;  // measurement: no S MMAs (wrong results)
     const bool dbg_one = args.dbg_skip_v == 6;      // measurement: one product only (wrong results)
     const bool skip_v = args.dbg_skip_v == 1;
     int it = 0;
@@ -542,8 +550,48 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q % WS) * TcSmem::w_slot_bytes(RC));
       const float* wvs = nas + TS;        // [TS][RV]
       const uint32_t colS = bq ? (uint32_t)TS : 0u;
+      bool done = false;
+      if constexpr (RV == 1 && BC == 32 && CW == 128) {
+        if (!ring && !dbg_noepi) {
+          // folded layout, W >= 0: S = t already (norms and log2 W_i / Wmax in the
+          // contraction, reading Q26): V_j = Wmax sum_i 2^S -- exp2 + FADD2 per pair.
+          // The four 32-column batches are loaded two ahead, so the S buffer is released
+          // after half of the tile's exponentials instead of three quarters.
+          auto fold_batch = [&](const uint32_t(&sv)[32]) {
 #pragma unroll
-      for (int hh = 0; hh < CW / BC; ++hh) {
+            for (int i = 0; i < 32; i += 2) {
+              const int k = i >> 1;
+              f2_t pk;
+              if (((k * NPOLY) & 15) < NPOLY) {
+                pk = exp2_poly2(f2_pack(fmaxf(__uint_as_float(sv[i]), -125.f), fmaxf(__uint_as_float(sv[i + 1]), -125.f)));
+              } else {
+                pk = f2_pack(ex2_approx(__uint_as_float(sv[i])), ex2_approx(__uint_as_float(sv[i + 1])));
+              }
+              vacc2[k & 1] = fadd2(vacc2[k & 1], pk);
+            }
+          };
+          const uint32_t ta = tbase + lane_off + colS + CW * hc;
+          uint32_t sa[32], sb[32];
+          tmem_ldn<32>(ta, sa);
+          tmem_wait_ld();
+          tmem_ldn<32>(ta + 32, sb);
+          fold_batch(sa);
+          tmem_wait_ld();
+          tmem_ldn<32>(ta + 64, sa);
+          fold_batch(sb);
+          tmem_wait_ld();
+          tmem_ldn<32>(ta + 96, sb);
+          tmem_wait_ld();
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&sempty[bq]);  // S buffer may be overwritten now
+          fold_batch(sa);
+          fold_batch(sb);
+          done = true;
+        }
+      }
+#pragma unroll
+      for (int hh = 0; hh < (done ? 0 : CW / BC); ++hh) {
         const int c0 = CW * hc + BC * hh;
         uint32_t sv[BC];
         tmem_ldn<BC>(tbase + lane_off + colS + c0, sv);
@@ -553,7 +601,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           __syncwarp();
           if (lane == 0) mbar_arrive(&sempty[bq]);  // S buffer may be overwritten now
         }
-        if (args.dbg_skip_v == 1) {  // measurement knob: MMA/TMA-only timing
+        if (dbg_noepi) {  // measurement knob: MMA/TMA-only timing
           if (__uint_as_float(sv[0]) == 12345.f) vblk[0] += 1.f;
           continue;
         }
