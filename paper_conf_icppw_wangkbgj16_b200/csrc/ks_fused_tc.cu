@@ -403,6 +403,69 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       }
       __syncwarp();
     };
+    if constexpr (VCC && AR) {
+      // Lean issue loop of the resident-target kind::f16 kernel (R = 1): the per-tile MMA
+      // sequence is fixed, so it is planned once (products per 16-column K step: 3 split
+      // products, 1 = hi.hi for folded norm columns only, 0 = padding) and every branch
+      // below is warp-uniform; the elected lane only predicates the tcgen05 instructions.
+      const uint32_t lead = leader ? 1u : 0u;
+      uint32_t plan = 0;
+      for (int st4 = 0; st4 < 2 * n_kc; ++st4) {
+        const int col0 = st4 * (kcw / 2);
+        const uint32_t np = col0 >= args.kcols ? 0u : (col0 >= args.kdims || !args.three) ? 1u : 3u;
+        plan |= np << (2 * st4);
+      }
+      if (dbg_no_mma) plan = 0;
+      const uint64_t dA0 = sdesc_k_sw64(smem + TcSmem::a_chunk(0, 0, 0));
+      const uint64_t dB0 = sdesc_k_sw64(smem + TcSmem::kStage0);
+      constexpr uint64_t kA16 = kChunkA >> 4, kB16 = kChunkB >> 4, kS16 = kStageBytes >> 4;
+      int seg = -1;
+      int64_t cur_tt = -1;
+      UnitIt cu = unit_begin(sc);
+      for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
+        const int bq = q & 1;
+        const uint32_t dS = tbase + (bq ? (uint32_t)TS : 0u);
+        if (cu.tt != cur_tt) {  // new target tile: release the previous operand buffer, wait for this one
+          if (seg >= 0) tc_commit_if(&aempty[seg & 1], lead);
+          ++seg;
+          cur_tt = cu.tt;
+          mbar_wait(&afull[seg & 1], (uint32_t)((seg >> 1) & 1));
+          tc_fence_after();
+        }
+        if (q >= 2) {  // the epilogue has read S(q-2) out of this buffer
+          PROF_BEGIN(w1);
+          mbar_wait(&sempty[bq], (uint32_t)(((q - 2) >> 1) & 1));
+          PROF_END(1, w1);
+          tc_fence_after();
+        }
+        for (int kc = 0; kc < n_kc; ++kc, ++it) {
+          const int s = it % kStages;
+          PROF_BEGIN(w0);
+          mbar_wait(&full[s], (uint32_t)(it / kStages) & 1);
+          PROF_END(0, w0);
+          PROF_BEGIN(w2);
+          tc_fence_after();
+          const uint64_t aH0 = dA0 + (uint64_t)((seg & 1) * 2 + kc) * 2 * kA16, aL0 = aH0 + kA16;
+          const uint64_t bH0 = dB0 + (uint64_t)s * kS16, bL0 = bH0 + kB16;
+#pragma unroll
+          for (int ks = 0; ks < 2; ++ks) {
+            const uint32_t np = (plan >> (2 * (2 * kc + ks))) & 3u;
+            const uint64_t o = (uint64_t)(ks * 2);  // 32 bytes along K
+            const uint32_t acc0 = (kc > 0 || ks > 0) ? 1u : 0u;
+            if (np == 3u) {  // lo.hi, hi.lo, hi.hi (small terms first)
+              mma_f16_ss_if(dS, aL0 + o, bH0 + o, idS, acc0, lead);
+              mma_f16_ss_if(dS, aH0 + o, bL0 + o, idS, 1u, lead);
+              mma_f16_ss_if(dS, aH0 + o, bH0 + o, idS, 1u, lead);
+            } else if (np == 1u) {
+              mma_f16_ss_if(dS, aH0 + o, bH0 + o, idS, acc0, lead);
+            }
+          }
+          tc_commit_if(&empty[s], lead);
+          PROF_END(2, w2);
+        }
+        tc_commit_if(&sfull[bq], lead);
+      }
+    } else {
     UnitIt cu = unit_begin(sc);
     int prev_st = 0;
     int seg = -1;
@@ -432,6 +495,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         PROF_BEGIN(w0);
         mbar_wait(&full[s], use & 1);
         PROF_END(0, w0);
+        PROF_BEGIN(w2);
         tc_fence_after();
         uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
         // operand descriptors: A (targets) from the stage or the resident buffer, B from the stage
@@ -475,7 +539,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         __syncwarp();
         if (leader) tc_commit(&empty[s]);
         __syncwarp();
+        PROF_END(2, w2);
       }
+      PROF_BEGIN(w3);
       if (leader) tc_commit(&sfull[bq]);
       __syncwarp();
       if constexpr (!VCC) {
@@ -485,6 +551,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         }
       }
       prev_st = cu.st;
+      PROF_END(3, w3);
     }
     if constexpr (!VCC) {
       if (count > 0) {
@@ -492,6 +559,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         v_mma(count - 1, prev_st, 1);
       }
     }
+    }  // general issue loop
   } else if (VCC && warp >= 4) {
     // ================= epilogue, R <= 16: V on CUDA cores
     // Two groups of EW/2 warps take alternate tiles (group = parity of the
@@ -1282,7 +1350,7 @@ cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream
       const char* ec = getenv("KS_TC_CLAMP");
       const bool clamp = ec && ec[0] == '1';
       if (clamp) return pp == 0 ? launch_rcsv<16, 4, 1, 16>(maps, a, st) : launch_rcsv<16, 4, 1, 20>(maps, a, st);
-      if (a.ares && a.k_pad <= 2 * kTcKC) {  // target operand resident (<= 2 chunks)
+      if (a.ares && a.f16 && a.k_pad <= 2 * kTcKC) {  // split-FP16, target operand resident (<= 2 chunks)
         switch (pp) {
           case 0: return launch_rcsv<16, 4, 1, 32>(maps, a, st);
           case 4: return launch_rcsv<16, 4, 1, 36>(maps, a, st);

@@ -16,15 +16,21 @@ __device__ __forceinline__ uint64_t sdesc_sw(const void* p, int sw) {
   return a | (1ull << 16) | (sbo << 32) | (1ull << 46) | (layout << 61);
 }
 
-template <int SW, int N>
+// MODE 0: MMAs only, 1: commit after every MMA, 2: commits only, 3: + tcgen05.fence::after_thread_sync
+// per MMA, 4: + try_wait on a completed mbarrier per MMA, 5: commit + fence + try_wait per MMA
+template <int SW, int N, int MODE = 0>
 __global__ void __launch_bounds__(128, 1) k(float* out) {
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ uint32_t tb;
   __shared__ __align__(8) uint64_t bar;
+  __shared__ __align__(8) uint64_t cbar;
+  __shared__ __align__(8) uint64_t done;
   const int tid = threadIdx.x, warp = tid >> 5;
   // A: 128 rows x SW bytes, B: 256 rows x SW bytes (one 'chunk' each), zero
   for (int i = tid; i < (128 + 256) * SW / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(smem)[i] = 0u;
-  if (tid == 0) { mbar_init(&bar, 1); fence_mbar_init(); }
+  if (tid == 0) { mbar_init(&bar, 1); mbar_init(&cbar, 1); mbar_init(&done, 1); fence_mbar_init(); }
+  __syncthreads();
+  if (tid == 0) mbar_arrive(&done);
   if (warp == 0) tmem_alloc(&tb, 512);
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   tc_fence_before();
@@ -39,8 +45,14 @@ __global__ void __launch_bounds__(128, 1) k(float* out) {
     for (int i = 0; i < NMMA; ++i) {
       const int ks = i % steps;
       const uint32_t d = tbase + (uint32_t)(((i / steps) & 1) * 256);
-      if (leader) mma_f16_ss(d, dA + (uint64_t)((ks * 32) >> 4), dB + (uint64_t)((ks * 32) >> 4), id, ks ? 1u : 0u);
+      if (leader && MODE != 2) mma_f16_ss(d, dA + (uint64_t)((ks * 32) >> 4), dB + (uint64_t)((ks * 32) >> 4), id, ks ? 1u : 0u);
       __syncwarp();
+      if (MODE == 1 || MODE == 2 || MODE == 5) {
+        if (leader) tc_commit(&cbar);
+        __syncwarp();
+      }
+      if (MODE == 3 || MODE == 5) tc_fence_after();
+      if (MODE == 4 || MODE == 5) mbar_wait(&done, 0);  // already complete
     }
     if (leader) tc_commit(&bar);
     __syncwarp();
@@ -52,17 +64,17 @@ __global__ void __launch_bounds__(128, 1) k(float* out) {
   if (tid == 0 && out[0] == 1234.5f) out[1] = 1.f;
 }
 
-template <int SW, int N>
+template <int SW, int N, int MODE = 0>
 void run(float* out, int G) {
   const int smem = (128 + 256) * SW + 1024;
-  cudaFuncSetAttribute(k<SW, N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaFuncSetAttribute(k<SW, N, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   cudaEvent_t e0, e1;
   cudaEventCreate(&e0);
   cudaEventCreate(&e1);
   float best = 1e9;
   for (int r = 0; r < 5; ++r) {
     cudaEventRecord(e0);
-    k<SW, N><<<G, 128, smem>>>(out);
+    k<SW, N, MODE><<<G, 128, smem>>>(out);
     cudaEventRecord(e1);
     cudaEventSynchronize(e1);
     float ms;
@@ -70,7 +82,7 @@ void run(float* out, int G) {
     if (ms < best) best = ms;
   }
   const double cyc = best * 1e-3 * 1.965e9 / NMMA;
-  printf("SWIZZLE_%dB N=%d: %.3f ms  %.1f cycles/MMA (dense rate %d)  %.0f TFLOP/s chip\n", SW, N, best, cyc,
+  printf("MODE %d SWIZZLE_%dB N=%d: %.3f ms  %.1f cycles/MMA (dense rate %d)  %.0f TFLOP/s chip\n", MODE, SW, N, best, cyc,
          128 * N * 16 * 2 / 8192, 128.0 * N * 16 * 2 * NMMA * G / (best * 1e-3) / 1e12);
 }
 int main() {
@@ -85,5 +97,12 @@ int main() {
   run<32, 256>(out, G);
   run<64, 128>(out, G);
   run<128, 128>(out, G);
+  run<64, 256, 1>(out, G);
+  run<64, 256, 2>(out, G);
+  run<64, 128, 1>(out, G);
+  run<64, 256, 3>(out, G);
+  run<64, 256, 4>(out, G);
+  run<64, 256, 5>(out, G);
+  run<64, 128, 5>(out, G);
   printf("%s\n", cudaGetErrorString(cudaDeviceSynchronize()));
 }

@@ -13,7 +13,7 @@ def show(name, w, labels):
     parts = ", ".join(f"{lab} {pf[:, w, k].mean() / t:.3f}" for k, lab in enumerate(labels))
     print(f"{name:22s} run {t / 1e6:8.3f} Mcyc  {parts}")
 show("warp0 operand TMA", 0, ["wait empty"])
-show("warp1 MMA", 1, ["wait full", "wait sempty"])
+show("warp1 MMA", 1, ["wait full", "wait sempty", "issue", "commit+rest"])
 show("warp3 norms/W loads", 3, ["wait wempty"])
 for w in (4, 5, 6, 7, 8, 12, 16, 19):
     show(f"epilogue warp {w}", w, ["wait wfull", "wait sfull", "compute", "tail"])
