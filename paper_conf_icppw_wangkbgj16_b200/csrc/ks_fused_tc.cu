@@ -49,14 +49,11 @@ template <int kStages, int TS, int RV, bool AR = false>
 struct TcSmemT {
   static constexpr bool VCC = RV > 0;
   static constexpr uint32_t kChunkB = TS * kTcKC * 4;                 // one hi or lo source chunk
-  // AR (target operand resident): stages hold B_hi, B_lo only; A lives in 2 buffers x
-  // 2 chunks x (hi, lo) loaded once per target tile; else stages hold A_hi, A_lo, B_hi, B_lo
+  // AR (target operand resident): the operand region (up to kW0) is laid out at run time
+  // (ArGeo); else stages hold A_hi, A_lo, B_hi, B_lo per 64-byte chunk
   static constexpr uint32_t kStageBytes = AR ? 2 * kChunkB : 2 * kChunkA + 2 * kChunkB;
   static constexpr uint32_t kStage0 = 0;
   static constexpr uint32_t kA0 = kStages * kStageBytes;
-  static constexpr uint32_t a_chunk(int buf, int kc, int plane) {
-    return kA0 + (uint32_t)((buf * 2 + kc) * 2 + plane) * kChunkA;
-  }
   static constexpr uint32_t wslot(int r_c) { return (uint32_t)r_c * 512u; }  // one of W^T hi/lo: 8 chunks x r_c x 64 B
   static constexpr uint32_t kW0 = kA0 + (AR ? 8 * kChunkA : 0u);
   // VCC: na[TS] | W[TS][RV];  else W^T hi | W^T lo | na[128].  Slots 1 KB aligned (SWIZZLE_64B atoms).
@@ -67,6 +64,35 @@ struct TcSmemT {
   static constexpr int kWSlots = VCC && RV < 8 ? 4 : 2;  // W/na ring depth (RV >= 8: 2 to fit 4 stages)
   static constexpr uint32_t bar_off(int r_c) { return kW0 + kWSlots * w_slot_bytes(r_c); }
   static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 512 + 4 * kTcTileT * 8; }  // + VCC scratch
+};
+
+// Resident-target (AR) kernels stage whole tiles: P operand planes per tile (per 64-byte
+// chunk its hi plane, plus its lo plane when the chunk holds dimension columns), the
+// target operand in two buffers of P planes, then D tile stages of P source planes in
+// the rest of the operand region (D <= kStages).  One full/empty barrier pair per tile.
+struct ArGeo {
+  int P, D;
+  uint32_t lo_mask;       // bit kc: chunk kc has a lo plane
+  uint32_t plane_off[2];  // first plane of chunk kc within a tile (A buffer or stage)
+  uint32_t a_bytes_a, stage_b;  // bytes of one A buffer / one tile stage
+  __device__ void init(int n_kc, int kcw, int kdims, uint32_t chunkA, uint32_t chunkB, uint32_t region,
+                       int max_stages) {
+    P = 0;
+    lo_mask = 0;
+    plane_off[0] = plane_off[1] = 0;
+#pragma unroll
+    for (int kc = 0; kc < 2; ++kc) {
+      if (kc >= n_kc) break;
+      plane_off[kc] = (uint32_t)P;
+      const bool lo = kc * kcw < kdims;
+      lo_mask |= lo ? (1u << kc) : 0u;
+      P += lo ? 2 : 1;
+    }
+    a_bytes_a = (uint32_t)P * chunkA;
+    stage_b = (uint32_t)P * chunkB;
+    const int d = (int)((region - 2 * a_bytes_a) / stage_b);
+    D = d < max_stages ? d : max_stages;
+  }
 };
 
 // Phase profiling (build with -DKS_PROF=1, run with KS_CTA_TIMES=file): per
@@ -269,7 +295,67 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   tc_fence_after();
   const uint32_t tbase = *tmem_base_smem;
 
-  if (warp == 0) {
+  if (AR && warp == 0) {
+    // ================= TMA producer, resident-target kernel: the target tile's operand once per
+    // target tile (buffer seg & 1), the source tile's planes as one stage per unit
+    const bool leader = elect_one();
+    if (leader) {
+      tma_prefetch_desc(&mA_hi);
+      tma_prefetch_desc(&mB_hi);
+    }
+    const int kcw = 2 * kTcKC;  // FP16 elements per 64-byte chunk
+    ArGeo g;
+    g.init(n_kc, kcw, args.kdims, kChunkA, kChunkB, TcSmem::kW0 - TcSmem::kStage0, kStages);
+    int s = 0;
+    uint32_t ph = 0;
+    int seg = -1;
+    int64_t cur_tt = -1;
+    UnitIt cu = unit_begin(sc);
+    for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
+      const int tt = (int)cu.tt, st = cu.st;
+      if (cu.tt != cur_tt) {
+        ++seg;
+        cur_tt = cu.tt;
+        const int ab = seg & 1;
+        mbar_wait(&aempty[ab], (uint32_t)(((seg >> 1) & 1) ^ 1));
+        uint8_t* ap = smem + TcSmem::kStage0 + ab * g.a_bytes_a;
+        if (leader && dbg_noload) {
+          mbar_arrive(&afull[ab]);
+        } else if (leader) {
+          mbar_arrive_expect_tx(&afull[ab], g.a_bytes_a);
+#pragma unroll
+          for (int kc = 0; kc < 2; ++kc) {
+            if (kc >= n_kc) break;
+            tma_load_2d(ap + g.plane_off[kc] * kChunkA, &mA_hi, kc * kcw, tt * kTcTileT, &afull[ab]);
+            if ((g.lo_mask >> kc) & 1u)
+              tma_load_2d(ap + (g.plane_off[kc] + 1) * kChunkA, &mA_lo, kc * kcw, tt * kTcTileT, &afull[ab]);
+          }
+        }
+        __syncwarp();
+      }
+      PROF_BEGIN(w0);
+      mbar_wait(&empty[s], ph ^ 1u);
+      PROF_END(0, w0);
+      uint8_t* sp = smem + TcSmem::kStage0 + 2 * g.a_bytes_a + s * g.stage_b;
+      if (leader && dbg_noload) {
+        mbar_arrive(&full[s]);
+      } else if (leader) {
+        mbar_arrive_expect_tx(&full[s], g.stage_b);
+#pragma unroll
+        for (int kc = 0; kc < 2; ++kc) {
+          if (kc >= n_kc) break;
+          tma_load_2d(sp + g.plane_off[kc] * kChunkB, &mB_hi, kc * kcw, st * TS, &full[s]);
+          if ((g.lo_mask >> kc) & 1u)
+            tma_load_2d(sp + (g.plane_off[kc] + 1) * kChunkB, &mB_lo, kc * kcw, st * TS, &full[s]);
+        }
+      }
+      __syncwarp();
+      if (++s == g.D) {
+        s = 0;
+        ph ^= 1u;
+      }
+    }
+  } else if (warp == 0) {
     // ================= TMA producer of the operand stages (whole warp converged; one elected lane issues)
     const bool leader = elect_one();
     if (leader) {
@@ -278,30 +364,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     }
     const int kcw = args.f16 ? 2 * kTcKC : kTcKC;  // elements per 64-byte chunk
     int it = 0;
-    int seg = -1;
-    int64_t cur_tt = -1;
     UnitIt cu = unit_begin(sc);
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
       const int tt = (int)cu.tt, st = cu.st;
-      if (AR && cu.tt != cur_tt) {  // new target tile: its operand into buffer seg & 1, once
-        ++seg;
-        cur_tt = cu.tt;
-        const int ab = seg & 1;
-        mbar_wait(&aempty[ab], (uint32_t)(((seg >> 1) & 1) ^ 1));
-        if (leader && dbg_noload) {
-          mbar_arrive(&afull[ab]);
-        } else if (leader) {
-          uint32_t bytes = 0;
-          for (int kc = 0; kc < n_kc; ++kc) bytes += (kc * kcw < args.kdims ? 2u : 1u) * kChunkA;
-          mbar_arrive_expect_tx(&afull[ab], bytes);
-          for (int kc = 0; kc < n_kc; ++kc) {
-            tma_load_2d(smem + TcSmem::a_chunk(ab, kc, 0), &mA_hi, kc * kcw, tt * kTcTileT, &afull[ab]);
-            if (kc * kcw < args.kdims)
-              tma_load_2d(smem + TcSmem::a_chunk(ab, kc, 1), &mA_lo, kc * kcw, tt * kTcTileT, &afull[ab]);
-          }
-        }
-        __syncwarp();
-      }
       for (int kc = 0; kc < n_kc; ++kc, ++it) {
         const int s = it % kStages;
         const uint32_t use = (uint32_t)(it / kStages);
@@ -314,17 +379,11 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         } else if (leader) {
           const int k0 = kc * kcw;  // element coordinate of the 64-byte chunk
           const bool lo = k0 < args.kdims;  // chunks holding only folded norm columns: hi planes only
-          if constexpr (AR) {
-            mbar_arrive_expect_tx(&full[s], lo ? 2 * kChunkB : kChunkB);
-            tma_load_2d(sp, &mB_hi, k0, st * TS, &full[s]);
-            if (lo) tma_load_2d(sp + kChunkB, &mB_lo, k0, st * TS, &full[s]);
-          } else {
-            mbar_arrive_expect_tx(&full[s], lo ? kStageBytes : kChunkA + kChunkB);
-            tma_load_2d(sp, &mA_hi, k0, tt * kTcTileT, &full[s]);
-            if (lo) tma_load_2d(sp + kChunkA, &mA_lo, k0, tt * kTcTileT, &full[s]);
-            tma_load_2d(sp + 2 * kChunkA, &mB_hi, k0, st * TS, &full[s]);
-            if (lo) tma_load_2d(sp + 2 * kChunkA + kChunkB, &mB_lo, k0, st * TS, &full[s]);
-          }
+          mbar_arrive_expect_tx(&full[s], lo ? kStageBytes : kChunkA + kChunkB);
+          tma_load_2d(sp, &mA_hi, k0, tt * kTcTileT, &full[s]);
+          if (lo) tma_load_2d(sp + kChunkA, &mA_lo, k0, tt * kTcTileT, &full[s]);
+          tma_load_2d(sp + 2 * kChunkA, &mB_hi, k0, st * TS, &full[s]);
+          if (lo) tma_load_2d(sp + 2 * kChunkA + kChunkB, &mB_lo, k0, st * TS, &full[s]);
         }
         __syncwarp();
       }
@@ -416,9 +475,14 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         plan |= np << (2 * st4);
       }
       if (dbg_no_mma) plan = 0;
-      const uint64_t dA0 = sdesc_k_sw64(smem + TcSmem::a_chunk(0, 0, 0));
-      const uint64_t dB0 = sdesc_k_sw64(smem + TcSmem::kStage0);
-      constexpr uint64_t kA16 = kChunkA >> 4, kB16 = kChunkB >> 4, kS16 = kStageBytes >> 4;
+      ArGeo g;
+      g.init(n_kc, kcw, args.kdims, kChunkA, kChunkB, TcSmem::kW0 - TcSmem::kStage0, kStages);
+      const uint64_t dA0 = sdesc_k_sw64(smem + TcSmem::kStage0);
+      const uint64_t dB0 = sdesc_k_sw64(smem + TcSmem::kStage0 + 2 * g.a_bytes_a);
+      constexpr uint64_t kA16 = kChunkA >> 4, kB16 = kChunkB >> 4;
+      const uint64_t aBuf16 = g.a_bytes_a >> 4, stage16 = g.stage_b >> 4;
+      int s = 0;
+      uint32_t ph = 0;
       int seg = -1;
       int64_t cur_tt = -1;
       UnitIt cu = unit_begin(sc);
@@ -430,23 +494,23 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           ++seg;
           cur_tt = cu.tt;
           mbar_wait(&afull[seg & 1], (uint32_t)((seg >> 1) & 1));
-          tc_fence_after();
         }
         if (q >= 2) {  // the epilogue has read S(q-2) out of this buffer
           PROF_BEGIN(w1);
           mbar_wait(&sempty[bq], (uint32_t)(((q - 2) >> 1) & 1));
           PROF_END(1, w1);
-          tc_fence_after();
         }
-        for (int kc = 0; kc < n_kc; ++kc, ++it) {
-          const int s = it % kStages;
-          PROF_BEGIN(w0);
-          mbar_wait(&full[s], (uint32_t)(it / kStages) & 1);
-          PROF_END(0, w0);
-          PROF_BEGIN(w2);
-          tc_fence_after();
-          const uint64_t aH0 = dA0 + (uint64_t)((seg & 1) * 2 + kc) * 2 * kA16, aL0 = aH0 + kA16;
-          const uint64_t bH0 = dB0 + (uint64_t)s * kS16, bL0 = bH0 + kB16;
+        PROF_BEGIN(w0);
+        mbar_wait(&full[s], ph);
+        PROF_END(0, w0);
+        PROF_BEGIN(w2);
+        tc_fence_after();
+        const uint64_t aT = dA0 + (uint64_t)(seg & 1) * aBuf16, bT = dB0 + (uint64_t)s * stage16;
+#pragma unroll
+        for (int kc = 0; kc < 2; ++kc) {
+          if (kc >= n_kc) break;
+          const uint64_t aH0 = aT + g.plane_off[kc] * kA16, aL0 = aH0 + kA16;
+          const uint64_t bH0 = bT + g.plane_off[kc] * kB16, bL0 = bH0 + kB16;
 #pragma unroll
           for (int ks = 0; ks < 2; ++ks) {
             const uint32_t np = (plan >> (2 * (2 * kc + ks))) & 3u;
@@ -460,27 +524,21 @@ __global__ void __launch_bounds__(kTcThreads, 1)
               mma_f16_ss_if(dS, aH0 + o, bH0 + o, idS, acc0, lead);
             }
           }
-          tc_commit_if(&empty[s], lead);
-          PROF_END(2, w2);
         }
+        tc_commit_if(&empty[s], lead);
         tc_commit_if(&sfull[bq], lead);
+        PROF_END(2, w2);
+        if (++s == g.D) {
+          s = 0;
+          ph ^= 1u;
+        }
       }
     } else {
     UnitIt cu = unit_begin(sc);
     int prev_st = 0;
-    int seg = -1;
-    int64_t cur_tt = -1;
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
       const int bq = q & 1;
       const uint32_t dS = tbase + (bq ? (uint32_t)TS : 0u);
-      if (AR && cu.tt != cur_tt) {  // new target tile: release the previous operand buffer, wait for this one
-        if (seg >= 0 && leader) tc_commit(&aempty[seg & 1]);
-        __syncwarp();
-        ++seg;
-        cur_tt = cu.tt;
-        mbar_wait(&afull[seg & 1], (uint32_t)((seg >> 1) & 1));
-        tc_fence_after();
-      }
       if constexpr (VCC) {
         if (q >= 2) {  // the epilogue has read S(q-2) out of this buffer
           PROF_BEGIN(w1);
@@ -498,11 +556,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         PROF_BEGIN(w2);
         tc_fence_after();
         uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
-        // operand descriptors: A (targets) from the stage or the resident buffer, B from the stage
-        const uint64_t dAh = AR ? sdesc_k_sw64(smem + TcSmem::a_chunk(seg & 1, kc, 0)) : sdesc_k_sw64(sp);
-        const uint64_t dAl = AR ? sdesc_k_sw64(smem + TcSmem::a_chunk(seg & 1, kc, 1)) : sdesc_k_sw64(sp + kChunkA);
-        const uint64_t dBh = sdesc_k_sw64(sp + (AR ? 0u : 2 * kChunkA));
-        const uint64_t dBl = sdesc_k_sw64(sp + (AR ? 0u : 2 * kChunkA) + kChunkB);
+        const uint64_t dAh = sdesc_k_sw64(sp), dAl = sdesc_k_sw64(sp + kChunkA);
+        const uint64_t dBh = sdesc_k_sw64(sp + 2 * kChunkA), dBl = sdesc_k_sw64(sp + 2 * kChunkA + kChunkB);
 #pragma unroll
         for (int ks = 0; ks < kTcKC / 8; ++ks) {
           const uint64_t aH = dAh + (uint64_t)((ks * 32) >> 4);
