@@ -25,15 +25,40 @@ __device__ __forceinline__ void batch(const uint32_t (&sv)[32], f2_t (&acc)[2]) 
   }
 }
 
-template <int NPOLY, int PIPE>
+// MMA = 1: warp 1 meanwhile issues back-to-back kind::f16 M=128 N=256 MMAs (zero operands)
+// into TMEM columns the epilogue does not read (tests TMEM / issue interference)
+template <int NPOLY, int PIPE, int MMA = 0>
 __global__ void __launch_bounds__(640, 1) k(float* out) {
+  extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ uint32_t tb_smem;
+  __shared__ int stop;
+  __shared__ __align__(8) uint64_t bar;
   const int tid = threadIdx.x, warp = tid >> 5;
   if (warp == 2) tmem_alloc(&tb_smem, 512);
+  if (tid == 0) { stop = 0; mbar_init(&bar, 1); fence_mbar_init(); }
+  for (int i = tid; i < 384 * 64 / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(smem)[i] = 0u;
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = tb_smem;
+  if (MMA && warp == 1) {
+    const bool leader = elect_one();
+    const uint64_t dA = sdesc_k_sw64(smem), dB = sdesc_k_sw64(smem + 128 * 64);
+    const uint32_t id = idesc_f16(128, 256);
+    int n = 0;
+    while (*(volatile int*)&stop < 16) {
+      if (leader) mma_f16_ss(tbase + 256, dA + (uint64_t)((n & 1) * 2), dB + (uint64_t)((n & 1) * 2), id, n & 1);
+      __syncwarp();
+      ++n;
+      if ((n & 63) == 0) {  // keep the queue bounded
+        if (leader) tc_commit(&bar);
+        __syncwarp();
+        mbar_wait(&bar, (uint32_t)(((n >> 6) - 1) & 1));
+      }
+    }
+    if (tid == 32 && blockIdx.x == 0) out[1] = (float)n;
+  }
   if (warp >= 4) {
     const int ew = warp - 4, g = ew & 3, h = ew >> 2;
     const uint32_t lane_off = (uint32_t)(32 * g) << 16;
@@ -43,7 +68,7 @@ __global__ void __launch_bounds__(640, 1) k(float* out) {
 #pragma unroll
         for (int hh = 0; hh < 4; ++hh) {
           uint32_t sv[32];
-          tmem_ldn<32>(tbase + lane_off + (q & 1) * 256 + (h & 1) * 128 + 32 * hh, sv);
+          tmem_ldn<32>(tbase + lane_off + (h & 1) * 128 + 32 * hh, sv);
           tmem_wait_ld();
           batch<NPOLY>(sv, acc);
         }
@@ -55,10 +80,10 @@ __global__ void __launch_bounds__(640, 1) k(float* out) {
 #pragma unroll
         for (int hh = 0; hh < 4; hh += 2) {
           tmem_wait_ld();
-          tmem_ldn<32>(tbase + lane_off + (q & 1) * 256 + (h & 1) * 128 + 32 * (hh + 1), sb);
+          tmem_ldn<32>(tbase + lane_off + (h & 1) * 128 + 32 * (hh + 1), sb);
           batch<NPOLY>(sa, acc);
           tmem_wait_ld();
-          tmem_ldn<32>(tbase + lane_off + ((q + (hh == 2)) & 1) * 256 + (h & 1) * 128 + 32 * ((hh + 2) & 3), sa);
+          tmem_ldn<32>(tbase + lane_off + (h & 1) * 128 + 32 * ((hh + 2) & 3), sa);
           batch<NPOLY>(sb, acc);
         }
       }
@@ -68,21 +93,24 @@ __global__ void __launch_bounds__(640, 1) k(float* out) {
     f2_unpack(acc[0], a, b);
     f2_unpack(acc[1], c, d);
     if (a + b + c + d == 1234.5f) out[0] = a;
+    if ((threadIdx.x & 31) == 0) atomicAdd(&stop, 1);
   }
   tc_fence_before();
   __syncthreads();
   if (warp == 2) tmem_dealloc(tbase, 512);
 }
 
-template <int NPOLY, int PIPE>
+template <int NPOLY, int PIPE, int MMA = 0>
 void run(float* out, int G) {
+  const int smem = 384 * 64 + 1024;
+  cudaFuncSetAttribute(k<NPOLY, PIPE, MMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   cudaEvent_t e0, e1;
   cudaEventCreate(&e0);
   cudaEventCreate(&e1);
   float best = 1e9;
   for (int r = 0; r < 5; ++r) {
     cudaEventRecord(e0);
-    k<NPOLY, PIPE><<<G, 640>>>(out);
+    k<NPOLY, PIPE, MMA><<<G, 640, smem>>>(out);
     cudaEventRecord(e1);
     cudaEventSynchronize(e1);
     float ms;
@@ -90,22 +118,23 @@ void run(float* out, int G) {
     if (ms < best) best = ms;
   }
   const double warp_elems_per_smsp = (double)TILES * 128 * 4;  // 4 compute warps per SMSP, 128 columns each
-  printf("NPOLY %d PIPE %d  %.3f ms  %.2f SMSP-cycles per warp-element @1965 (MUFU floor %.2f)\n", NPOLY, PIPE,
+  float nm = 0.f;
+  cudaMemcpy(&nm, out + 1, 4, cudaMemcpyDeviceToHost);
+  printf("NPOLY %d PIPE %d MMA %d (%.0f MMAs/CTA) %.3f ms  %.2f SMSP-cycles per warp-element @1965 (MUFU floor %.2f)\n", NPOLY, PIPE, MMA, MMA ? nm : 0.f,
          best, best * 1e-3 * 1.965e9 / warp_elems_per_smsp, 8.1 * (16 - NPOLY) / 16);
 }
 int main() {
   cudaDeviceProp p;
   cudaGetDeviceProperties(&p, 0);
   float* out;
-  cudaMalloc(&out, 4);
+  cudaMalloc(&out, 8);
   const int G = p.multiProcessorCount;
   run<0, 0>(out, G);
   run<4, 0>(out, G);
   run<6, 0>(out, G);
   run<8, 0>(out, G);
-  run<0, 1>(out, G);
-  run<4, 1>(out, G);
   run<6, 1>(out, G);
-  run<8, 1>(out, G);
+  run<0, 0, 1>(out, G);
+  run<6, 0, 1>(out, G);
   printf("%s\n", cudaGetErrorString(cudaDeviceSynchronize()));
 }
