@@ -133,6 +133,9 @@ struct ks_ctx {
   CUtensorMap tmB_hi, tmB_lo;
   DBuf<float> mu;         // [k_pad]
   DBuf<double> mean_part; // [nparts][K]
+  DBuf<float> mean_pmm;   // [nparts][K][2] column min/max
+  DBuf<unsigned> mean_pw; // [nparts][2] weight statistics
+  DBuf<unsigned> stats_counter;  // arrival counter of the statistics kernel (left zero)
   CUtensorMap tmap_src;
 
   // eval scratch
@@ -190,6 +193,28 @@ ks_status timed_end(ks_ctx* ctx, cudaEvent_t stop) {
   return KS_OK;
 }
 
+// One launch: mu (always), amax (FP16 modes), wstat (want_w, R = 1).
+cudaError_t source_stats(ks_ctx* ctx, const float* alpha, const float* W, bool want_w, int64_t M, int k_pad,
+                         bool want_amax) {
+  cudaStream_t st = ctx->stream;
+  const int K = ctx->K;
+  int nparts = (int)((M + 255) / 256);  // blocks of >= 256 rows each (one wave; short final reduction)
+  if (nparts < 1) nparts = 1;
+  if (nparts > 1024) nparts = 1024;
+  cudaError_t e;
+  if ((e = ctx->mean_part.reserve((size_t)nparts * K, st, false)) != cudaSuccess) return e;
+  if ((e = ctx->mean_pmm.reserve((size_t)nparts * K * 2, st, false)) != cudaSuccess) return e;
+  if ((e = ctx->mean_pw.reserve((size_t)nparts * 2, st, false)) != cudaSuccess) return e;
+  if ((e = ctx->stats_counter.reserve(1, st, true)) != cudaSuccess) return e;
+  if ((e = ctx->mu.reserve(k_pad, st, false)) != cudaSuccess) return e;
+  if (want_amax && (e = ctx->amax.reserve(1, st, false)) != cudaSuccess) return e;
+  if (want_w && (e = ctx->wstat.reserve(2, st, false)) != cudaSuccess) return e;
+  ctx->launches += 1;
+  return ks::launch_source_stats(alpha, W, M, K, k_pad, nparts, ctx->mean_part.p, ctx->mean_pmm.p, ctx->mean_pw.p,
+                                 ctx->stats_counter.p, ctx->mu.p, want_amax ? ctx->amax.p : nullptr,
+                                 want_w ? ctx->wstat.p : nullptr, st);
+}
+
 ks_status prepare_fp32(ks_ctx* ctx, const float* alpha, const float* W, int64_t M) {
   const int K = ctx->K;
   const int k_pad = fp32_k_pad(K);
@@ -198,12 +223,7 @@ ks_status prepare_fp32(ks_ctx* ctx, const float* alpha, const float* W, int64_t 
   const size_t need = (size_t)(k_pad + 2) * (size_t)m_pad;
   KS_CUDA(ctx->src.reserve(need, st, false), "allocate source buffer");
   KS_CUDA(ctx->mu.reserve(k_pad, st, false), "allocate mean buffer");
-  int nparts = (int)((M + 63) / 64);  // source-mean blocks of <= 64 rows each
-  if (nparts < 1) nparts = 1;
-  if (nparts > 2048) nparts = 2048;
-  KS_CUDA(ctx->mean_part.reserve((size_t)nparts * K, st, false), "allocate mean partials");
-  KS_CUDA(ks::launch_source_mean(alpha, M, K, k_pad, ctx->mean_part.p, nparts, ctx->mu.p, st), "source mean");
-  ctx->launches += (M > 0) ? 2 : 1;
+  KS_CUDA(source_stats(ctx, alpha, nullptr, false, M, k_pad, false), "source mean");
   KS_CUDA(ks::launch_prep_fp32(alpha, W, M, m_pad, K, k_pad, ctx->mu.p, ctx->c, ctx->src.p, st), "source prep");
   ctx->launches += 1;
 
@@ -348,22 +368,10 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(ctx->wt_lo.reserve(nw, st, false), "allocate W lo");
   KS_CUDA(ctx->wv.reserve((size_t)m_pad * (vcc ? vcc : 1), st, false), "allocate W rows");
   KS_CUDA(ctx->mu.reserve(k_pad, st, false), "allocate mean buffer");
-  int nparts = (int)((M + 63) / 64);  // source-mean blocks of <= 64 rows each
-  if (nparts < 1) nparts = 1;
-  if (nparts > 2048) nparts = 2048;
-  KS_CUDA(ctx->mean_part.reserve((size_t)nparts * K, st, false), "allocate mean partials");
-  KS_CUDA(ks::launch_source_mean(alpha, M, K, k_pad, ctx->mean_part.p, nparts, ctx->mu.p, st), "source mean");
-  ctx->launches += (M > 0) ? 2 : 1;
-  if (use_wstat) {
-    KS_CUDA(ctx->wstat.reserve(2, st, false), "allocate weight stats");
-    KS_CUDA(ks::launch_weight_stats(W, M, ctx->wstat.p, st), "weight stats");
-    ctx->launches += (M > 0) ? 1 : 0;
-  }
+  // mean, max |alpha - mu| (FP16 scaling) and the R = 1 weight statistics in one launch
+  KS_CUDA(source_stats(ctx, alpha, W, use_wstat, M, k_pad, f16), "source statistics");
   const unsigned* wst = use_wstat ? ctx->wstat.p : nullptr;
   if (f16) {
-    KS_CUDA(ctx->amax.reserve(1, st, false), "allocate source max");
-    KS_CUDA(ks::launch_source_absmax(alpha, M, K, ctx->mu.p, ctx->amax.p, st), "source max (FP16 scaling)");
-    ctx->launches += (M > 0) ? 1 : 0;
     KS_CUDA(ks::launch_prep_f16_sources(alpha, W, M, m_pad, K, k_pad, R, vcc ? 0 : r_pad, ctx->mu.p, ctx->c,
                                         ctx->amax.p, fold, ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p,
                                         ctx->wt_lo.p, ctx->wv.p, vcc, wst, st),
@@ -575,6 +583,9 @@ ks_status ks_destroy(ks_ctx* ctx) {
   ctx->wstat.release();
   ctx->mu.release();
   ctx->mean_part.release();
+  ctx->mean_pmm.release();
+  ctx->mean_pw.release();
+  ctx->stats_counter.release();
   ctx->partial.release();
   ctx->counters.release();
   ctx->dbg_times.release();

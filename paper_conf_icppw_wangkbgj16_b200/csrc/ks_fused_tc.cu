@@ -1086,15 +1086,6 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 }
 
 // ---------------------------------------------------------------- prep (a1 / a2 for the TC path)
-// One warp per point: lanes stride over the coordinates (coalesced reads of a
-// row and coalesced writes of its padded split row), the norm is a fixed-order
-// FP64 warp reduction (lane partials in lane order via shuffles).
-__device__ __forceinline__ double warp_sum_fixed(double v) {
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
-  return __shfl_sync(0xffffffffu, v, 0);
-}
-
 // Exponent s such that amax * 2^s lies in [2^12, 2^13) (FP16 mode operand
 // scaling; clamped so that 2^-(sA + sB) stays a normal FP32 number).
 __device__ __forceinline__ int f16_scale_exp(float amax) {
@@ -1111,7 +1102,34 @@ __device__ __forceinline__ void split_f16(float x, __half& hi, __half& lo) {
 }
 
 
-template <bool F16>
+// Prep kernels: G lanes per point (G in {4, 8, 16, 32}), so a warp prepares 32/G
+// points at once and its loads and stores stay contiguous per point; a lane owns
+// dimensions gl, gl + G, ... of the input and the pairs (2 gl, 2 gl + 1) + 2G it
+// of the padded output row (one 4-byte FP16 pair or 8-byte TF32 pair per store).
+// The point count (m_pad, n_pad) is a multiple of 128, so a warp's points are all
+// in range or all out (full-mask shuffles).  Norms: FP64 partials of the G lanes,
+// combined by an xor butterfly (every lane of the group gets the same bits).
+template <int G>
+__device__ __forceinline__ double group_sum(double v) {
+#pragma unroll
+  for (int o = G / 2; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+template <int G>
+__device__ __forceinline__ float group_max(float v) {
+#pragma unroll
+  for (int o = G / 2; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+// KS_PREP_G = 4, 8, 16 or 32 overrides (measurement knob)
+int prep_group(int K) {
+  const char* e = getenv("KS_PREP_G");
+  const int g = e ? atoi(e) : 0;
+  if (g == 4 || g == 8 || g == 16 || g == 32) return g;
+  return K <= 8 ? 4 : 8;
+}
+
+template <bool F16, int G>
 __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const float* __restrict__ W, int64_t M,
                                        int64_t m_pad, int K, int k_pad, int R, int r_pad,
                                        const float* __restrict__ mu, double c, int aug,
@@ -1119,16 +1137,17 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
                                        void* __restrict__ src_lo, float* __restrict__ na,
                                        float* __restrict__ wt_hi, float* __restrict__ wt_lo,
                                        float* __restrict__ wv, int rv, const unsigned* __restrict__ wstat) {
-  const int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int lane = threadIdx.x & 31;
+  const int lane = threadIdx.x & 31, gl = lane & (G - 1);
+  const int64_t i = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
   if (i >= m_pad) return;
   const bool live = i < M;
   double n = 0.0;
-  for (int d = lane; d < K; d += 32) {
+#pragma unroll 4
+  for (int d = gl; d < K; d += G) {
     const float x = live ? alpha[i * K + d] - mu[d] : 0.f;  // FP32 centring, same op as the target side
     n += (double)x * (double)x;
   }
-  n = warp_sum_fixed(n);
+  n = group_sum<G>(n);
   const float nai = live ? (float)(-c * n) : 0.f;
   const double c2 = 2.0 * c;
   const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u;
@@ -1148,32 +1167,38 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
       sA = ldexpf(1.f, f16_scale_exp((float)(c2 * (double)__uint_as_float(*amax))));
     }
   }
-  for (int d = lane; d < k_pad; d += 32) {
-    float a = 0.f;
+  auto coord = [&](int d) -> float {
     if (d < K) {
       const float x = live ? alpha[i * K + d] - mu[d] : 0.f;
-      a = (float)(c2 * (double)x);
-    } else if (!F16 && aug && d == K) {
-      a = 1.f;   // multiplies nb_j of the target
-    } else if (!F16 && aug && d == K + 1) {
-      a = nai;   // times 1 on the target side
+      return (float)(c2 * (double)x);
     }
+    if (!F16 && aug && d == K) return 1.f;   // multiplies nb_j of the target
+    if (!F16 && aug && d == K + 1) return nai;  // times 1 on the target side
+    return 0.f;
+  };
+  for (int d = 2 * gl; d < k_pad; d += 2 * G) {
+    const float a0 = coord(d), a1 = coord(d + 1);
     if constexpr (F16) {
-      __half h, l;
-      split_f16(a * sA, h, l);  // exact power-of-2 scaling
+      __half h0, l0, h1, l1;
+      split_f16(a0 * sA, h0, l0);  // exact power-of-2 scaling
+      split_f16(a1 * sA, h1, l1);
       if (fa && d >= K && d < K + 6) {  // folded norm columns: hi planes only
-        h = d < K + 3 ? np[d - K] : __float2half(1.f);
-        l = __float2half(0.f);
+        h0 = d < K + 3 ? np[d - K] : __float2half(1.f);
+        l0 = __float2half(0.f);
       }
-      static_cast<__half*>(src_hi)[i * k_pad + d] = h;
-      static_cast<__half*>(src_lo)[i * k_pad + d] = l;
+      if (fa && d + 1 >= K && d + 1 < K + 6) {
+        h1 = d + 1 < K + 3 ? np[d + 1 - K] : __float2half(1.f);
+        l1 = __float2half(0.f);
+      }
+      static_cast<__half2*>(src_hi)[(i * k_pad + d) >> 1] = __halves2half2(h0, h1);
+      static_cast<__half2*>(src_lo)[(i * k_pad + d) >> 1] = __halves2half2(l0, l1);
     } else {
-      const float ah = to_tf32(a);
-      static_cast<float*>(src_hi)[i * k_pad + d] = ah;
-      static_cast<float*>(src_lo)[i * k_pad + d] = to_tf32(a - ah);
+      const float ah0 = to_tf32(a0), ah1 = to_tf32(a1);
+      static_cast<float2*>(src_hi)[(i * k_pad + d) >> 1] = make_float2(ah0, ah1);
+      static_cast<float2*>(src_lo)[(i * k_pad + d) >> 1] = make_float2(to_tf32(a0 - ah0), to_tf32(a1 - ah1));
     }
   }
-  if (lane == 0) {
+  if (gl == 0) {
     if (fa) {
       na[i] = 0.f;  // folded: the norm and log-weight ride in the contraction
     } else if (logw) {
@@ -1183,13 +1208,13 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
       na[i] = aug && !F16 ? 0.f : nai;  // aug: the norms ride in the contraction, the epilogue adds 0
     }
   }
-  for (int r = lane; r < rv; r += 32) {
+  for (int r = gl; r < rv; r += G) {
     if (logw)  // R = 1, W >= 0: the slot holds lw_i = log2(W_i / Wmax), the clamp bound (Q23)
-      wv[i * rv + r] = live ? (float)(log2((double)W[i]) - log2((double)__uint_as_float(wstat[0]))) : -INFINITY;
+      wv[i * rv + r] = (float)wl;
     else
       wv[i * rv + r] = (live && r < R) ? W[i * R + r] : 0.f;
   }
-  for (int r = lane; r < r_pad; r += 32) {
+  for (int r = gl; r < r_pad; r += G) {
     const float w = (live && r < R) ? W[i * R + r] : 0.f;
     const float wh = to_tf32(w);
     wt_hi[(int64_t)r * m_pad + i] = wh;
@@ -1197,24 +1222,25 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
   }
 }
 
-template <bool F16>
+template <bool F16, int G>
 __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N, int64_t n_pad, int K, int k_pad,
                                        const float* __restrict__ mu, double c, int aug,
                                        const unsigned* __restrict__ amax, void* __restrict__ tgt_hi,
                                        void* __restrict__ tgt_lo, float* __restrict__ nb,
                                        float* __restrict__ tsc) {
-  const int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int lane = threadIdx.x & 31;
+  const int lane = threadIdx.x & 31, gl = lane & (G - 1);
+  const int64_t j = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
   if (j >= n_pad) return;
   const bool live = j < N;
   double n = 0.0;
   float bmax = 0.f;
-  for (int d = lane; d < K; d += 32) {
+#pragma unroll 4
+  for (int d = gl; d < K; d += G) {
     const float x = live ? beta[j * K + d] - mu[d] : 0.f;
     n += (double)x * (double)x;
     bmax = fmaxf(bmax, fabsf(x));
   }
-  n = warp_sum_fixed(n);
+  n = group_sum<G>(n);
   const float nbj = live ? (float)(-c * n) : 0.f;
   float sB = 1.f, rj = 1.f;
   bool fa = false, far = false;  // folded layout active; row beyond every source (kernel row 0)
@@ -1227,87 +1253,84 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
       if (far) mp[0] = __float2half(kFoldNegInf);
       else split3_f16(-c * n, mp);
     } else {
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) bmax = fmaxf(bmax, __shfl_xor_sync(0xffffffffu, bmax, o));
+      bmax = group_max<G>(bmax);
       const int eA = f16_scale_exp((float)(2.0 * c * (double)__uint_as_float(*amax)));
       const int eB = f16_scale_exp(bmax);
       sB = ldexpf(1.f, eB);
       rj = ldexpf(1.f, -(eA + eB));
     }
   }
-  for (int d = lane; d < k_pad; d += 32) {
-    float x = 0.f;
-    if (d < K) x = (live && !far) ? beta[j * K + d] - mu[d] : 0.f;
-    else if (!F16 && aug && d == K) x = nbj;
-    else if (!F16 && aug && d == K + 1) x = 1.f;
+  auto coord = [&](int d) -> float {
+    if (d < K) return (live && !far) ? beta[j * K + d] - mu[d] : 0.f;
+    if (!F16 && aug && d == K) return nbj;
+    if (!F16 && aug && d == K + 1) return 1.f;
+    return 0.f;
+  };
+  for (int d = 2 * gl; d < k_pad; d += 2 * G) {
+    const float x0 = coord(d), x1 = coord(d + 1);
     if constexpr (F16) {
-      __half h, l;
-      split_f16(x * sB, h, l);
+      __half h0, l0, h1, l1;
+      split_f16(x0 * sB, h0, l0);
+      split_f16(x1 * sB, h1, l1);
       if (fa && d >= K && d < K + 6) {  // folded norm columns: hi planes only
-        h = d < K + 3 ? __float2half(1.f) : mp[d - K - 3];
-        l = __float2half(0.f);
+        h0 = d < K + 3 ? __float2half(1.f) : mp[d - K - 3];
+        l0 = __float2half(0.f);
       }
-      static_cast<__half*>(tgt_hi)[j * k_pad + d] = h;
-      static_cast<__half*>(tgt_lo)[j * k_pad + d] = l;
+      if (fa && d + 1 >= K && d + 1 < K + 6) {
+        h1 = d + 1 < K + 3 ? __float2half(1.f) : mp[d + 1 - K - 3];
+        l1 = __float2half(0.f);
+      }
+      static_cast<__half2*>(tgt_hi)[(j * k_pad + d) >> 1] = __halves2half2(h0, h1);
+      static_cast<__half2*>(tgt_lo)[(j * k_pad + d) >> 1] = __halves2half2(l0, l1);
     } else {
-      const float xh = to_tf32(x);
-      static_cast<float*>(tgt_hi)[j * k_pad + d] = xh;
-      static_cast<float*>(tgt_lo)[j * k_pad + d] = to_tf32(x - xh);
+      const float xh0 = to_tf32(x0), xh1 = to_tf32(x1);
+      static_cast<float2*>(tgt_hi)[(j * k_pad + d) >> 1] = make_float2(xh0, xh1);
+      static_cast<float2*>(tgt_lo)[(j * k_pad + d) >> 1] = make_float2(to_tf32(x0 - xh0), to_tf32(x1 - xh1));
     }
   }
-  if (lane == 0) {
+  if (gl == 0) {
     nb[j] = aug ? 0.f : nbj;  // aug (TF32) / folded (FP16): the norm rides in the contraction
     tsc[j] = rj;
   }
 }
 
-// max_i,d |alpha[i][d] - mu[d]| as FP32 bits (non-negative floats order as unsigned ints).
-__global__ void source_absmax_kernel(const float* __restrict__ alpha, int64_t total, int K,
-                                     const float* __restrict__ mu, unsigned* __restrict__ amax) {
-  float m = 0.f;
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x)
-    m = fmaxf(m, fabsf(alpha[e] - mu[e % K]));
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
-  if ((threadIdx.x & 31) == 0) atomicMax(amax, __float_as_uint(m));
-}
-
-__global__ void weight_stats_kernel(const float* __restrict__ W, int64_t M, unsigned* __restrict__ wstat) {
-  float m = 0.f;
-  unsigned neg = 0u;
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < M; e += (int64_t)gridDim.x * blockDim.x) {
-    const float w = W[e];
-    m = fmaxf(m, fabsf(w));
-    neg |= (w < 0.f || w != w) ? 1u : 0u;  // NaN weights take the general path
+template <bool F16>
+static cudaError_t launch_prep_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K,
+                                       int k_pad, int R, int r_pad, const float* mu, double c, int aug,
+                                       const unsigned* amax, void* src_hi, void* src_lo, float* na, float* wt_hi,
+                                       float* wt_lo, float* wv, int rv, const unsigned* wstat, cudaStream_t st) {
+  if (m_pad == 0) return cudaSuccess;
+  const int bs = 256, G = prep_group(K);
+  const unsigned grid = (unsigned)((m_pad * G + bs - 1) / bs);
+#define KS_PREP_S(g)                                                                                          \
+  prep_tc_sources_kernel<F16, g><<<grid, bs, 0, st>>>(alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, amax, \
+                                                      src_hi, src_lo, na, wt_hi, wt_lo, wv, rv, wstat)
+  switch (G) {
+    case 4: KS_PREP_S(4); break;
+    case 8: KS_PREP_S(8); break;
+    case 16: KS_PREP_S(16); break;
+    default: KS_PREP_S(32); break;
   }
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
-    neg |= __shfl_xor_sync(0xffffffffu, neg, o);
-  }
-  if ((threadIdx.x & 31) == 0) {
-    atomicMax(&wstat[0], __float_as_uint(m));
-    if (neg) atomicOr(&wstat[1], 1u);
-  }
-}
-
-cudaError_t launch_weight_stats(const float* W, int64_t M, unsigned* wstat, cudaStream_t st) {
-  cudaError_t e = cudaMemsetAsync(wstat, 0, 2 * sizeof(unsigned), st);
-  if (e != cudaSuccess || M == 0) return e;
-  int64_t blocks = (M + 255) / 256;
-  if (blocks > 4 * 148) blocks = 4 * 148;
-  weight_stats_kernel<<<(unsigned)blocks, 256, 0, st>>>(W, M, wstat);
+#undef KS_PREP_S
   return cudaGetLastError();
 }
 
-cudaError_t launch_source_absmax(const float* alpha, int64_t M, int K, const float* mu, unsigned* amax,
-                                 cudaStream_t st) {
-  cudaError_t e = cudaMemsetAsync(amax, 0, sizeof(unsigned), st);
-  if (e != cudaSuccess || M == 0) return e;
-  const int64_t total = M * K;
-  int64_t blocks = (total + 255) / 256;
-  if (blocks > 4 * 148) blocks = 4 * 148;
-  source_absmax_kernel<<<(unsigned)blocks, 256, 0, st>>>(alpha, total, K, mu, amax);
+template <bool F16>
+static cudaError_t launch_prep_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad,
+                                       const float* mu, double c, int aug, const unsigned* amax, void* tgt_hi,
+                                       void* tgt_lo, float* nb, float* tsc, cudaStream_t st) {
+  if (n_pad == 0) return cudaSuccess;
+  const int bs = 256, G = prep_group(K);
+  const unsigned grid = (unsigned)((n_pad * G + bs - 1) / bs);
+#define KS_PREP_T(g) \
+  prep_tc_targets_kernel<F16, g><<<grid, bs, 0, st>>>(beta, N, n_pad, K, k_pad, mu, c, aug, amax, tgt_hi, tgt_lo, nb, tsc)
+  switch (G) {
+    case 4: KS_PREP_T(4); break;
+    case 8: KS_PREP_T(8); break;
+    case 16: KS_PREP_T(16); break;
+    default: KS_PREP_T(32); break;
+  }
+#undef KS_PREP_T
   return cudaGetLastError();
 }
 
@@ -1315,42 +1338,28 @@ cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M
                                    int R, int r_pad, const float* mu, double c, int aug, float* src_hi,
                                    float* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv, int rv,
                                    const unsigned* wstat, cudaStream_t st) {
-  if (m_pad == 0) return cudaSuccess;
-  const int bs = 256;  // 8 points per block
-  prep_tc_sources_kernel<false><<<(unsigned)((m_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
-      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, nullptr, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv, wstat);
-  return cudaGetLastError();
+  return launch_prep_sources<false>(alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, nullptr, src_hi, src_lo, na,
+                                    wt_hi, wt_lo, wv, rv, wstat, st);
 }
 
 cudaError_t launch_prep_f16_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,
                                     int R, int r_pad, const float* mu, double c, const unsigned* amax, int fold,
                                     void* src_hi, void* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv,
                                     int rv, const unsigned* wstat, cudaStream_t st) {
-  if (m_pad == 0) return cudaSuccess;
-  const int bs = 256;
-  prep_tc_sources_kernel<true><<<(unsigned)((m_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
-      alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, fold, amax, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv, wstat);
-  return cudaGetLastError();
+  return launch_prep_sources<true>(alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, fold, amax, src_hi, src_lo, na,
+                                   wt_hi, wt_lo, wv, rv, wstat, st);
 }
 
 cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
                                    double c, int aug, float* tgt_hi, float* tgt_lo, float* nb, float* tsc,
                                    cudaStream_t st) {
-  if (n_pad == 0) return cudaSuccess;
-  const int bs = 256;
-  prep_tc_targets_kernel<false><<<(unsigned)((n_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
-      beta, N, n_pad, K, k_pad, mu, c, aug, nullptr, tgt_hi, tgt_lo, nb, tsc);
-  return cudaGetLastError();
+  return launch_prep_targets<false>(beta, N, n_pad, K, k_pad, mu, c, aug, nullptr, tgt_hi, tgt_lo, nb, tsc, st);
 }
 
 cudaError_t launch_prep_f16_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
                                     double c, const unsigned* amax, int fold, void* tgt_hi, void* tgt_lo, float* nb,
                                     float* tsc, cudaStream_t st) {
-  if (n_pad == 0) return cudaSuccess;
-  const int bs = 256;
-  prep_tc_targets_kernel<true><<<(unsigned)((n_pad * 32 + bs - 1) / bs), bs, 0, st>>>(
-      beta, N, n_pad, K, k_pad, mu, c, fold, amax, tgt_hi, tgt_lo, nb, tsc);
-  return cudaGetLastError();
+  return launch_prep_targets<true>(beta, N, n_pad, K, k_pad, mu, c, fold, amax, tgt_hi, tgt_lo, nb, tsc, st);
 }
 
 // Pipeline depth: KS_TC_STAGES (3..6) overrides the default (measurement knob).

@@ -23,8 +23,14 @@ struct StreamK {
 
 // ---------------------------------------------------------------- prep (a1)
 // mu[d] (FP32, d < k_pad; zero for d >= K) = mean_i alpha[i][d], FP64 accumulation, fixed order.
-cudaError_t launch_source_mean(const float* alpha, int64_t M, int K, int k_pad, double* part, int nparts,
-                               float* mu, cudaStream_t st);
+// Source statistics, one launch (ks_prep.cu): mu [k_pad] (FP32 mean, 0 for
+// padding dims); if amax != nullptr its FP32 bits of max |alpha - mu|; if W !=
+// nullptr (R = 1) wstat = {bits of max |W_i|, any W_i < 0 or NaN}.  Scratch:
+// part [nparts][K] doubles, pmm [nparts][K][2] floats, pw [nparts][2]; counter
+// must be zero before the first call and is left zero.
+cudaError_t launch_source_stats(const float* alpha, const float* W, int64_t M, int K, int k_pad, int nparts,
+                                double* part, float* pmm, unsigned* pw, unsigned* counter, float* mu,
+                                unsigned* amax, unsigned* wstat, cudaStream_t st);
 
 // FP32 path source layout, dimension-major [k_pad + 2][m_pad]:
 //   rows d < k_pad : a[d][i]  = RN(2c * (alpha[i][d] - mu[d]))
@@ -110,17 +116,14 @@ cudaError_t launch_prep_tc_targets(const float* beta, int64_t N, int64_t n_pad, 
                                    cudaStream_t st);
 // FP16 mode (KS_PREC_3XF16).  k_pad is a multiple of 2*kTcKC halves (one
 // 64-byte row chunk per stage, as in TF32 mode).  amax = max |alpha - mu|
-// (FP32 bits, atomicMax; must be zeroed first).  Sources are scaled by
+// (FP32 bits, from launch_source_stats).  Sources are scaled by
 // sA = 2^(13 - e), e = exponent of RN(2c * amax) (frexp convention), targets
 // per row by sB_j = 2^(13 - e_j) from max_k |beta_jk - mu_k|; each scaled
 // value x is split x = hi + lo, hi = RN_f16(x), lo = RN_f16(x - hi);
 // tsc[j] = 2^-(log2 sA + log2 sB_j) undoes the scaling on S.
-// R = 1 weight statistics: wstat[0] = FP32 bits of max |W_i|, wstat[1] = 1 if any W_i < 0.
-// With W >= 0 and max > 0 the source prep stores na_i + log2(W_i / max) in na
+// R = 1 weight statistics (launch_source_stats): wstat[0] = FP32 bits of max |W_i|,
+// wstat[1] = 1 if any W_i < 0.  With W >= 0 and max > 0 the source prep stores na_i + log2(W_i / max) in na
 // (-inf for W_i = 0) and the fused kernel sums 2^t, scaling by max at the end.
-cudaError_t launch_weight_stats(const float* W, int64_t M, unsigned* wstat, cudaStream_t st);
-cudaError_t launch_source_absmax(const float* alpha, int64_t M, int K, const float* mu, unsigned* amax,
-                                 cudaStream_t st);
 // fold = 1 (R = 1): folded layout, k_pad >= K + 6 -- columns K..K+5 carry the
 // norms (and log-weights) as FP16 pieces when c K amax^2 <= 2^12 (checked on
 // the device); operands are then scaled by 2^eF / 2^-eF and tsc = 1, nb = na = 0.

@@ -15,63 +15,183 @@
 
 namespace ks {
 
-// Each block sums a contiguous chunk of rows in a fixed order.  For K <= 256
-// the 256 threads form rpp = 256/K row lanes x K dims (coalesced reads); the
-// rpp lane sums of a dim are then added in lane order.  For K > 256 thread t
-// owns dims t, t+256, ...
-__global__ void source_mean_partial_kernel(const float* __restrict__ alpha, int64_t M, int K, int nparts,
-                                           double* __restrict__ part) {
+// Source statistics in one launch.  Each block reduces a contiguous chunk of
+// rows in a fixed order: FP64 column sums, FP32 column min/max and (R = 1 log-
+// weight mode) max |W_i| and "any W_i < 0 or NaN".  The last block to finish
+// (arrival counter, reset for the next call) reduces the block partials in
+// fixed block order -- the result is bitwise independent of which block is
+// last -- and writes
+//   mu[d]   = sum_i alpha_id / M (FP32; 0 for padding dims),
+//   amax    = max_{i,d} |fl(alpha_id - mu_d)| as FP32 bits, from the column
+//             extremes: fl(x - mu) is monotone in x and RN is sign-symmetric, so
+//             max(fl(max_d - mu_d), fl(mu_d - min_d)) is that maximum exactly,
+//   wstat   = {bits of max |W_i|, any W_i < 0 or NaN}.
+// For K <= 256 the 256 threads form rpp = 256/K row lanes x K dims (coalesced
+// reads); the rpp lane partials of a dim are combined in lane order.  For
+// K > 256 thread t owns dims t, t+256, ...  The final reduction uses the same
+// thread layout over the block partials.
+__global__ void source_stats_kernel(const float* __restrict__ alpha, const float* __restrict__ W, int64_t M, int K,
+                                    int k_pad, int nparts, double* __restrict__ part, float* __restrict__ pmm,
+                                    unsigned* __restrict__ pw, unsigned* __restrict__ counter,
+                                    float* __restrict__ mu, unsigned* __restrict__ amax,
+                                    unsigned* __restrict__ wstat) {
   __shared__ double red[256];
+  __shared__ float rmn[256], rmx[256];
+  __shared__ unsigned s_w[2], s_amax;
+  __shared__ bool s_last;
   const int b = blockIdx.x;
   const int t = threadIdx.x;
   const int64_t chunk = (M + nparts - 1) / nparts;
-  const int64_t r0 = b * chunk;
+  const int64_t r0 = b * chunk < M ? b * chunk : M;
   const int64_t r1 = (r0 + chunk < M) ? r0 + chunk : M;
+  if (t == 0) {
+    s_w[0] = 0u;
+    s_w[1] = 0u;
+    s_amax = 0u;
+  }
   if (K <= 256) {
     const int rpp = 256 / K;
     const int ro = t / K, d = t % K;
     double s = 0.0;
+    float mn = INFINITY, mx = -INFINITY;
     if (ro < rpp)
-      for (int64_t r = r0 + ro; r < r1; r += rpp) s += (double)alpha[r * K + d];
+#pragma unroll 8
+      for (int64_t r = r0 + ro; r < r1; r += rpp) {
+        const float x = alpha[r * K + d];
+        s += (double)x;
+        mn = fminf(mn, x);
+        mx = fmaxf(mx, x);
+      }
     red[t] = s;
+    rmn[t] = mn;
+    rmx[t] = mx;
     __syncthreads();
     if (t < K) {
       double acc = 0.0;
-      for (int q = 0; q < rpp; ++q) acc += red[q * K + t];
+      for (int q = 0; q < rpp; ++q) {
+        acc += red[q * K + t];
+        mn = fminf(mn, rmn[q * K + t]);
+        mx = fmaxf(mx, rmx[q * K + t]);
+      }
       part[(int64_t)b * K + t] = acc;
+      pmm[((int64_t)b * K + t) * 2] = mn;
+      pmm[((int64_t)b * K + t) * 2 + 1] = mx;
     }
   } else {
     for (int d = t; d < K; d += blockDim.x) {
       double s = 0.0;
-      for (int64_t r = r0; r < r1; ++r) s += (double)alpha[r * K + d];
+      float mn = INFINITY, mx = -INFINITY;
+#pragma unroll 8
+      for (int64_t r = r0; r < r1; ++r) {
+        const float x = alpha[r * K + d];
+        s += (double)x;
+        mn = fminf(mn, x);
+        mx = fmaxf(mx, x);
+      }
       part[(int64_t)b * K + d] = s;
+      pmm[((int64_t)b * K + d) * 2] = mn;
+      pmm[((int64_t)b * K + d) * 2 + 1] = mx;
     }
   }
-}
-
-// One warp per dimension: lanes sum the block partials in a fixed strided
-// order, then a fixed shuffle tree (deterministic).
-__global__ void source_mean_final_kernel(const double* __restrict__ part, int nparts, int64_t M, int K,
-                                         int k_pad, float* __restrict__ mu) {
-  const int d = (int)(((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
-  const int lane = threadIdx.x & 31;
-  if (d >= k_pad) return;
-  double s = 0.0;
-  if (d < K)
-    for (int b = lane; b < nparts; b += 32) s += part[(int64_t)b * K + d];
+  if (wstat != nullptr) {  // R = 1 weight statistics of the same rows
+    float m = 0.f;
+    unsigned neg = 0u;
+#pragma unroll 4
+    for (int64_t r = r0 + t; r < r1; r += blockDim.x) {
+      const float w = W[r];
+      m = fmaxf(m, fabsf(w));
+      neg |= (w < 0.f || w != w) ? 1u : 0u;  // NaN weights take the general path
+    }
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) s += __shfl_down_sync(0xffffffffu, s, o);
-  if (lane == 0) mu[d] = (d < K && M > 0) ? (float)(s / (double)M) : 0.f;
+    for (int o = 16; o > 0; o >>= 1) {
+      m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+      neg |= __shfl_xor_sync(0xffffffffu, neg, o);
+    }
+    __syncthreads();  // s_w initialised
+    if ((t & 31) == 0) {
+      atomicMax(&s_w[0], __float_as_uint(m));
+      atomicOr(&s_w[1], neg);
+    }
+  }
+  __syncthreads();
+  if (wstat != nullptr && t == 0) {
+    pw[2 * b] = s_w[0];
+    pw[2 * b + 1] = s_w[1];
+  }
+  // publish the partials, then elect the last block
+  __threadfence();
+  __syncthreads();
+  if (t == 0) s_last = atomicAdd(counter, 1u) == (unsigned)(nparts - 1);
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  // fixed-order reduction of the block partials, all threads busy: for K <= 256,
+  // rpp threads per dim stride over the blocks (loads unrolled), then thread d
+  // combines its dim's rpp partials in order; for K > 256 a thread per dim
+  for (int d0 = 0; d0 < K; d0 += 256) {
+    const int kk = K - d0 < 256 ? K - d0 : 256;  // dims in this pass
+    const int rpp = 256 / kk;
+    const int ro = t / kk, d = d0 + t % kk;
+    double s = 0.0;
+    float mn = INFINITY, mx = -INFINITY;
+    if (ro < rpp)
+#pragma unroll 8
+      for (int q = ro; q < nparts; q += rpp) {
+        s += __ldcg(&part[(int64_t)q * K + d]);
+        const float2 m2 = __ldcg(reinterpret_cast<const float2*>(&pmm[((int64_t)q * K + d) * 2]));
+        mn = fminf(mn, m2.x);
+        mx = fmaxf(mx, m2.y);
+      }
+    __syncthreads();  // red/rmn/rmx free
+    red[t] = s;
+    rmn[t] = mn;
+    rmx[t] = mx;
+    __syncthreads();
+    if (t < kk) {
+      double acc = 0.0;
+      for (int q = 0; q < rpp; ++q) {
+        acc += red[q * kk + t];
+        mn = fminf(mn, rmn[q * kk + t]);
+        mx = fmaxf(mx, rmx[q * kk + t]);
+      }
+      const float m = M > 0 ? (float)(acc / (double)M) : 0.f;
+      mu[d0 + t] = m;
+      if (M > 0) {
+        // NaN coordinates give a NaN mean; fmaxf(NaN, 0) = 0 then ignores them
+        const float a = fmaxf(fmaxf(mx - m, m - mn), 0.f);
+        atomicMax(&s_amax, __float_as_uint(a));
+      }
+    }
+  }
+  for (int d = K + t; d < k_pad; d += blockDim.x) mu[d] = 0.f;
+  if (wstat != nullptr && t < 32) {
+    unsigned m = 0u, neg = 0u;
+    for (int q = t; q < nparts; q += 32) {
+      m = max(m, __ldcg(&pw[2 * q]));
+      neg |= __ldcg(&pw[2 * q + 1]);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      m = max(m, __shfl_xor_sync(0xffffffffu, m, o));
+      neg |= __shfl_xor_sync(0xffffffffu, neg, o);
+    }
+    if (t == 0) {
+      wstat[0] = m;  // non-negative FP32 values order as their bit patterns
+      wstat[1] = neg;
+    }
+  }
+  __syncthreads();
+  if (t == 0) {
+    if (amax != nullptr) *amax = s_amax;
+    *counter = 0u;  // ready for the next call (stream order)
+  }
 }
 
-cudaError_t launch_source_mean(const float* alpha, int64_t M, int K, int k_pad, double* part, int nparts,
-                               float* mu, cudaStream_t st) {
-  if (M > 0) {
-    source_mean_partial_kernel<<<nparts, 256, 0, st>>>(alpha, M, K, nparts, part);
-  }
-  const int warps_per_block = 8;
-  source_mean_final_kernel<<<(k_pad + warps_per_block - 1) / warps_per_block, 32 * warps_per_block, 0, st>>>(
-      part, M > 0 ? nparts : 0, M, K, k_pad, mu);
+cudaError_t launch_source_stats(const float* alpha, const float* W, int64_t M, int K, int k_pad, int nparts,
+                                double* part, float* pmm, unsigned* pw, unsigned* counter, float* mu,
+                                unsigned* amax, unsigned* wstat, cudaStream_t st) {
+  source_stats_kernel<<<nparts, 256, 0, st>>>(alpha, W, M, K, k_pad, nparts, part, pmm, pw, counter, mu, amax,
+                                              wstat);
   return cudaGetLastError();
 }
 
