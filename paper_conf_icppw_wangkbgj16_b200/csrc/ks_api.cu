@@ -135,7 +135,8 @@ struct ks_ctx {
   DBuf<double> mean_part; // [nparts][K]
   DBuf<float> mean_pmm;   // [nparts][K][2] column min/max
   DBuf<unsigned> mean_pw; // [nparts][2] weight statistics
-  DBuf<unsigned> stats_counter;  // arrival counter of the statistics kernel (left zero)
+  DBuf<unsigned> stats_counter;  // arrival counter of the statistics kernels (left zero)
+  DBuf<unsigned> wcol, wcol_part; // FP16 V-MMA: per-column max |W| bits [r_pad], block partials
   CUtensorMap tmap_src;
 
   // eval scratch
@@ -330,6 +331,23 @@ ks_status encode_wt(CUtensorMap* map, const float* base, int64_t m_pad, int r_pa
   return KS_OK;
 }
 
+// wcat [2 r_pad][m_pad] FP16 viewed as {32 sources, 2 r_pad rows, m_pad/32 chunks}: one box =
+// 4 chunks x 2 r_c rows x 64 B = the K-major SWIZZLE_64B B operand ([W_hi | W_lo] rows) of the
+// FP16 V-MMA for one 128-source tile.
+ks_status encode_wcat(CUtensorMap* map, const void* base, int64_t m_pad, int r_pad, int r_c) {
+  PFN_encodeTiled enc = get_encode();
+  if (!enc) return fail(KS_ECUDA, "cuTensorMapEncodeTiled unavailable from the driver");
+  cuuint64_t dims[3] = {32, (cuuint64_t)(2 * r_pad), (cuuint64_t)(m_pad / 32)};
+  cuuint64_t strides[2] = {(cuuint64_t)m_pad * 2, 64};
+  cuuint32_t box[3] = {32, (cuuint32_t)(2 * r_c), (cuuint32_t)(ks::kTcTileS / 32)};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 3, const_cast<void*>(base), dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(KS_ECUDA, "cuTensorMapEncodeTiled (wcat 3D) failed (CUresult %d)", (int)r);
+  return KS_OK;
+}
+
 // Fold the norms into the MMA (two extra K columns) when that costs no extra K chunk.
 // KS_TC_AUG=0/1 overrides (measurement knob).
 int tc_aug(int K) {
@@ -372,10 +390,21 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(source_stats(ctx, alpha, W, use_wstat, M, k_pad, f16), "source statistics");
   const unsigned* wst = use_wstat ? ctx->wstat.p : nullptr;
   if (f16) {
-    KS_CUDA(ks::launch_prep_f16_sources(alpha, W, M, m_pad, K, k_pad, R, vcc ? 0 : r_pad, ctx->mu.p, ctx->c,
+    KS_CUDA(ks::launch_prep_f16_sources(alpha, W, M, m_pad, K, k_pad, R, 0, ctx->mu.p, ctx->c,
                                         ctx->amax.p, fold, ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p,
                                         ctx->wt_lo.p, ctx->wv.p, vcc, wst, st),
             "source prep (TC, FP16)");
+    if (vcc == 0) {  // weighted sum on the tensor cores in FP16 (reading Q27): wcat in the W hi buffer
+      int np = (int)((M + 1023) / 1024);
+      if (np < 1) np = 1;
+      if (np > 256) np = 256;
+      KS_CUDA(ctx->wcol.reserve((size_t)r_pad, st, true), "allocate W column scales");
+      KS_CUDA(ctx->wcol_part.reserve((size_t)np * R, st, false), "allocate W column partials");
+      KS_CUDA(ks::launch_prep_wcat(W, M, m_pad, R, r_pad, np, ctx->wcol_part.p, ctx->stats_counter.p, ctx->wcol.p,
+                                   ctx->wt_hi.p, st),
+              "weight prep (FP16 V-MMA)");
+      ctx->launches += (M > 0) ? 2 : 1;
+    }
   } else {
     KS_CUDA(ks::launch_prep_tc_sources(alpha, W, M, m_pad, K, k_pad, R, vcc ? 0 : r_pad, ctx->mu.p, ctx->c, aug,
                                        ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p, ctx->wt_lo.p,
@@ -454,6 +483,7 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.c = ctx->c;
   a.K = ctx->K;
   a.wv = ctx->wv.p;
+  a.wcol = ctx->wcol.p;
   a.vcc = ctx->tc_vcc;
   {
     const char* e = getenv("KS_TC_ARES");  // measurement knob: 0 = reload the target operand per unit
@@ -488,10 +518,16 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
     a.r_c = r_c;
     a.r_off = r_off;
     a.r_valid = (ctx->R - r_off < r_c) ? (ctx->R - r_off) : r_c;
-    s = encode_wt(&maps[4], ctx->wt_hi.p, ctx->m_pad, ctx->r_pad, r_c);
-    if (s != KS_OK) return s;
-    s = encode_wt(&maps[5], ctx->wt_lo.p, ctx->m_pad, ctx->r_pad, r_c);
-    if (s != KS_OK) return s;
+    if (f16) {  // FP16 V-MMA: one wcat map (hi and lo rows of the r_c columns in one box)
+      s = encode_wcat(&maps[4], ctx->wt_hi.p, ctx->m_pad, ctx->r_pad, r_c);
+      if (s != KS_OK) return s;
+      maps[5] = maps[4];
+    } else {
+      s = encode_wt(&maps[4], ctx->wt_hi.p, ctx->m_pad, ctx->r_pad, r_c);
+      if (s != KS_OK) return s;
+      s = encode_wt(&maps[5], ctx->wt_lo.p, ctx->m_pad, ctx->r_pad, r_c);
+      if (s != KS_OK) return s;
+    }
     cudaEvent_t stop;
     s = timed_begin(ctx, &stop);
     if (s != KS_OK) return s;
@@ -585,6 +621,8 @@ ks_status ks_destroy(ks_ctx* ctx) {
   ctx->mean_part.release();
   ctx->mean_pmm.release();
   ctx->mean_pw.release();
+  ctx->wcol.release();
+  ctx->wcol_part.release();
   ctx->stats_counter.release();
   ctx->partial.release();
   ctx->counters.release();

@@ -55,12 +55,16 @@ struct TcSmemT {
   static constexpr uint32_t kStage0 = 0;
   static constexpr uint32_t kA0 = kStages * kStageBytes;
   static constexpr uint32_t wslot(int r_c) { return (uint32_t)r_c * 512u; }  // one of W^T hi/lo: 8 chunks x r_c x 64 B
-  static constexpr uint32_t kW0 = kA0 + (AR ? 8 * kChunkA : 0u);
-  // VCC: na[TS] | W[TS][RV];  else W^T hi | W^T lo | na[128].  Slots 1 KB aligned (SWIZZLE_64B atoms).
+  // AR: VCC (R = 1) two target-operand buffers of <= 4 planes; !VCC (FP16 V-MMA, K <= 256) one
+  // buffer of all 8 chunks' hi and lo planes (128 KB)
+  static constexpr uint32_t kW0 = kA0 + (AR ? (VCC ? 8u : 16u) * kChunkA : 0u);
+  // VCC: na[TS] | W[TS][RV];  AR (FP16 V-MMA): wcat | na[128];  else W^T hi | W^T lo | na[128].
+  // Slots 1 KB aligned (SWIZZLE_64B atoms).
   static constexpr uint32_t w_slot_bytes(int r_c) {
-    return VCC ? ((uint32_t)(4 * TS * (1 + RV)) + 1023u) & ~1023u : (2 * wslot(r_c) + 512 + 1023) & ~1023u;
+    return VCC ? ((uint32_t)(4 * TS * (1 + RV)) + 1023u) & ~1023u
+               : ((AR ? 1u : 2u) * wslot(r_c) + 512 + 1023) & ~1023u;
   }
-  static constexpr uint32_t na_off(int r_c) { return VCC ? 0u : 2 * wslot(r_c); }
+  static constexpr uint32_t na_off(int r_c) { return VCC ? 0u : (AR ? 1u : 2u) * wslot(r_c); }
   static constexpr int kWSlots = VCC && RV < 8 ? 4 : 2;  // W/na ring depth (RV >= 8: 2 to fit 4 stages)
   static constexpr uint32_t bar_off(int r_c) { return kW0 + kWSlots * w_slot_bytes(r_c); }
   static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 512 + 4 * kTcTileT * 8; }  // + VCC scratch
@@ -136,6 +140,23 @@ __device__ __forceinline__ void split3_f16(double x, __half* p) {
 }
 constexpr double kFoldFar = 16384.0;   // c ||beta_hat_j||^2 above this: every kernel value of row j is < 2^-4096
 constexpr float kFoldNegInf = -32768.f;  // stands for -inf in FP16 operands (no inf * 0 in the MMA)
+
+// ---- FP16 V-MMA (split-FP16 mode, tensor-core weighted sum; reading Q27 in DESIGN.md).
+// P is written back into its own S columns as FP16 pairs: per 16-source K step, 8 columns
+// of hi pairs then 8 columns of lo pairs of P 2^kPExp (t + kPExp into the ex2, so P 2^kPExp
+// <= 2^14 < FP16 max).  Weights: column r scaled by 2^s_r, s_r = wcol_exp(max_i |W_ir|)
+// (max in [2^14, 2^15)), split hi/lo, rows of wcat [2 r_pad][m_pad] grouped by 16 columns:
+// row 32g + u = hi of column 16g + u, row 32g + 16 + u = lo.  Per K step one MMA
+// P_hi [W_hi | W_lo] (N = 2 r_c) and, per group, P_lo W_hi (N = 16) into the hi.hi columns;
+// the epilogue reads V_hh + V_hl and scales by 2^-(kPExp + s_r) in FP64 (exact).
+constexpr int kPExp = 14;
+__device__ __forceinline__ int wcol_exp(unsigned bits) {
+  const float m = __uint_as_float(bits);
+  if (!(m > 0.f) || !(m <= 3.0e38f)) return 0;
+  int e;
+  frexpf(m, &e);  // m = f 2^e, f in [0.5, 1)
+  return 15 - e;
+}
 
 __device__ __forceinline__ int64_t sk_start(int64_t b, int64_t U, int64_t G) { return (b * U) / G; }
 __device__ __forceinline__ int64_t sk_owner(int64_t u, int64_t U, int64_t G) { return ((u + 1) * G - 1) / U; }
@@ -295,7 +316,59 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   tc_fence_after();
   const uint32_t tbase = *tmem_base_smem;
 
-  if (AR && warp == 0) {
+  if (!VCC && AR && warp == 0) {
+    // ================= TMA producer, FP16 V-MMA kernel with the target operand resident (K <= 256):
+    // the target tile's hi/lo planes of every chunk once per target tile into the one A buffer
+    // (after the MMAs of the previous target tile are done with it), source chunks into the ring
+    const bool leader = elect_one();
+    if (leader) {
+      tma_prefetch_desc(&mA_hi);
+      tma_prefetch_desc(&mB_hi);
+    }
+    const int kcw = 2 * kTcKC;  // FP16 elements per 64-byte chunk
+    int it = 0, seg = -1;
+    int64_t cur_tt = -1;
+    UnitIt cu = unit_begin(sc);
+    for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
+      const int tt = (int)cu.tt, st = cu.st;
+      if (cu.tt != cur_tt) {
+        ++seg;
+        cur_tt = cu.tt;
+        if (seg > 0) mbar_wait(&aempty[0], (uint32_t)((seg - 1) & 1));
+        uint8_t* ap = smem + TcSmem::kA0;
+        if (leader && dbg_noload) {
+          mbar_arrive(&afull[0]);
+        } else if (leader) {
+          uint32_t bytes = 0;
+          for (int kc = 0; kc < n_kc; ++kc) bytes += (kc * kcw < args.kdims) ? 2 * kChunkA : kChunkA;
+          mbar_arrive_expect_tx(&afull[0], bytes);
+          for (int kc = 0; kc < n_kc; ++kc) {
+            tma_load_2d(ap + 2 * kc * kChunkA, &mA_hi, kc * kcw, tt * kTcTileT, &afull[0]);
+            if (kc * kcw < args.kdims) tma_load_2d(ap + (2 * kc + 1) * kChunkA, &mA_lo, kc * kcw, tt * kTcTileT, &afull[0]);
+          }
+        }
+        __syncwarp();
+      }
+      for (int kc = 0; kc < n_kc; ++kc, ++it) {
+        const int s = it % kStages;
+        const uint32_t use = (uint32_t)(it / kStages);
+        PROF_BEGIN(w0);
+        mbar_wait(&empty[s], (use & 1) ^ 1);
+        PROF_END(0, w0);
+        uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
+        if (leader && dbg_noload) {
+          mbar_arrive(&full[s]);
+        } else if (leader) {
+          const int k0 = kc * kcw;
+          const bool lo = k0 < args.kdims;
+          mbar_arrive_expect_tx(&full[s], lo ? 2 * kChunkB : kChunkB);
+          tma_load_2d(sp, &mB_hi, k0, st * TS, &full[s]);
+          if (lo) tma_load_2d(sp + kChunkB, &mB_lo, k0, st * TS, &full[s]);
+        }
+        __syncwarp();
+      }
+    }
+  } else if (AR && warp == 0) {
     // ================= TMA producer, resident-target kernel: the target tile's operand once per
     // target tile (buffer seg & 1), the source tile's planes as one stage per unit
     const bool leader = elect_one();
@@ -408,6 +481,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           mbar_arrive_expect_tx(&wfull[slot], 4 * TS * (1 + RV));
           bulk_load(ws, args.na + (int64_t)st * TS, 4 * TS, &wfull[slot]);
           bulk_load(ws + 4 * TS, args.wv + (int64_t)st * TS * RV, 4 * TS * RV, &wfull[slot]);
+        } else if (args.f16) {  // FP16 V-MMA: the wcat tile [4 chunks][2 r_c rows][32 sources] (one plane)
+          mbar_arrive_expect_tx(&wfull[slot], TcSmem::wslot(RC) + 512);
+          tma_load_3d(ws, &mW_hi, 0, 2 * args.r_off, st * (kTcTileS / 32), &wfull[slot]);
+          bulk_load(ws + TcSmem::na_off(RC), args.na + (int64_t)st * kTcTileS, 512, &wfull[slot]);
         } else {
           mbar_arrive_expect_tx(&wfull[slot], 2 * TcSmem::wslot(RC) + 512);
           tma_load_3d(ws, &mW_hi, 0, args.r_off, st * (kTcTileS / 16), &wfull[slot]);
@@ -442,8 +519,27 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       const uint32_t colP = (bp ? kColS1 : kColS0) + 64 * hh;
       const uint32_t colL = kColPlo + 64 * hh;
       bool acc = !first;
+      if (args.f16) {
+        // FP16 V-MMA, P in place (hi pairs at colP + 16 ks, lo pairs 8 columns on):
+        // P_hi [W_hi | W_lo] (N = 2 r_c), then P_lo W_hi per group of 16 columns (N = 16)
+        const uint32_t idV2 = idesc_f16(128, 2 * RC), idV1 = idesc_f16(128, 16);
+        const uint64_t bw0 = sdesc_k_sw64(ws);
+#pragma unroll
+        for (int ks = 0; ks < 4; ++ks) {
+          const int kk = 4 * hh + ks;  // K step (16 sources) within the tile
+          const uint64_t bd = bw0 + (uint64_t)(((kk >> 1) * (2 * RC * 64) + (kk & 1) * 32) >> 4);
+          const uint32_t aHi = tbase + colP + 16 * ks;
+          if (leader && !skip_v) {
+            mma_f16_ts(tbase + kColV, aHi, bd, idV2, acc ? 1u : 0u);
+#pragma unroll
+            for (int g = 0; g < RC / 16; ++g)
+              mma_f16_ts(tbase + kColV + 32 * g, aHi + 8, bd + (uint64_t)((g * 32 * 64) >> 4), idV1, 1u);
+          }
+          acc = true;
+        }
+      }
       // products: P_lo.W_hi, P_hi.W_lo, P_hi.W_hi (small terms first)
-      for (int pr = 3 - nprod; pr < 3 && !skip_v; ++pr) {
+      for (int pr = 3 - nprod; pr < 3 && !skip_v && !args.f16; ++pr) {
         const uint32_t aCol = (pr == 0) ? colL : colP;
         const uint64_t bd0 = sdesc_k_sw64(ws + ((pr == 1) ? TcSmem::wslot(RC) : 0u));
 #pragma unroll
@@ -536,9 +632,22 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     } else {
     UnitIt cu = unit_begin(sc);
     int prev_st = 0;
+    int seg = -1;  // AR (FP16 V-MMA, resident target operand): target tile index
+    int64_t cur_tt = -1;
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
       const int bq = q & 1;
       const uint32_t dS = tbase + (bq ? (uint32_t)TS : 0u);
+      if constexpr (AR && !VCC) {
+        if (cu.tt != cur_tt) {  // new target tile: release the A buffer, wait for the new operand
+          if (seg >= 0) {
+            if (leader) tc_commit(&aempty[0]);
+            __syncwarp();
+          }
+          ++seg;
+          cur_tt = cu.tt;
+          mbar_wait(&afull[0], (uint32_t)(seg & 1));
+        }
+      }
       if constexpr (VCC) {
         if (q >= 2) {  // the epilogue has read S(q-2) out of this buffer
           PROF_BEGIN(w1);
@@ -556,8 +665,18 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         PROF_BEGIN(w2);
         tc_fence_after();
         uint8_t* sp = smem + TcSmem::kStage0 + s * kStageBytes;
-        const uint64_t dAh = sdesc_k_sw64(sp), dAl = sdesc_k_sw64(sp + kChunkA);
-        const uint64_t dBh = sdesc_k_sw64(sp + 2 * kChunkA), dBl = sdesc_k_sw64(sp + 2 * kChunkA + kChunkB);
+        uint64_t dAh, dAl, dBh, dBl;
+        if constexpr (AR && !VCC) {  // A resident (chunk kc: hi, lo planes), B hi | lo per stage
+          dAh = sdesc_k_sw64(smem + TcSmem::kA0 + 2 * kc * kChunkA);
+          dAl = sdesc_k_sw64(smem + TcSmem::kA0 + (2 * kc + 1) * kChunkA);
+          dBh = sdesc_k_sw64(sp);
+          dBl = sdesc_k_sw64(sp + kChunkB);
+        } else {
+          dAh = sdesc_k_sw64(sp);
+          dAl = sdesc_k_sw64(sp + kChunkA);
+          dBh = sdesc_k_sw64(sp + 2 * kChunkA);
+          dBl = sdesc_k_sw64(sp + 2 * kChunkA + kChunkB);
+        }
 #pragma unroll
         for (int ks = 0; ks < kTcKC / 8; ++ks) {
           const uint64_t aH = dAh + (uint64_t)((ks * 32) >> 4);
@@ -935,6 +1054,14 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     double vacc[HC];
 #pragma unroll
     for (int r = 0; r < HC; ++r) vacc[r] = 0.0;
+    // FP16 V-MMA: this thread's V columns r are the TMEM columns 32 (r / 16) + r % 16 (hi.hi
+    // + lo.hi) and 16 further (hi.lo); unscaled by 2^-(kPExp + s_r) when collected
+    const uint32_t vcol = args.f16 ? 32u * (uint32_t)(rbase / 16) + (uint32_t)(rbase % 16) : (uint32_t)rbase;
+    double vsc[HC];
+#pragma unroll
+    for (int r = 0; r < HC; ++r)
+      vsc[r] = (args.f16 && rbase + r < args.r_valid) ? ldexp(1.0, -(kPExp + wcol_exp(args.wcol[args.r_off + rbase + r])))
+                                                      : 1.0;
     float nbj = 0.f, rjs = 1.f;
     int seg_q = 0;                        // first local unit of the current segment
     int seg_st0 = 0;                      // its source tile
@@ -943,7 +1070,15 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     // of a segment write V / partial.
     auto v_collect = [&](int p, int64_t tt, int spp) {
       const bool seg_end = (p == count - 1) || (spp + 1 == n_s);
-      {
+      if (args.f16) {
+        uint32_t v[HC], w[HC];
+        tmem_ldn<HC>(tbase + lane_off + kColV + vcol, v);
+        tmem_ldn<HC>(tbase + lane_off + kColV + vcol + 16, w);
+        tmem_wait_ld();
+#pragma unroll
+        for (int r = 0; r < HC; ++r)
+          vacc[r] += ((double)__uint_as_float(v[r]) + (double)__uint_as_float(w[r])) * vsc[r];
+      } else {
         uint32_t v[HC];
         tmem_ldn<HC>(tbase + lane_off + kColV + rbase, v);
         tmem_wait_ld();
@@ -1027,6 +1162,48 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC) +
                                                        TcSmem::na_off(RC));
       const uint32_t colS = bq ? kColS1 : kColS0;
+      if (args.f16) {
+        // FP16 V-MMA: P 2^kPExp split into FP16 hi/lo pairs, written back over this warp's 16 S
+        // columns of each source half (one K step of the V-MMA): words 0..7 hi of sources
+        // (2w, 2w+1), 8..15 lo.  Both halves loaded at once; half 1 is computed while half 0's
+        // store is in flight, one wait::st for both.
+        static_assert(CB == 16, "one 16-source K step per warp and half");
+        uint32_t sv0[CB], sv1[CB];
+        tmem_ldn<CB>(tbase + lane_off + colS + CB * h, sv0);
+        tmem_ldn<CB>(tbase + lane_off + colS + 64 + CB * h, sv1);
+        tmem_wait_ld();
+        auto p_pairs = [&](const uint32_t(&sv)[CB], int c0, uint32_t(&pw)[16]) {
+#pragma unroll
+          for (int i = 0; i < CB; i += 4) {
+            const float4 na4 = *reinterpret_cast<const float4*>(nas + c0 + i);
+            const float nav[4] = {na4.x + nbj, na4.y + nbj, na4.z + nbj, na4.w + nbj};
+            float p[4];
+#pragma unroll
+            for (int e = 0; e < 4; ++e)  // clamp d^2 >= 0, then the 2^kPExp scale
+              p[e] = ex2_approx(fminf(fmaf(__uint_as_float(sv[i + e]), rjs, nav[e]), 0.f) + (float)kPExp);
+#pragma unroll
+            for (int u = 0; u < 2; ++u) {
+              const __half2 hv = __floats2half2_rn(p[2 * u], p[2 * u + 1]);
+              const float2 hf = __half22float2(hv);
+              const __half2 lv = __floats2half2_rn(p[2 * u] - hf.x, p[2 * u + 1] - hf.y);  // exact remainders
+              pw[(i >> 1) + u] = *reinterpret_cast<const uint32_t*>(&hv);
+              pw[8 + (i >> 1) + u] = *reinterpret_cast<const uint32_t*>(&lv);
+            }
+          }
+        };
+        uint32_t pw0[16], pw1[16];
+        p_pairs(sv0, CB * h, pw0);
+        tmem_stn<16>(tbase + lane_off + colS + CB * h, pw0);
+        p_pairs(sv1, 64 + CB * h, pw1);
+        tmem_stn<16>(tbase + lane_off + colS + 64 + CB * h, pw1);
+        tmem_wait_st();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) {
+          mbar_arrive(&pready[bq * 2 + 0]);
+          mbar_arrive(&pready[bq * 2 + 1]);
+        }
+      } else {
 #pragma unroll 1
       for (int hh = 0; hh < 2; ++hh) {
         if (q > 0) {  // V(q-1, hh) has consumed this source half's P_lo buffer
@@ -1059,6 +1236,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         __syncwarp();
         if (lane == 0) mbar_arrive(&pready[bq * 2 + hh]);
       }
+      }  // TF32 V-MMA
       prev_tt = cu.tt;
       prev_st = cu.st;
     }
@@ -1294,6 +1472,68 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
   }
 }
 
+// FP16 V-MMA weights (reading Q27): per-column max |W_ir| (block partials, fixed-order
+// last-block reduction; NaN ignored), then wcat = FP16 hi/lo of W_ir 2^s_r in the
+// grouped row layout the V-MMA B operand reads (zero for padding rows/sources).
+__global__ void weight_colmax_kernel(const float* __restrict__ W, int64_t M, int R, int nparts,
+                                     unsigned* __restrict__ pcol, unsigned* __restrict__ counter,
+                                     unsigned* __restrict__ wcol) {
+  __shared__ unsigned cm[256];
+  __shared__ bool s_last;
+  const int t = threadIdx.x, b = blockIdx.x;
+  for (int c = t; c < R; c += blockDim.x) cm[c] = 0u;
+  __syncthreads();
+  const int64_t chunk = (M + nparts - 1) / nparts;
+  const int64_t r0 = b * chunk < M ? b * chunk : M;
+  const int64_t r1 = r0 + chunk < M ? r0 + chunk : M;
+  for (int64_t e = r0 * R + t; e < r1 * R; e += blockDim.x) {
+    const float w = fabsf(W[e]);
+    if (w == w) atomicMax(&cm[e % R], __float_as_uint(w));
+  }
+  __syncthreads();
+  for (int c = t; c < R; c += blockDim.x) pcol[(int64_t)b * R + c] = cm[c];
+  __threadfence();
+  __syncthreads();
+  if (t == 0) s_last = atomicAdd(counter, 1u) == (unsigned)(nparts - 1);
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  for (int c = t; c < R; c += blockDim.x) {
+    unsigned m = 0u;
+    for (int q = 0; q < nparts; ++q) m = max(m, __ldcg(&pcol[(int64_t)q * R + c]));
+    wcol[c] = m;
+  }
+  if (t == 0) *counter = 0u;
+}
+
+__global__ void prep_wcat_kernel(const float* __restrict__ W, int64_t M, int64_t m_pad, int R, int r_pad,
+                                 const unsigned* __restrict__ wcol, __half* __restrict__ wcat) {
+  const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;  // sources fastest
+  if (e >= (int64_t)r_pad * m_pad) return;
+  const int r = (int)(e / m_pad);
+  const int64_t i = e - (int64_t)r * m_pad;
+  const float w = (i < M && r < R) ? ldexpf(W[i * R + r], wcol_exp(wcol[r])) : 0.f;  // exact power-of-2 scaling
+  __half hi, lo;
+  split_f16(w, hi, lo);
+  const int64_t row = 32 * (r >> 4) + (r & 15);
+  wcat[row * m_pad + i] = hi;
+  wcat[(row + 16) * m_pad + i] = lo;
+}
+
+cudaError_t launch_prep_wcat(const float* W, int64_t M, int64_t m_pad, int R, int r_pad, int nparts, unsigned* pcol,
+                             unsigned* counter, unsigned* wcol, void* wcat, cudaStream_t st) {
+  if (M > 0) {
+    weight_colmax_kernel<<<nparts, 256, 0, st>>>(W, M, R, nparts, pcol, counter, wcol);
+  } else {
+    cudaError_t e = cudaMemsetAsync(wcol, 0, sizeof(unsigned) * R, st);
+    if (e != cudaSuccess) return e;
+  }
+  const int64_t n = (int64_t)r_pad * m_pad;
+  prep_wcat_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(W, M, m_pad, R, r_pad, wcol,
+                                                                 static_cast<__half*>(wcat));
+  return cudaGetLastError();
+}
+
 template <bool F16>
 static cudaError_t launch_prep_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K,
                                        int k_pad, int R, int r_pad, const float* mu, double c, int aug,
@@ -1433,6 +1673,12 @@ cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream
     case 8: return launch_rcsv<16, 4, 8>(maps, a, st);
     case 16: return launch_rcsv<16, 3, 16>(maps, a, st);
     default: break;
+  }
+  // FP16 V-MMA with the target operand resident (K <= 256; KS_TC_ARES=0 reloads it per unit):
+  // 4 source stages fit beside the 128 KB operand at r_c = 16, 3 at r_c = 32
+  if (a.f16 && a.ares && a.k_pad <= 8 * kTcKC) {
+    if (a.r_c == 16) return launch_rcsv<16, 4, 0, 32>(maps, a, st);
+    if (a.r_c == 32) return launch_rcsv<32, 3, 0, 32>(maps, a, st);
   }
   const int ns = tc_stages(a.r_c);
   if (a.r_c == 16) {

@@ -90,6 +90,7 @@ struct TcArgs {
   int K;
   int vcc;              // RV > 0: weighted sum on CUDA cores over RV padded columns (no W^T tiles, no V MMA)
   const float* wv;      // [m_pad][RV] weights, zero padded (vcc)
+  const unsigned* wcol; // FP16 V-MMA (f16, !vcc): [r_pad] FP32 bits of max_i |W_ir| (column scale exponents)
   int wslots;           // VCC W/na ring depth (2..4; 0 = default)
   int ares;             // R = 1, <= 2 operand chunks: target operand resident per target tile (no reload per unit)
   int dbg_skip_v;       // measurement only (KS_TC_DEBUG_SKIP_V=1): do not issue the V MMAs (wrong results)
@@ -134,6 +135,11 @@ cudaError_t launch_prep_f16_sources(const float* alpha, const float* W, int64_t 
 cudaError_t launch_prep_f16_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
                                     double c, const unsigned* amax, int fold, void* tgt_hi, void* tgt_lo, float* nb,
                                     float* tsc, cudaStream_t st);
+// FP16 V-MMA weights (f16 mode, R > RV limit or forced): wcol [R] = bits of max_i |W_ir|
+// (scratch pcol [nparts][R], counter zero before, left zero), wcat [2 r_pad][m_pad] halves
+// (row 32g + u = hi of column 16g + u scaled by 2^s_r, row 32g + 16 + u = lo).
+cudaError_t launch_prep_wcat(const float* W, int64_t M, int64_t m_pad, int R, int r_pad, int nparts, unsigned* pcol,
+                             unsigned* counter, unsigned* wcol, void* wcat, cudaStream_t st);
 // maps: A_hi, A_lo (targets), B_hi, B_lo (sources), W_hi, W_lo (weights^T)
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st);
 int fused_tc_stages();

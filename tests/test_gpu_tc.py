@@ -135,6 +135,30 @@ def test_tensor_core_v_path(oracle_mod, monkeypatch, R):
     check(oracle_mod, a, W, b, h)
 
 
+@pytest.mark.parametrize("R", [20, 48])
+def test_v_mma_column_scales(oracle_mod, R):
+    """R > 16: the weighted sum runs as a second tcgen05 MMA; in split-FP16 mode
+    W is scaled per column by a power of two into FP16 range (Q27).
+    Columns spanning 10^-30 .. 10^30, an all-zero column, a column with one
+    tiny and one huge weight, and a column with a NaN-free mix of signs must
+    each meet the per-column bar."""
+    a, W, b, h = workloads.custom(1900, 300, 96, R, 3.0, seed=R, wkind="signed")
+    W = W.astype(np.float64)
+    W *= 10.0 ** np.linspace(-30, 30, R)[None, :]
+    W[:, 1] = 0.0
+    W[:, 2] = 0.0
+    W[5, 2], W[700, 2] = 1e-20, 1e20
+    W[:, 3] = np.where(np.arange(W.shape[0]) % 7 == 0, 1e-8, 1.0) * np.sign(W[:, 3] + 1e-300)
+    W = W.astype(np.float32)
+    V, info = gpu_eval(a, W, b, h)
+    Vr = oracle_mod.oracle_eval(a, W, b, float(h))
+    col = np.abs(W.astype(np.float64)).sum(axis=0)
+    assert np.all(V[:, 1] == 0.0)
+    ok = col > 0
+    err = np.max(np.abs(V - Vr)[:, ok] / col[ok])
+    assert err <= TOL_3XTF32, f"e_norm {err:.3e}"
+
+
 @pytest.mark.parametrize("wcase", ["zeros", "all_zero", "one_negative", "tiny", "huge"])
 def test_r1_weight_modes(oracle_mod, wcase):
     """R = 1: W >= 0 takes the log-weight epilogue (log2 W_i folded into the

@@ -64,6 +64,198 @@ __global__ void __launch_bounds__(128, 1) k(float* out) {
   if (tid == 0 && out[0] == 1234.5f) out[1] = 1.f;
 }
 
+// A from TMEM (kind::f16, the V = P.W shape): D [128 x N] at column 0, A at column 256.. (8 columns
+// per K = 16 step), B = N rows x 64 bytes (SWIZZLE_64B) in shared memory.
+template <int N>
+__global__ void __launch_bounds__(128, 1) k_ts(float* out) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ uint32_t tb;
+  __shared__ __align__(8) uint64_t bar;
+  const int tid = threadIdx.x, warp = tid >> 5;
+  for (int i = tid; i < 256 * 64 / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(smem)[i] = 0u;
+  if (tid == 0) { mbar_init(&bar, 1); fence_mbar_init(); }
+  if (warp == 0) tmem_alloc(&tb, 512);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = tb;
+  if (warp == 0) {
+    const bool leader = elect_one();
+    const uint64_t dB = sdesc_sw(smem, 64);
+    const uint32_t id = idesc_f16(128, N);
+    for (int i = 0; i < NMMA; ++i) {
+      const int ks = i & 1;
+      if (leader) mma_f16_ts(tbase, tbase + 256 + 8 * (i & 15), dB + (uint64_t)((ks * 32) >> 4), id, (i & 15) ? 1u : 0u);
+      __syncwarp();
+    }
+    if (leader) tc_commit(&bar);
+    __syncwarp();
+    mbar_wait(&bar, 0);
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) tmem_dealloc(tbase, 512);
+  if (tid == 0 && out[0] == 1234.5f) out[1] = 1.f;
+}
+// One fused-kernel unit of the FP16 V-MMA path: NS ss MMAs (M=128, N=128, K=16) into S at column
+// 0, then NV A-from-TMEM MMAs (alternating N = 32 and N = 16) into V at column 384, A at 128..
+template <int NS, int NV, int RND = 0>
+__global__ void __launch_bounds__(128, 1) k_unit(float* out, int units) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ uint32_t tb;
+  __shared__ __align__(8) uint64_t bar;
+  const int tid = threadIdx.x, warp = tid >> 5;
+  for (int i = tid; i < (128 + 256) * 64 / 4; i += blockDim.x) {
+    // random FP16 pairs in (-1, 1) when RND (data-dependent tensor power), else zeros
+    uint32_t x = (uint32_t)i * 2654435761u + 12345u;
+    x ^= x >> 13; x *= 0x5bd1e995u; x ^= x >> 15;
+    reinterpret_cast<uint32_t*>(smem)[i] = RND ? ((x & 0x3BFF3BFFu) | (x & 0x80008000u)) : 0u;
+  }
+  if (tid == 0) { mbar_init(&bar, 1); fence_mbar_init(); }
+  if (warp == 0) tmem_alloc(&tb, 512);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = tb;
+  if (warp == 0) {
+    const bool leader = elect_one();
+    const uint64_t dA = sdesc_sw(smem, 64), dB = sdesc_sw(smem + 128 * 64, 64);
+    const uint32_t idS = idesc_f16(128, 128), id32 = idesc_f16(128, 32), id16 = idesc_f16(128, 16);
+    for (int u = 0; u < units; ++u) {
+      for (int i = 0; i < NS; ++i)
+        if (leader) mma_f16_ss(tbase + 128 * (u & 1), dA + (uint64_t)(((i & 1) * 32) >> 4), dB + (uint64_t)(((i & 1) * 32) >> 4), idS, i ? 1u : 0u);
+      for (int i = 0; i < NV; ++i)
+        if (leader) mma_f16_ts(tbase + 384, tbase + 128 * ((u + 1) & 1) + 8 * (i & 15), dB, (i & 1) ? id16 : id32, 1u);
+      __syncwarp();
+    }
+    if (leader) tc_commit(&bar);
+    __syncwarp();
+    mbar_wait(&bar, 0);
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) tmem_dealloc(tbase, 512);
+  if (tid == 0 && out[0] == 1234.5f) out[1] = 1.f;
+}
+// The fused kernel's S pattern: per 64-byte chunk (4 chunks of distinct planes A_hi, A_lo,
+// B_hi, B_lo, 8 KB each), 2 K steps x 3 split products lo.hi, hi.lo, hi.hi (M=128, N=128),
+// random FP16 data; NV A-from-TMEM MMAs per 8 chunks.
+template <int NV>
+__global__ void __launch_bounds__(128, 1) k_split(float* out, int units) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ uint32_t tb;
+  __shared__ __align__(8) uint64_t bar;
+  const int tid = threadIdx.x, warp = tid >> 5;
+  for (int i = tid; i < 4 * 32768 / 4; i += blockDim.x) {
+    uint32_t x = (uint32_t)i * 2654435761u + 12345u;
+    x ^= x >> 13; x *= 0x5bd1e995u; x ^= x >> 15;
+    reinterpret_cast<uint32_t*>(smem)[i] = (x & 0x3BFF3BFFu) | (x & 0x80008000u);
+  }
+  if (tid == 0) { mbar_init(&bar, 1); fence_mbar_init(); }
+  if (warp == 0) tmem_alloc(&tb, 512);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = tb;
+  if (warp == 0) {
+    const bool leader = elect_one();
+    const uint32_t idS = idesc_f16(128, 128), id32 = idesc_f16(128, 32), id16 = idesc_f16(128, 16);
+    for (int u = 0; u < units; ++u) {
+      const uint32_t d = tbase + 128 * (u & 1);
+      for (int kc = 0; kc < 8; ++kc) {
+        uint8_t* base = smem + (kc & 3) * 32768;
+        const uint64_t aH = sdesc_sw(base, 64), aL = sdesc_sw(base + 8192, 64);
+        const uint64_t bH = sdesc_sw(base + 16384, 64), bL = sdesc_sw(base + 24576, 64);
+        for (int ks = 0; ks < 2; ++ks) {
+          const uint64_t o = (uint64_t)ks * 2;
+          const uint32_t acc = (kc | ks) ? 1u : 0u;
+          if (leader) {
+            mma_f16_ss(d, aL + o, bH + o, idS, acc);
+            mma_f16_ss(d, aH + o, bL + o, idS, 1u);
+            mma_f16_ss(d, aH + o, bH + o, idS, 1u);
+          }
+        }
+      }
+      for (int i = 0; i < NV; ++i)
+        if (leader) mma_f16_ts(tbase + 384, tbase + 128 * ((u + 1) & 1) + 8 * (i & 15), sdesc_sw(smem, 64), (i & 1) ? id16 : id32, 1u);
+      __syncwarp();
+    }
+    if (leader) tc_commit(&bar);
+    __syncwarp();
+    mbar_wait(&bar, 0);
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) tmem_dealloc(tbase, 512);
+  if (tid == 0 && out[0] == 1234.5f) out[1] = 1.f;
+}
+template <int NV>
+void run_split(float* out, int G) {
+  const int smem = 4 * 32768 + 1024, units = 256;
+  cudaFuncSetAttribute(k_split<NV>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  float best = 1e9;
+  for (int r = 0; r < 5; ++r) {
+    cudaEventRecord(e0);
+    k_split<NV><<<G, 128, smem>>>(out, units);
+    cudaEventRecord(e1);
+    cudaEventSynchronize(e1);
+    float ms;
+    cudaEventElapsedTime(&ms, e0, e1);
+    if (ms < best) best = ms;
+  }
+  printf("split unit (random, 8 chunks x 6 MMAs N=128 + %d ts): %.1f cycles per unit at 1965 MHz (%.3f ms)\n", NV,
+         best * 1e-3 * 1.965e9 / units, best);
+}
+
+template <int NS, int NV, int RND = 0>
+void run_unit(float* out, int G) {
+  const int smem = (128 + 256) * 64 + 1024, units = 256;
+  cudaFuncSetAttribute(k_unit<NS, NV, RND>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  float best = 1e9;
+  for (int r = 0; r < 5; ++r) {
+    cudaEventRecord(e0);
+    k_unit<NS, NV, RND><<<G, 128, smem>>>(out, units);
+    cudaEventRecord(e1);
+    cudaEventSynchronize(e1);
+    float ms;
+    cudaEventElapsedTime(&ms, e0, e1);
+    if (ms < best) best = ms;
+  }
+  printf("unit%s: %d ss N=128 + %d ts (N=32/16): %.1f cycles per unit at 1965 MHz (ss alone ~%d)\n", RND ? " (random data)" : "", NS, NV,
+         best * 1e-3 * 1.965e9 / units, NS * 70);
+}
+
+template <int N>
+void run_ts(float* out, int G) {
+  const int smem = 256 * 64 + 1024;
+  cudaFuncSetAttribute(k_ts<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  float best = 1e9;
+  for (int r = 0; r < 5; ++r) {
+    cudaEventRecord(e0);
+    k_ts<N><<<G, 128, smem>>>(out);
+    cudaEventRecord(e1);
+    cudaEventSynchronize(e1);
+    float ms;
+    cudaEventElapsedTime(&ms, e0, e1);
+    if (ms < best) best = ms;
+  }
+  const double cyc = best * 1e-3 * 1.965e9 / NMMA;
+  printf("A in TMEM, kind::f16 M=128 N=%d K=16: %.3f ms  %.1f cycles/MMA (dense rate %.1f)\n", N, best, cyc,
+         128.0 * N * 16 * 2 / 8192);
+}
+
 template <int SW, int N, int MODE = 0>
 void run(float* out, int G) {
   const int smem = (128 + 256) * SW + 1024;
@@ -97,6 +289,20 @@ int main() {
   run<32, 256>(out, G);
   run<64, 128>(out, G);
   run<128, 128>(out, G);
+  run<64, 224>(out, G);
+  run<64, 192>(out, G);
+  run_split<0>(out, G);
+  run_split<16>(out, G);
+  run_unit<48, 0>(out, G);
+  run_unit<48, 0, 1>(out, G);
+  run_unit<48, 16, 1>(out, G);
+  run_unit<48, 16>(out, G);
+  run_unit<48, 8>(out, G);
+  run_unit<48, 2>(out, G);
+  run_unit<96, 16>(out, G);
+  run_ts<16>(out, G);
+  run_ts<32>(out, G);
+  run_ts<64>(out, G);
   run<64, 256, 1>(out, G);
   run<64, 256, 2>(out, G);
   run<64, 128, 1>(out, G);
