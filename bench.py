@@ -361,12 +361,11 @@ def run_ours(args):
         bf16 = pk.get("bf16_tflops_sustained" if long_step else "bf16_tflops") or pk.get("bf16_tflops")
         peak_kind = "sustained" if long_step and pk.get("bf16_tflops_sustained") else "burst"
         if f16:
-            # S contraction on kind::f16 (BF16/FP16 rate); the R > 16 V-MMA stays TF32 and is
-            # counted at twice its FLOPs (TF32 runs at half the FP16 rate): FP16-equivalent FLOPs
-            flops_pair = nprod * 2 * (K + (0 if vcc else 2 * R))
+            # S contraction and (R > 16) the V = P W contraction on kind::f16 (BF16/FP16 rate):
+            # 3 split products of 2K, and of 2R (P_hi [W_hi | W_lo] + P_lo W_hi), per pair
+            flops_pair = nprod * 2 * (K + (0 if vcc else R))
             peak = bf16 if bf16 else 2250.0
-            formula = ("%d products x 2K per pair" % nprod) if vcc else \
-                      ("%d products x 2(K+2R) per pair, FP16-equivalent" % nprod)
+            formula = ("%d products x 2K per pair" % nprod) if vcc else ("%d products x 2(K+R) per pair" % nprod)
             unit = "TFLOP/s (FP16 tensor; %s)" % formula
             deriv = ("MEASURED_PEAKS bf16 (%s) %.1f (kind::f16 = BF16 rate)" % (peak_kind, bf16)) if bf16 else \
                     "fallback nominal dense FP16 2.25 PFLOP/s"
@@ -380,12 +379,12 @@ def run_ours(args):
         achieved = pairs_launch * flops_pair / (kms / 1e3) / 1e12
         tensor = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": unit, "frac": achieved / peak,
                   "peak_derivation": deriv}
-        # the exponential: one 2^t per pair on MUFU.EX2 (16 / clk / SM), except the
-        # R = 1 epilogue's 4 of 16 that run as a polynomial on the FMA pipe
+        # the exponential: one 2^t per pair on MUFU.EX2 (16 / clk / SM), except the R = 1
+        # epilogue's 6 of 16 (folded layout; 4 of 16 unfolded) that run as a polynomial on the FMA pipe
         sfu_peak = 16 * sms * max_mhz * 1e6
         ex2_rate = pairs_launch / (kms / 1e3)
         sfu = {"bound": "alu", "achieved": ex2_rate / 1e9, "peak": sfu_peak / 1e9, "frac": ex2_rate / sfu_peak,
-               "unit": "G exponentials/s (MUFU.EX2 peak; R = 1 computes 1/4 of them on the FMA pipe)",
+               "unit": "G exponentials/s (MUFU.EX2 peak; R = 1 computes 6/16 of them on the FMA pipe)",
                "peak_derivation": f"16 ex2/clk/SM x {sms} SMs x {max_mhz} MHz (sm_max)"}
         # the binding resource is the primary roofline, the other the co-bound
         prim, co = (sfu, tensor) if sfu["frac"] >= tensor["frac"] else (tensor, sfu)
