@@ -128,9 +128,12 @@ KS_API ks_status ks_set_sources(ks_ctx *ctx, const float *alpha, const float *W,
 KS_API ks_status ks_eval(ks_ctx *ctx, const float *beta, int64_t N, float *V);
 
 /* Same as ks_set_sources / ks_eval but alpha, W, beta, V are HOST pointers.
- * The library stages them through its own device buffers (host->device copy,
- * compute, device->host copy) and returns after V is in host memory.
- * Pinned host memory gives the fastest copies; pageable memory works. */
+ * The library stages them through its own device buffers.  ks_set_sources_host
+ * returns once alpha and W have been copied (the caller may reuse them); the
+ * source preparation then runs on the context's stream.  ks_eval_host uploads
+ * beta on a library copy stream (overlapping that preparation), evaluates, and
+ * returns after V is in host memory.  Pinned host memory gives the fastest
+ * copies; pageable memory works. */
 KS_API ks_status ks_set_sources_host(ks_ctx *ctx, const float *alpha, const float *W,
                               int64_t M, int R);
 KS_API ks_status ks_eval_host(ks_ctx *ctx, const float *beta, int64_t N, float *V);

@@ -109,6 +109,10 @@ struct ks_ctx {
   double c = 0.0;  // log2(e) / (2 h^2)
   ks_precision prec_req = KS_PREC_AUTO;
   cudaStream_t stream = nullptr;
+  // host API: a copy stream for the target upload (overlaps the source prep still running on
+  // `stream`) and events that end the host calls once their uploads are done
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_copied = nullptr, ev_beta = nullptr;
 
   // current sources
   bool have_src = false;
@@ -632,6 +636,12 @@ ks_status ks_destroy(ks_ctx* ctx) {
   ctx->h_beta.release();
   ctx->h_V.release();
   for (cudaEvent_t ev : ctx->ev) cudaEventDestroy(ev);
+  if (ctx->ev_copied) cudaEventDestroy(ctx->ev_copied);
+  if (ctx->ev_beta) cudaEventDestroy(ctx->ev_beta);
+  if (ctx->copy_stream) {
+    cudaStreamSynchronize(ctx->copy_stream);
+    cudaStreamDestroy(ctx->copy_stream);
+  }
   delete ctx;
   return KS_OK;
 }
@@ -714,6 +724,16 @@ ks_status ks_reserve(ks_ctx* ctx, int64_t N_max) {
   return KS_OK;
 }
 
+namespace {
+ks_status host_api_init(ks_ctx* ctx) {
+  if (ctx->copy_stream) return KS_OK;
+  KS_CUDA(cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking), "create copy stream");
+  KS_CUDA(cudaEventCreateWithFlags(&ctx->ev_copied, cudaEventDisableTiming), "create event");
+  KS_CUDA(cudaEventCreateWithFlags(&ctx->ev_beta, cudaEventDisableTiming), "create event");
+  return KS_OK;
+}
+}  // namespace
+
 ks_status ks_set_sources_host(ks_ctx* ctx, const float* alpha, const float* W, int64_t M, int R) {
   if (check_ctx(ctx)) return KS_EINVAL;
   if (M < 0) return fail(KS_EINVAL, "M=%lld < 0", (long long)M);
@@ -724,13 +744,18 @@ ks_status ks_set_sources_host(ks_ctx* ctx, const float* alpha, const float* W, i
   const size_t na = (size_t)M * ctx->K, nw = (size_t)M * R;
   KS_CUDA(ctx->h_alpha.reserve(na ? na : 1, ctx->stream, false), "allocate alpha staging");
   KS_CUDA(ctx->h_W.reserve(nw ? nw : 1, ctx->stream, false), "allocate W staging");
+  s = host_api_init(ctx);
+  if (s != KS_OK) return s;
   if (M > 0) {
     KS_CUDA(cudaMemcpyAsync(ctx->h_alpha.p, alpha, na * 4, cudaMemcpyHostToDevice, ctx->stream), "copy alpha H2D");
     KS_CUDA(cudaMemcpyAsync(ctx->h_W.p, W, nw * 4, cudaMemcpyHostToDevice, ctx->stream), "copy W H2D");
   }
+  KS_CUDA(cudaEventRecord(ctx->ev_copied, ctx->stream), "cudaEventRecord");
   s = ks_set_sources(ctx, ctx->h_alpha.p, ctx->h_W.p, M, R);
   if (s != KS_OK) return s;
-  KS_CUDA(cudaStreamSynchronize(ctx->stream), "synchronize");
+  // return once the host buffers have been read; the source prep runs on (stream-ordered
+  // before any later call on this context)
+  KS_CUDA(cudaEventSynchronize(ctx->ev_copied), "synchronize");
   return KS_OK;
 }
 
@@ -743,9 +768,15 @@ ks_status ks_eval_host(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   ks_status s = set_device(ctx);
   if (s != KS_OK) return s;
   const size_t nb = (size_t)N * ctx->K, nv = (size_t)N * ctx->R;
+  s = host_api_init(ctx);
+  if (s != KS_OK) return s;
   KS_CUDA(ctx->h_beta.reserve(nb, ctx->stream, false), "allocate beta staging");
   KS_CUDA(ctx->h_V.reserve(nv, ctx->stream, false), "allocate V staging");
-  KS_CUDA(cudaMemcpyAsync(ctx->h_beta.p, beta, nb * 4, cudaMemcpyHostToDevice, ctx->stream), "copy beta H2D");
+  // the upload runs on the copy stream (overlapping a source prep still in flight on `stream`;
+  // the staging buffer's previous readers finished before the previous ks_eval_host returned)
+  KS_CUDA(cudaMemcpyAsync(ctx->h_beta.p, beta, nb * 4, cudaMemcpyHostToDevice, ctx->copy_stream), "copy beta H2D");
+  KS_CUDA(cudaEventRecord(ctx->ev_beta, ctx->copy_stream), "cudaEventRecord");
+  KS_CUDA(cudaStreamWaitEvent(ctx->stream, ctx->ev_beta, 0), "cudaStreamWaitEvent");
   s = ks_eval(ctx, ctx->h_beta.p, N, ctx->h_V.p);
   if (s != KS_OK) return s;
   KS_CUDA(cudaMemcpyAsync(V, ctx->h_V.p, nv * 4, cudaMemcpyDeviceToHost, ctx->stream), "copy V D2H");

@@ -1640,7 +1640,8 @@ static cudaError_t launch_rcsv(const CUtensorMap* m, const TcArgs& a, cudaStream
 
 // exponential pairs of 16 on the FMA pipe, measured (kernel ms): unfolded log-weight epilogue cfg3
 // PP 0 1.34, 4 1.31, 6 1.41, 8 1.55; folded layout cfg3 PP 0 1.135, 4 1.057, 6 1.046, 8 1.150,
-// cfg5 301.0 / 270.2 / 254.7 / 284.7, cfg2 0.091 / 0.085 / 0.081 / 0.089
+// cfg5 301.0 / 270.2 / 254.7 / 284.7, cfg2 0.091 / 0.085 / 0.081 / 0.089; resident-target kernel
+// (same box) PP 5 / 6 / 7: cfg3 1.0086 / 1.0083 / 1.0370, cfg5 263.4 / 259.8 / 257.9
 static constexpr int kTcPolyDefault = 6;
 
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st) {
@@ -1658,6 +1659,8 @@ cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream
         switch (pp) {
           case 0: return launch_rcsv<16, 4, 1, 32>(maps, a, st);
           case 4: return launch_rcsv<16, 4, 1, 36>(maps, a, st);
+          case 5: return launch_rcsv<16, 4, 1, 37>(maps, a, st);
+          case 7: return launch_rcsv<16, 4, 1, 39>(maps, a, st);
           default: return launch_rcsv<16, 4, 1, 38>(maps, a, st);
         }
       }
