@@ -405,13 +405,10 @@ static bool fp32_split() {
 template <int KP, bool SPLIT>
 static cudaError_t launch_kps(const CUtensorMap* tmap, const Fp32Args& a, cudaStream_t st) {
   using C = Fp32Cfg<KP>;
-  static bool attr_done = false;
-  if (!attr_done) {
-    cudaError_t e = cudaFuncSetAttribute(ks_fused_fp32_kernel<KP, SPLIT>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::kSmemBytes);
-    if (e != cudaSuccess) return e;
-    attr_done = true;
-  }
+  static std::atomic<uint64_t> attr_done{0};
+  cudaError_t e = smem_optin_once(attr_done, reinterpret_cast<const void*>(ks_fused_fp32_kernel<KP, SPLIT>),
+                                  (int)C::kSmemBytes);
+  if (e != cudaSuccess) return e;
   ks_fused_fp32_kernel<KP, SPLIT><<<a.sk.grid, C::kThreads, C::kSmemBytes, st>>>(*tmap, a);
   return cudaGetLastError();
 }

@@ -65,9 +65,11 @@ struct TcSmemT {
                : ((AR ? 1u : 2u) * wslot(r_c) + 512 + 1023) & ~1023u;
   }
   static constexpr uint32_t na_off(int r_c) { return VCC ? 0u : (AR ? 1u : 2u) * wslot(r_c); }
-  static constexpr int kWSlots = VCC && RV < 8 ? 4 : 2;  // W/na ring depth (RV >= 8: 2 to fit 4 stages)
+  // W/na ring depth (RV >= 8: 2 to fit 4 stages; FP16 V-MMA with the resident target operand: 3,
+  // so the next tile's weights load while the MMAs of two tiles run)
+  static constexpr int kWSlots = VCC && RV < 8 ? 4 : (AR && !VCC ? 3 : 2);
   static constexpr uint32_t bar_off(int r_c) { return kW0 + kWSlots * w_slot_bytes(r_c); }
-  static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 512 + 4 * kTcTileT * 8; }  // + VCC scratch
+  static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 512 + (VCC ? 4 * kTcTileT * 8 : 0); }  // + VCC scratch
 };
 
 // Resident-target (AR) kernels stage whole tiles: P operand planes per tile (per 64-byte
@@ -513,9 +515,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       const int bp = p & 1;
       const uint32_t use = (uint32_t)(p >> 1);
       mbar_wait(&pready[bp * 2 + hh], use & 1);
-      if (hh == 0) mbar_wait(&wfull[p & 1], use & 1);
+      if (hh == 0) mbar_wait(&wfull[p % WS], (uint32_t)((p / WS) & 1));
       tc_fence_after();
-      uint8_t* ws = smem + TcSmem::kW0 + (p & 1) * TcSmem::w_slot_bytes(RC);
+      uint8_t* ws = smem + TcSmem::kW0 + (p % WS) * TcSmem::w_slot_bytes(RC);
       const uint32_t colP = (bp ? kColS1 : kColS0) + 64 * hh;
       const uint32_t colL = kColPlo + 64 * hh;
       bool acc = !first;
@@ -554,7 +556,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       __syncwarp();
       if (leader) {
         tc_commit(&vdone[hh]);
-        if (hh == 1) tc_commit(&wempty[p & 1]);
+        if (hh == 1) tc_commit(&wempty[p % WS]);
       }
       __syncwarp();
     };
@@ -1145,7 +1147,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
       const int bq = q & 1;
       const uint32_t use = (uint32_t)(q >> 1);
-      mbar_wait(&wfull[q & 1], use & 1);
+      mbar_wait(&wfull[q % WS], (uint32_t)((q / WS) & 1));
       mbar_wait(&sfull[bq], use & 1);
       tc_fence_after();
       if (q > 0 && ((prev_st + 1 == n_s) || ((prev_st + 1) % kFlush == 0))) {
@@ -1159,7 +1161,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         nbj = __ldg(args.nb + cu.tt * kTcTileT + row);  // 0 when args.aug
         rjs = __ldg(args.tsc + cu.tt * kTcTileT + row);
       }
-      const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q & 1) * TcSmem::w_slot_bytes(RC) +
+      const float* nas = reinterpret_cast<const float*>(smem + TcSmem::kW0 + (q % WS) * TcSmem::w_slot_bytes(RC) +
                                                        TcSmem::na_off(RC));
       const uint32_t colS = bq ? kColS1 : kColS0;
       if (args.f16) {
@@ -1624,16 +1626,13 @@ int fused_tc_rv(int R) { return R <= 1 ? 1 : R <= 2 ? 2 : R <= 4 ? 4 : R <= 8 ? 
 
 template <int RC, int NS, int RV, int PP = 0>
 static cudaError_t launch_rcsv(const CUtensorMap* m, const TcArgs& a, cudaStream_t st) {
-  static bool attr_done = false;
+  static std::atomic<uint64_t> attr_done{0};
   using Sm = TcSmemT<NS, RV ? 256 : kTcTileS, RV, (PP & 32) != 0>;
   const size_t smem = Sm::total(RC);
   static_assert(Sm::total(RC) <= 232448, "exceeds 227 KB of shared memory");
-  if (!attr_done) {
-    cudaError_t e = cudaFuncSetAttribute(ks_fused_tc_kernel<RC, NS, RV, PP>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    attr_done = true;
-  }
+  cudaError_t e = smem_optin_once(attr_done, reinterpret_cast<const void*>(ks_fused_tc_kernel<RC, NS, RV, PP>),
+                                  (int)smem);
+  if (e != cudaSuccess) return e;
   ks_fused_tc_kernel<RC, NS, RV, PP><<<a.sk.grid, kTcThreads, smem, st>>>(m[0], m[1], m[2], m[3], m[4], m[5], a);
   return cudaGetLastError();
 }
@@ -1678,10 +1677,10 @@ cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream
     default: break;
   }
   // FP16 V-MMA with the target operand resident (K <= 256; KS_TC_ARES=0 reloads it per unit):
-  // 4 source stages fit beside the 128 KB operand at r_c = 16, 3 at r_c = 32
+  // 4 source stages fit beside the 128 KB operand and 3 W slots at r_c = 16, 2 at r_c = 32
   if (a.f16 && a.ares && a.k_pad <= 8 * kTcKC) {
     if (a.r_c == 16) return launch_rcsv<16, 4, 0, 32>(maps, a, st);
-    if (a.r_c == 32) return launch_rcsv<32, 3, 0, 32>(maps, a, st);
+    if (a.r_c == 32) return launch_rcsv<32, 2, 0, 32>(maps, a, st);
   }
   const int ns = tc_stages(a.r_c);
   if (a.r_c == 16) {

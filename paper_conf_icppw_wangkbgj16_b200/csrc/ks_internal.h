@@ -4,9 +4,24 @@
 
 #include <cuda.h>
 #include <cuda_runtime.h>
+#include <atomic>
 #include <cstdint>
 
 namespace ks {
+
+// The dynamic shared-memory opt-in (cudaFuncAttributeMaxDynamicSharedMemorySize) is per device:
+// set it once per (kernel instantiation, device).  `done` is a per-instantiation bitmask of
+// device ordinals (devices >= 64 set it on every launch).
+inline cudaError_t smem_optin_once(std::atomic<uint64_t>& done, const void* fn, int bytes) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  const uint64_t bit = dev < 64 ? (1ull << dev) : 0ull;
+  if (bit && (done.load(std::memory_order_acquire) & bit)) return cudaSuccess;
+  e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  if (e == cudaSuccess && bit) done.fetch_or(bit, std::memory_order_acq_rel);
+  return e;
+}
 
 constexpr int kTileT = 256;   // targets per CTA tile (FP32 path)
 constexpr int kTileS = 128;   // sources per pipeline stage (FP32 path)

@@ -197,6 +197,28 @@ def test_host_api_matches_device_api():
     assert np.array_equal(gpu_eval(a, W, b, h), gpu_eval(a, W, b, h, host=True))
 
 
+def test_host_api_buffers_reusable_on_return():
+    """ks_set_sources_host returns once alpha and W are uploaded (the preparation
+    continues on the stream) and ks_eval_host once V is on the host: overwriting
+    the caller's host arrays right after each call must not change any result,
+    including across a source replacement and back-to-back evaluations."""
+    a, W, b, h = workloads.make(3, M=5000, N=2100, wkind="pos")
+    ref = gpu_eval(a, W, b, h)
+    a2, W2, b2 = a.copy(), W.copy(), b.copy()
+    with ks.KernelSum(a.shape[1], float(h), _PREC["p"]) as plan:
+        plan.set_sources_host(a2, W2)
+        a2[:] = 7.0
+        W2[:] = -3.0
+        V1 = plan.eval_host(b2).astype(np.float64)
+        b2[:] = 0.0
+        V2 = plan.eval_host(b).astype(np.float64)
+        plan.set_sources_host(np.ascontiguousarray(a[::-1]), np.ascontiguousarray(W[::-1]))
+        V3 = plan.eval_host(b).astype(np.float64)
+    assert np.array_equal(V1, ref) and np.array_equal(V2, ref)
+    # reversed source order: same sums up to rounding order
+    assert np.max(np.abs(V3 - ref)) <= 1e-5 * np.abs(W).sum()
+
+
 def test_repeated_eval_and_reset_sources(oracle_mod):
     """Counters are left zero across launches; sources can be replaced."""
     a, W, b, h = workloads.make(3, M=4000, N=200, wkind="pos")
