@@ -492,6 +492,8 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   {
     const char* e = getenv("KS_TC_ARES");  // measurement knob: 0 = reload the target operand per unit
     a.ares = (e && e[0] == '0') ? 0 : 1;
+    const char* es = getenv("KS_TC_AR_STAGES");  // measurement knob: 5 = one source stage more
+    a.ar_stages = (es && es[0] == '5') ? 5 : 4;
   }
   {
     const char* e = getenv("KS_TC_WSLOTS");  // measurement knob

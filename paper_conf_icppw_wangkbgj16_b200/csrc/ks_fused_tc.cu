@@ -65,9 +65,8 @@ struct TcSmemT {
                : ((AR ? 1u : 2u) * wslot(r_c) + 512 + 1023) & ~1023u;
   }
   static constexpr uint32_t na_off(int r_c) { return VCC ? 0u : (AR ? 1u : 2u) * wslot(r_c); }
-  // W/na ring depth (RV >= 8: 2 to fit 4 stages; FP16 V-MMA with the resident target operand: 3,
-  // so the next tile's weights load while the MMAs of two tiles run)
-  static constexpr int kWSlots = VCC && RV < 8 ? 4 : (AR && !VCC ? 3 : 2);
+  // W/na ring depth (RV >= 8: 2 to fit 4 stages)
+  static constexpr int kWSlots = VCC && RV < 8 ? 4 : 2;
   static constexpr uint32_t bar_off(int r_c) { return kW0 + kWSlots * w_slot_bytes(r_c); }
   static constexpr uint32_t total(int r_c) { return bar_off(r_c) + 512 + (VCC ? 4 * kTcTileT * 8 : 0); }  // + VCC scratch
 };
@@ -1147,15 +1146,22 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     for (int q = 0; q < count; ++q, unit_next(sc, cu)) {
       const int bq = q & 1;
       const uint32_t use = (uint32_t)(q >> 1);
+      PROF_BEGIN(e0);
       mbar_wait(&wfull[q % WS], (uint32_t)((q / WS) & 1));
+      PROF_END(0, e0);
+      PROF_BEGIN(e1);
       mbar_wait(&sfull[bq], use & 1);
       tc_fence_after();
+      PROF_END(1, e1);
+      PROF_BEGIN(e3);
       if (q > 0 && ((prev_st + 1 == n_s) || ((prev_st + 1) % kFlush == 0))) {
         // block end: V(q-1) complete, fold it into FP64 registers (and write at segment end)
         mbar_wait(&vdone[1], (uint32_t)((q - 1) & 1));
         tc_fence_after();
         v_collect(q - 1, prev_tt, prev_st);
       }
+      PROF_END(3, e3);
+      PROF_BEGIN(e2);
       if (q == seg_q) {  // new segment: this target tile's norms
         seg_st0 = cu.st;
         nbj = __ldg(args.nb + cu.tt * kTcTileT + row);  // 0 when args.aug
@@ -1205,6 +1211,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           mbar_arrive(&pready[bq * 2 + 0]);
           mbar_arrive(&pready[bq * 2 + 1]);
         }
+        PROF_END(2, e2);
       } else {
 #pragma unroll 1
       for (int hh = 0; hh < 2; ++hh) {
@@ -1677,10 +1684,11 @@ cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream
     default: break;
   }
   // FP16 V-MMA with the target operand resident (K <= 256; KS_TC_ARES=0 reloads it per unit):
-  // 4 source stages fit beside the 128 KB operand and 3 W slots at r_c = 16, 2 at r_c = 32
+  // 4 source stages beside the 128 KB operand at r_c = 16 (5 fit, KS_TC_AR_STAGES=5: measured
+  // 116.6 vs 114.5 ms at cfg4 -- the kernel is at the board power cap, not load-latency bound), 3 at r_c = 32
   if (a.f16 && a.ares && a.k_pad <= 8 * kTcKC) {
-    if (a.r_c == 16) return launch_rcsv<16, 4, 0, 32>(maps, a, st);
-    if (a.r_c == 32) return launch_rcsv<32, 2, 0, 32>(maps, a, st);
+    if (a.r_c == 16) return a.ar_stages == 5 ? launch_rcsv<16, 5, 0, 32>(maps, a, st) : launch_rcsv<16, 4, 0, 32>(maps, a, st);
+    if (a.r_c == 32) return launch_rcsv<32, 3, 0, 32>(maps, a, st);
   }
   const int ns = tc_stages(a.r_c);
   if (a.r_c == 16) {

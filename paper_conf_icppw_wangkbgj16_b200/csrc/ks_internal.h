@@ -108,6 +108,7 @@ struct TcArgs {
   const unsigned* wcol; // FP16 V-MMA (f16, !vcc): [r_pad] FP32 bits of max_i |W_ir| (column scale exponents)
   int wslots;           // VCC W/na ring depth (2..4; 0 = default)
   int ares;             // R = 1, <= 2 operand chunks: target operand resident per target tile (no reload per unit)
+  int ar_stages;        // FP16 V-MMA, resident target operand: source stages (4; 5 measurement knob)
   int dbg_skip_v;       // measurement only (KS_TC_DEBUG_SKIP_V=1): do not issue the V MMAs (wrong results)
   const float* na;      // [m_pad]  -c ||alpha_hat||^2
   const float* nb;      // [n_pad]  -c ||beta_hat||^2

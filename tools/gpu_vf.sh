@@ -8,7 +8,7 @@ KS_TC_VCC=0 timeout 900 python -m pytest tests/test_gpu_tc.py -m gpu -q -x > $OU
 tail -3 $OUT/pytest_gpu.log; tail -15 $OUT/pytest_gpu_vcc0.log; tail -6 $OUT/smoke.log
 timeout 600 python bench.py --cfg 4 --steps 3 --warmup 1 --no-cpu-baseline > $OUT/bench_cfg4.json 2>&1
 KS_TC_VCC=0 timeout 600 python bench.py --cfg 4 --steps 3 --warmup 1 --no-cpu-baseline > $OUT/bench_cfg4_vf.json 2>&1
-KS_TC_VCC=0 KS_TC_ARES=0 timeout 600 python bench.py --cfg 4 --steps 3 --warmup 1 --no-cpu-baseline > $OUT/bench_cfg4_vf_noar.json 2>&1
+KS_TC_VCC=0 KS_TC_AR_STAGES=4 timeout 600 python bench.py --cfg 4 --steps 3 --warmup 1 --no-cpu-baseline > $OUT/bench_cfg4_vf_ar4.json 2>&1
 for f in $OUT/bench*.json; do python - "$f" <<'PY'
 import json,sys
 try:
