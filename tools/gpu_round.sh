@@ -20,6 +20,7 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:ks_f
    python bench.py --precision fp32 --steps 1 --warmup 4 --no-cpu-baseline > $OUT/ncu_full_fp32.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:ks_fused -s 2 -c 1 -o $OUT/prof_cfg4 \
    python bench.py --cfg 4 --steps 1 --warmup 2 --no-cpu-baseline > $OUT/ncu_full4.log 2>&1
+timeout 900 python tools/grid.py $OUT > $OUT/grid.log 2>&1
 tail -3 $OUT/pytest_gpu.log; tail -4 $OUT/smoke.log
 for f in $OUT/bench*.json; do python - "$f" <<'PY'
 import json,sys
