@@ -269,11 +269,6 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   long long pf[5] = {0, 0, 0, 0, 0};
   const long long pf_t0 = clock64();
 #endif
-  // R = 1: W >= 0 (log-weights) and the folded layout active -> the epilogue is exp2 + sum
-  // of the raw accumulator and needs no per-tile norms or weights (no W/na ring)
-  const bool logw_k = RV == 1 && args.wstat != nullptr && args.wstat[1] == 0u && args.wstat[0] != 0u;
-  const bool fold_k = RV == 1 && args.fold && f16_fold_ok(args.amax, args.c, args.K);
-  const bool ring = !(logw_k && fold_k && !CLAMP_LW);
   // measurement knobs (KS_TC_DEBUG_SKIP_V, wrong results): 1 no epilogue math, 4 W/na loaded once,
   // 5 no S MMAs, 6 one product, 7 no MMAs and no operand loads, 8 = 1 + 5, 9 = 1 + no operand
   // loads, 10 = 1 + 7
@@ -316,6 +311,14 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = *tmem_base_smem;
+  // programmatic dependent launch: the prologue above overlaps the target prep; nothing the
+  // preceding kernels wrote is read before this point
+  pdl_wait();
+  // R = 1: W >= 0 (log-weights) and the folded layout active -> the epilogue is exp2 + sum
+  // of the raw accumulator and needs no per-tile norms or weights (no W/na ring)
+  const bool logw_k = RV == 1 && args.wstat != nullptr && args.wstat[1] == 0u && args.wstat[0] != 0u;
+  const bool fold_k = RV == 1 && args.fold && f16_fold_ok(args.amax, args.c, args.K);
+  const bool ring = !(logw_k && fold_k && !CLAMP_LW);
 
   if (!VCC && AR && warp == 0) {
     // ================= TMA producer, FP16 V-MMA kernel with the target operand resident (K <= 256):
@@ -1324,6 +1327,8 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
                                        void* __restrict__ src_lo, float* __restrict__ na,
                                        float* __restrict__ wt_hi, float* __restrict__ wt_lo,
                                        float* __restrict__ wv, int rv, const unsigned* __restrict__ wstat) {
+  pdl_trigger();  // let the next kernel launch early
+  pdl_wait();     // the source statistics are complete
   const int lane = threadIdx.x & 31, gl = lane & (G - 1);
   const int64_t i = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
   if (i >= m_pad) return;
@@ -1415,6 +1420,8 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
                                        const unsigned* __restrict__ amax, void* __restrict__ tgt_hi,
                                        void* __restrict__ tgt_lo, float* __restrict__ nb,
                                        float* __restrict__ tsc) {
+  pdl_trigger();  // let the fused kernel's CTAs start their prologue
+  pdl_wait();     // the source statistics (mu, amax) are complete
   const int lane = threadIdx.x & 31, gl = lane & (G - 1);
   const int64_t j = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
   if (j >= n_pad) return;
@@ -1551,9 +1558,9 @@ static cudaError_t launch_prep_sources(const float* alpha, const float* W, int64
   if (m_pad == 0) return cudaSuccess;
   const int bs = 256, G = prep_group(K);
   const unsigned grid = (unsigned)((m_pad * G + bs - 1) / bs);
-#define KS_PREP_S(g)                                                                                          \
-  prep_tc_sources_kernel<F16, g><<<grid, bs, 0, st>>>(alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, amax, \
-                                                      src_hi, src_lo, na, wt_hi, wt_lo, wv, rv, wstat)
+#define KS_PREP_S(g)                                                                                        \
+  return launch_pdl(prep_tc_sources_kernel<F16, g>, grid, bs, 0, st, alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, \
+                    aug, amax, src_hi, src_lo, na, wt_hi, wt_lo, wv, rv, wstat)
   switch (G) {
     case 4: KS_PREP_S(4); break;
     case 8: KS_PREP_S(8); break;
@@ -1571,8 +1578,9 @@ static cudaError_t launch_prep_targets(const float* beta, int64_t N, int64_t n_p
   if (n_pad == 0) return cudaSuccess;
   const int bs = 256, G = prep_group(K);
   const unsigned grid = (unsigned)((n_pad * G + bs - 1) / bs);
-#define KS_PREP_T(g) \
-  prep_tc_targets_kernel<F16, g><<<grid, bs, 0, st>>>(beta, N, n_pad, K, k_pad, mu, c, aug, amax, tgt_hi, tgt_lo, nb, tsc)
+#define KS_PREP_T(g)                                                                                           \
+  return launch_pdl(prep_tc_targets_kernel<F16, g>, grid, bs, 0, st, beta, N, n_pad, K, k_pad, mu, c, aug, amax, \
+                    tgt_hi, tgt_lo, nb, tsc)
   switch (G) {
     case 4: KS_PREP_T(4); break;
     case 8: KS_PREP_T(8); break;
@@ -1640,8 +1648,8 @@ static cudaError_t launch_rcsv(const CUtensorMap* m, const TcArgs& a, cudaStream
   cudaError_t e = smem_optin_once(attr_done, reinterpret_cast<const void*>(ks_fused_tc_kernel<RC, NS, RV, PP>),
                                   (int)smem);
   if (e != cudaSuccess) return e;
-  ks_fused_tc_kernel<RC, NS, RV, PP><<<a.sk.grid, kTcThreads, smem, st>>>(m[0], m[1], m[2], m[3], m[4], m[5], a);
-  return cudaGetLastError();
+  return launch_pdl(ks_fused_tc_kernel<RC, NS, RV, PP>, a.sk.grid, kTcThreads, smem, st, m[0], m[1], m[2], m[3], m[4],
+                    m[5], a);
 }
 
 // exponential pairs of 16 on the FMA pipe, measured (kernel ms): unfolded log-weight epilogue cfg3

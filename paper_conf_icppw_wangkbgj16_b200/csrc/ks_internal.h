@@ -9,6 +9,30 @@
 
 namespace ks {
 
+// Programmatic dependent launch (PDL): kernels of the TC path after the source statistics are
+// launched with programmatic stream serialization, start their CTAs while the preceding
+// kernel finishes (it calls pdl_trigger early) and block in pdl_wait until it has completed
+// and its writes are visible; every such kernel calls pdl_wait before touching memory the
+// preceding kernels write or read.  KS_PDL=0 launches them plainly (measurement knob).
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+bool pdl_enabled();
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                       Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
+
 // The dynamic shared-memory opt-in (cudaFuncAttributeMaxDynamicSharedMemorySize) is per device:
 // set it once per (kernel instantiation, device).  `done` is a per-instantiation bitmask of
 // device ordinals (devices >= 64 set it on every launch).

@@ -13,6 +13,8 @@
 //      coordinates, norms and weights into shared memory.
 #include "ks_internal.h"
 
+#include <cstdlib>
+
 namespace ks {
 
 // Source statistics in one launch.  Each block reduces a contiguous chunk of
@@ -39,6 +41,7 @@ __global__ void source_stats_kernel(const float* __restrict__ alpha, const float
   __shared__ float rmn[256], rmx[256];
   __shared__ unsigned s_w[2], s_amax;
   __shared__ bool s_last;
+  pdl_trigger();  // the source prep may start its CTAs (it waits for this grid to complete)
   const int b = blockIdx.x;
   const int t = threadIdx.x;
   const int64_t chunk = (M + nparts - 1) / nparts;
@@ -185,6 +188,14 @@ __global__ void source_stats_kernel(const float* __restrict__ alpha, const float
     if (amax != nullptr) *amax = s_amax;
     *counter = 0u;  // ready for the next call (stream order)
   }
+}
+
+bool pdl_enabled() {
+  static const bool on = [] {
+    const char* e = getenv("KS_PDL");
+    return !(e && e[0] == '0');
+  }();
+  return on;
 }
 
 cudaError_t launch_source_stats(const float* alpha, const float* W, int64_t M, int K, int k_pad, int nparts,
