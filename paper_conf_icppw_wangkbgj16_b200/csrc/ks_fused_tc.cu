@@ -1664,8 +1664,9 @@ cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream
     case 1: {
       // R = 1: exponential pairs of 16 on the FMA pipe (KS_TC_POLY = 0, 4, 6 or 8)
       // and the exact d^2 >= 0 clamp of the log-weight epilogue (KS_TC_CLAMP=1; costs 15% at cfg3)
+      // one operand chunk (K <= 26 folded): the contraction is shorter, 7 of 16 on the FMA pipe
       const char* e = getenv("KS_TC_POLY");
-      const int pp = e ? atoi(e) : kTcPolyDefault;
+      const int pp = e ? atoi(e) : (a.ares && a.f16 && a.k_pad <= kTcKC ? 7 : kTcPolyDefault);
       const char* ec = getenv("KS_TC_CLAMP");
       const bool clamp = ec && ec[0] == '1';
       if (clamp) return pp == 0 ? launch_rcsv<16, 4, 1, 16>(maps, a, st) : launch_rcsv<16, 4, 1, 20>(maps, a, st);
