@@ -449,6 +449,8 @@ def run_ours(args):
         e2e_step()
         torch.cuda.synchronize()
         e_ms.append(1e3 * (time.perf_counter() - t0))
+    if os.environ.get("KS_BENCH_E2E_DEBUG"):
+        print("e2e per-step ms:", " ".join("%.3f" % x for x in e_ms), file=sys.stderr)
     t = torch.tensor([sum(e_ms) / len(e_ms)], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)

@@ -203,9 +203,14 @@ cudaError_t source_stats(ks_ctx* ctx, const float* alpha, const float* W, bool w
                          bool want_amax) {
   cudaStream_t st = ctx->stream;
   const int K = ctx->K;
-  int nparts = (int)((M + 255) / 256);  // blocks of >= 256 rows each (one wave; short final reduction)
-  if (nparts < 1) nparts = 1;
-  if (nparts > 1024) nparts = 1024;
+  // ~8 K coordinates per block (256 rows at K = 32, 32 rows at K = 256): a few unrolled loads
+  // per thread; at most 1024 blocks when the last block reduces them (K <= 32), 4096 when
+  // K + 1 blocks do (launch_source_stats)
+  const int64_t rows = K >= 8192 ? 1 : 8192 / K;
+  int64_t np64 = (M + rows - 1) / rows;
+  if (np64 < 1) np64 = 1;
+  if (np64 > (K > 32 ? 4096 : 1024)) np64 = K > 32 ? 4096 : 1024;
+  const int nparts = (int)np64;
   cudaError_t e;
   if ((e = ctx->mean_part.reserve((size_t)nparts * K, st, false)) != cudaSuccess) return e;
   if ((e = ctx->mean_pmm.reserve((size_t)nparts * K * 2, st, false)) != cudaSuccess) return e;
@@ -214,7 +219,7 @@ cudaError_t source_stats(ks_ctx* ctx, const float* alpha, const float* W, bool w
   if ((e = ctx->mu.reserve(k_pad, st, false)) != cudaSuccess) return e;
   if (want_amax && (e = ctx->amax.reserve(1, st, false)) != cudaSuccess) return e;
   if (want_w && (e = ctx->wstat.reserve(2, st, false)) != cudaSuccess) return e;
-  ctx->launches += 1;
+  ctx->launches += K > 32 ? 2 : 1;
   return ks::launch_source_stats(alpha, W, M, K, k_pad, nparts, ctx->mean_part.p, ctx->mean_pmm.p, ctx->mean_pw.p,
                                  ctx->stats_counter.p, ctx->mu.p, want_amax ? ctx->amax.p : nullptr,
                                  want_w ? ctx->wstat.p : nullptr, st);

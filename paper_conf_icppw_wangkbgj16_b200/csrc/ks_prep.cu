@@ -121,6 +121,10 @@ __global__ void source_stats_kernel(const float* __restrict__ alpha, const float
     pw[2 * b] = s_w[0];
     pw[2 * b + 1] = s_w[1];
   }
+  if (counter == nullptr) {  // K > 32: stats_final_kernel reduces the partials (one block per dim)
+    if (b == 0 && t == 0 && amax != nullptr) *amax = 0u;
+    return;
+  }
   // publish the partials, then elect the last block
   __threadfence();
   __syncthreads();
@@ -198,11 +202,75 @@ bool pdl_enabled() {
   return on;
 }
 
+// K > 32: the block partials are reduced by K + 1 blocks instead of the last one -- block d
+// sums dimension d over all partials (thread t: partials t, t + 256, ... in order, then a
+// fixed shared-memory tree), writes mu[d] and folds its max |fl(alpha_d - mu_d)| into amax
+// (atomicMax: order-independent; zeroed by the partial kernel); block K writes the padding
+// dims of mu and the weight statistics.
+__global__ void __launch_bounds__(256) stats_final_kernel(int64_t M, int K, int k_pad, int nparts,
+                                                          const double* __restrict__ part,
+                                                          const float* __restrict__ pmm,
+                                                          const unsigned* __restrict__ pw, float* __restrict__ mu,
+                                                          unsigned* __restrict__ amax, unsigned* __restrict__ wstat) {
+  __shared__ double red[256];
+  __shared__ float rmn[256], rmx[256];
+  const int d = blockIdx.x, t = threadIdx.x;
+  if (d == K) {
+    for (int e = K + t; e < k_pad; e += blockDim.x) mu[e] = 0.f;
+    if (wstat != nullptr && t < 32) {
+      unsigned m = 0u, neg = 0u;
+      for (int q = t; q < nparts; q += 32) {
+        m = max(m, pw[2 * q]);
+        neg |= pw[2 * q + 1];
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        m = max(m, __shfl_xor_sync(0xffffffffu, m, o));
+        neg |= __shfl_xor_sync(0xffffffffu, neg, o);
+      }
+      if (t == 0) {
+        wstat[0] = m;
+        wstat[1] = neg;
+      }
+    }
+    return;
+  }
+  double s = 0.0;
+  float mn = INFINITY, mx = -INFINITY;
+#pragma unroll 4
+  for (int q = t; q < nparts; q += blockDim.x) {
+    s += part[(int64_t)q * K + d];
+    const float2 m2 = *reinterpret_cast<const float2*>(&pmm[((int64_t)q * K + d) * 2]);
+    mn = fminf(mn, m2.x);
+    mx = fmaxf(mx, m2.y);
+  }
+  red[t] = s;
+  rmn[t] = mn;
+  rmx[t] = mx;
+  __syncthreads();
+  for (int o = 128; o > 0; o >>= 1) {
+    if (t < o) {
+      red[t] += red[t + o];
+      rmn[t] = fminf(rmn[t], rmn[t + o]);
+      rmx[t] = fmaxf(rmx[t], rmx[t + o]);
+    }
+    __syncthreads();
+  }
+  if (t == 0) {
+    const float m = M > 0 ? (float)(red[0] / (double)M) : 0.f;
+    mu[d] = m;
+    // NaN coordinates give a NaN mean; fmaxf(NaN, 0) = 0 then ignores them
+    if (M > 0 && amax != nullptr) atomicMax(amax, __float_as_uint(fmaxf(fmaxf(rmx[0] - m, m - rmn[0]), 0.f)));
+  }
+}
+
 cudaError_t launch_source_stats(const float* alpha, const float* W, int64_t M, int K, int k_pad, int nparts,
                                 double* part, float* pmm, unsigned* pw, unsigned* counter, float* mu,
                                 unsigned* amax, unsigned* wstat, cudaStream_t st) {
-  source_stats_kernel<<<nparts, 256, 0, st>>>(alpha, W, M, K, k_pad, nparts, part, pmm, pw, counter, mu, amax,
-                                              wstat);
+  const bool split = K > 32;  // wide points: reduce the partials with K + 1 blocks
+  source_stats_kernel<<<nparts, 256, 0, st>>>(alpha, W, M, K, k_pad, nparts, part, pmm, pw, split ? nullptr : counter,
+                                              mu, amax, wstat);
+  if (split) stats_final_kernel<<<K + 1, 256, 0, st>>>(M, K, k_pad, nparts, part, pmm, pw, mu, amax, wstat);
   return cudaGetLastError();
 }
 
