@@ -369,9 +369,16 @@ int tc_k_pad(int K) { return (int)round_up(K + 2 * tc_aug(K), ks::kTcKC); }
 ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M, int R) {
   const int K = ctx->K;
   const bool f16 = ctx->prec_eff == KS_PREC_3XF16;
-  // R == 1: weighted sum on CUDA cores (KS_TC_VCC=0 forces the tensor-core V path; measurement knob)
+  // Weighted sum: on CUDA cores (vcc = padded R, 256-source tiles) or as a second tensor-core
+  // MMA (vcc = 0).  Split-FP16 crossover measured at M = N = 65,536 (tools/vsweep.py, DESIGN.md
+  // SS7): the tensor-core V costs the same for any R, the CUDA-core V grows with R -- CUDA cores
+  // for R <= 4, and for R <= 8 when K > 48; TF32 modes keep CUDA cores up to R = 16.
+  // KS_TC_VCC=0 / 1 forces the tensor-core / CUDA-core (R <= 16) variant (measurement knob).
   const char* ev = getenv("KS_TC_VCC");
-  const int vcc = (ev && ev[0] == '0') ? 0 : ks::fused_tc_rv(R);
+  int vcc = ks::fused_tc_rv(R);
+  if (f16 && (R > 8 || (R > 4 && K <= 48))) vcc = 0;
+  if (ev && ev[0] == '0') vcc = 0;
+  if (ev && ev[0] == '1') vcc = ks::fused_tc_rv(R);
   // R = 1 with W >= 0: log-weights in na (decided on the device, no host sync);
   // KS_TC_LOGW=0 disables (measurement knob)
   const char* elw = getenv("KS_TC_LOGW");

@@ -126,11 +126,12 @@ def test_cfg4_full_size_sampled(oracle_mod):
     check(oracle_mod, a, W, b, h, J=J)
 
 
-@pytest.mark.parametrize("R", [1, 16])
-def test_tensor_core_v_path(oracle_mod, monkeypatch, R):
-    """R <= 16 takes the CUDA-core weighted sum by default; KS_TC_VCC=0 keeps
-    the second (P x W) tcgen05 MMA of the R > 16 path on these shapes too."""
-    monkeypatch.setenv("KS_TC_VCC", "0")
+@pytest.mark.parametrize("R,force", [(1, "0"), (4, "0"), (16, "0"), (8, "1"), (16, "1")])
+def test_weighted_sum_variants(oracle_mod, monkeypatch, R, force):
+    """The weighted sum runs on CUDA cores (small R) or as a second (P x W) tcgen05
+    MMA (large R; the split-FP16 crossover is R > 8, or R > 4 at K <= 48).
+    KS_TC_VCC=0 / 1 forces either variant on these shapes."""
+    monkeypatch.setenv("KS_TC_VCC", force)
     a, W, b, h = workloads.custom(2100, 333, 64, R, 3.0, seed=11 + R, wkind="signed")
     check(oracle_mod, a, W, b, h)
 
