@@ -36,7 +36,6 @@ namespace ks {
 
 namespace {
 
-constexpr int kMaxStages = 6;                    // A/B ring depth bound (32 KB per stage)
 constexpr int kFlush = 4;                        // units per V accumulation block
 constexpr uint32_t kChunkA = kTcTileT * kTcKC * 4;  // one hi or lo target-operand chunk (8 KB)
 // TMEM columns: S0 | S1 (P_hi written in place) | P_lo for source half 0 | half 1 | V
@@ -181,10 +180,6 @@ struct Sched {
     v0 = 0;
     if (b < Gr) { v0 = sk_start(b, Urem, Gr); v1 = sk_start(b + 1, Urem, Gr); }
     count = qw + (int)(v1 - v0);
-  }
-  __device__ void unit(int q, int64_t& tt, int& st) const {
-    if (q < qw) { tt = (int64_t)(q / n_s) * G + b; st = q % n_s; }
-    else { const int64_t v = v0 + (q - qw); tt = rem_t0 + v / n_s; st = (int)(v % n_s); }
   }
   __device__ bool first_in_block(int q, int st) const {
     return q == 0 || q == qw || st == 0 || (st % kFlush) == 0;
