@@ -131,8 +131,9 @@ KS_API ks_status ks_eval(ks_ctx *ctx, const float *beta, int64_t N, float *V);
  * The library stages them through its own device buffers.  ks_set_sources_host
  * returns once alpha and W have been copied (the caller may reuse them); the
  * source preparation then runs on the context's stream.  ks_eval_host uploads
- * beta on a library copy stream (overlapping that preparation), evaluates, and
- * returns after V is in host memory.  Pinned host memory gives the fastest
+ * beta on a library copy stream (overlapping that preparation) in up to 4 chunks
+ * for large N, evaluating chunk c while chunk c + 1 uploads and downloading its V
+ * while chunk c + 1 evaluates, and returns after V is in host memory.  Pinned host memory gives the fastest
  * copies; pageable memory works. */
 KS_API ks_status ks_set_sources_host(ks_ctx *ctx, const float *alpha, const float *W,
                               int64_t M, int R);

@@ -112,7 +112,8 @@ struct ks_ctx {
   // host API: a copy stream for the target upload (overlaps the source prep still running on
   // `stream`) and events that end the host calls once their uploads are done
   cudaStream_t copy_stream = nullptr;
-  cudaEvent_t ev_copied = nullptr, ev_beta = nullptr;
+  cudaEvent_t ev_copied = nullptr;
+  cudaEvent_t ev_bc[4] = {}, ev_v[4] = {};  // chunked ks_eval_host: chunk uploaded / evaluated
 
   // current sources
   bool have_src = false;
@@ -651,7 +652,10 @@ ks_status ks_destroy(ks_ctx* ctx) {
   ctx->h_V.release();
   for (cudaEvent_t ev : ctx->ev) cudaEventDestroy(ev);
   if (ctx->ev_copied) cudaEventDestroy(ctx->ev_copied);
-  if (ctx->ev_beta) cudaEventDestroy(ctx->ev_beta);
+  for (int c = 0; c < 4; ++c) {
+    if (ctx->ev_bc[c]) cudaEventDestroy(ctx->ev_bc[c]);
+    if (ctx->ev_v[c]) cudaEventDestroy(ctx->ev_v[c]);
+  }
   if (ctx->copy_stream) {
     cudaStreamSynchronize(ctx->copy_stream);
     cudaStreamDestroy(ctx->copy_stream);
@@ -743,7 +747,10 @@ ks_status host_api_init(ks_ctx* ctx) {
   if (ctx->copy_stream) return KS_OK;
   KS_CUDA(cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking), "create copy stream");
   KS_CUDA(cudaEventCreateWithFlags(&ctx->ev_copied, cudaEventDisableTiming), "create event");
-  KS_CUDA(cudaEventCreateWithFlags(&ctx->ev_beta, cudaEventDisableTiming), "create event");
+  for (int c = 0; c < 4; ++c) {
+    KS_CUDA(cudaEventCreateWithFlags(&ctx->ev_bc[c], cudaEventDisableTiming), "create event");
+    KS_CUDA(cudaEventCreateWithFlags(&ctx->ev_v[c], cudaEventDisableTiming), "create event");
+  }
   return KS_OK;
 }
 }  // namespace
@@ -786,14 +793,49 @@ ks_status ks_eval_host(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   if (s != KS_OK) return s;
   KS_CUDA(ctx->h_beta.reserve(nb, ctx->stream, false), "allocate beta staging");
   KS_CUDA(ctx->h_V.reserve(nv, ctx->stream, false), "allocate V staging");
-  // the upload runs on the copy stream (overlapping a source prep still in flight on `stream`;
-  // the staging buffer's previous readers finished before the previous ks_eval_host returned)
-  KS_CUDA(cudaMemcpyAsync(ctx->h_beta.p, beta, nb * 4, cudaMemcpyHostToDevice, ctx->copy_stream), "copy beta H2D");
-  KS_CUDA(cudaEventRecord(ctx->ev_beta, ctx->copy_stream), "cudaEventRecord");
-  KS_CUDA(cudaStreamWaitEvent(ctx->stream, ctx->ev_beta, 0), "cudaStreamWaitEvent");
-  s = ks_eval(ctx, ctx->h_beta.p, N, ctx->h_V.p);
-  if (s != KS_OK) return s;
-  KS_CUDA(cudaMemcpyAsync(V, ctx->h_V.p, nv * 4, cudaMemcpyDeviceToHost, ctx->stream), "copy V D2H");
+  // The uploads run on the copy stream (overlapping a source prep still in flight on `stream`;
+  // the staging buffer's previous readers finished before the previous ks_eval_host returned).
+  // Large N: up to 4 chunks of >= half a wave of 128-target tiles each; chunk c is evaluated
+  // while chunk c + 1 uploads and its V downloads while chunk c + 1 evaluates (KS_EVAL_CHUNKS=n
+  // forces n; measured at cfg3, same box: 1 / 2 / 3 / 4 chunks 1.455 / 1.383 / 1.386 / 1.363 ms
+  // per host-API step).
+  const char* ec = getenv("KS_EVAL_CHUNKS");
+  const int64_t half_wave = (int64_t)ctx->num_sms * 64;
+  int nch = (int)(N / half_wave);
+  if (ec && ec[0] >= '1' && ec[0] <= '4') nch = ec[0] - '0';
+  if (nch > 4) nch = 4;
+  if (nch < 1) nch = 1;
+  int64_t off[4] = {0, 0, 0, 0}, cnt[4] = {0, 0, 0, 0};
+  {
+    const int64_t per = round_up((N + nch - 1) / nch, 128);
+    int64_t o = 0;
+    for (int c = 0; c < nch; ++c) {
+      off[c] = o;
+      cnt[c] = (N - o < per) ? N - o : per;
+      o += cnt[c];
+    }
+  }
+  cudaEvent_t* evb = ctx->ev_bc;
+  const int K = ctx->K, R = ctx->R;
+  for (int c = 0; c < nch; ++c) {
+    if (cnt[c] == 0) continue;
+    KS_CUDA(cudaMemcpyAsync(ctx->h_beta.p + off[c] * K, beta + off[c] * K, (size_t)cnt[c] * K * 4,
+                            cudaMemcpyHostToDevice, ctx->copy_stream),
+            "copy beta H2D");
+    KS_CUDA(cudaEventRecord(evb[c], ctx->copy_stream), "cudaEventRecord");
+  }
+  for (int c = 0; c < nch; ++c) {
+    if (cnt[c] == 0) continue;
+    KS_CUDA(cudaStreamWaitEvent(ctx->stream, evb[c], 0), "cudaStreamWaitEvent");
+    s = ks_eval(ctx, ctx->h_beta.p + off[c] * K, cnt[c], ctx->h_V.p + off[c] * R);
+    if (s != KS_OK) return s;
+    KS_CUDA(cudaEventRecord(ctx->ev_v[c], ctx->stream), "cudaEventRecord");
+    KS_CUDA(cudaStreamWaitEvent(ctx->copy_stream, ctx->ev_v[c], 0), "cudaStreamWaitEvent");
+    KS_CUDA(cudaMemcpyAsync(V + off[c] * R, ctx->h_V.p + off[c] * R, (size_t)cnt[c] * R * 4,
+                            cudaMemcpyDeviceToHost, ctx->copy_stream),
+            "copy V D2H");
+  }
+  KS_CUDA(cudaStreamSynchronize(ctx->copy_stream), "synchronize");
   KS_CUDA(cudaStreamSynchronize(ctx->stream), "synchronize");
   return KS_OK;
 }

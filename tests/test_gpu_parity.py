@@ -197,6 +197,19 @@ def test_host_api_matches_device_api():
     assert np.array_equal(gpu_eval(a, W, b, h), gpu_eval(a, W, b, h, host=True))
 
 
+@pytest.mark.parametrize("N", [20000, 40000 + 77])
+def test_host_api_chunked_eval(oracle_mod, N):
+    """ks_eval_host splits a large target set into up to 4 chunks (upload of chunk c + 1 and
+    download of chunk c - 1 overlap the evaluation of chunk c); the result meets the bar and
+    matches the one-piece device evaluation to rounding (the stream-K grouping differs)."""
+    a, W, b, h = workloads.make(3, M=3000, N=N, wkind="pos")
+    Vd = gpu_eval(a, W, b, h)
+    Vh = gpu_eval(a, W, b, h, host=True)
+    assert np.max(np.abs(Vh - Vd)) <= 1e-6 * np.abs(W).sum()
+    J = workloads.sample_targets(N, 300, seed=5)
+    check(oracle_mod, a, W, b, h, J=J, V=Vh)
+
+
 def test_host_api_buffers_reusable_on_return():
     """ks_set_sources_host returns once alpha and W are uploaded (the preparation
     continues on the stream) and ks_eval_host once V is on the host: overwriting
