@@ -850,7 +850,10 @@ ks_status ks_get_info(const ks_ctx* ctx, ks_info* out) {
   out->tile_t = tc ? ks::kTcTileT : ks::kTileT;
   out->tile_s = tc ? ks::fused_tc_tile_s(ctx->tc_vcc) : ks::kTileS;
   out->num_ctas = ctx->last_grid;
-  out->stages = !ctx->k_pad ? 0 : (tc ? ks::fused_tc_stages() : ks::fused_fp32_stages(ctx->k_pad));
+  out->stages = !ctx->k_pad ? 0
+                : (tc ? ks::fused_tc_stages(ctx->tc_vcc, ctx->tc_f16 != 0, ctx->tc_f16 ? ctx->k_pad / 2 : ctx->k_pad,
+                                            ctx->r_pad >= 32 ? 32 : 16)
+                      : ks::fused_fp32_stages(ctx->k_pad));
   out->num_sms = ctx->num_sms;
   out->m = ctx->M;
   out->m_pad = ctx->m_pad;

@@ -1630,7 +1630,16 @@ size_t fused_tc_smem(int r_c) {
     default: return r_c <= 16 ? TcSmemT<5, 128, 0>::total(16) : TcSmemT<4, 128, 0>::total(32);
   }
 }
-int fused_tc_stages() { return tc_stages(16); }
+// Operand ring depth of the kernel launch_fused_tc picks (for ks_get_info): vcc = RV (0: the
+// tensor-core weighted sum), k_pad_f32 = operand row length in FP32 units, r_c of the first launch.
+// The resident-target R = 1 kernel sizes its ring at run time (up to the 4 allocated stages).
+int fused_tc_stages(int vcc, bool f16, int k_pad_f32, int r_c) {
+  if (vcc == 1) return 4;
+  if (vcc == 2 || vcc == 4 || vcc == 8) return 4;
+  if (vcc == 16) return 3;
+  if (f16 && k_pad_f32 <= 8 * kTcKC) return r_c == 16 ? 4 : 3;
+  return tc_stages(r_c);
+}
 int fused_tc_tile_s(int rv) { return rv ? 256 : kTcTileS; }
 int fused_tc_rv(int R) { return R <= 1 ? 1 : R <= 2 ? 2 : R <= 4 ? 4 : R <= 8 ? 8 : R <= 16 ? 16 : 0; }
 

@@ -182,7 +182,7 @@ cudaError_t launch_prep_wcat(const float* W, int64_t M, int64_t m_pad, int R, in
                              unsigned* counter, unsigned* wcol, void* wcat, cudaStream_t st);
 // maps: A_hi, A_lo (targets), B_hi, B_lo (sources), W_hi, W_lo (weights^T)
 cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream_t st);
-int fused_tc_stages();
+int fused_tc_stages(int vcc, bool f16, int k_pad_f32, int r_c);
 int fused_tc_tile_s(int rv);  // sources per tile: 256 with the CUDA-core weighted sum, 128 otherwise
 int fused_tc_rv(int R);       // padded weight columns of the CUDA-core weighted sum, 0 if R > 16
 size_t fused_tc_smem(int r_c);
