@@ -56,7 +56,7 @@ typedef enum {
 } ks_status;
 
 typedef enum {
-  KS_PREC_AUTO = 0,     /* 3XF16; FP32 path if K <= 32, R == 1, M <= 4096    */
+  KS_PREC_AUTO = 0,     /* 3XF16 (the tcgen05 path) for every shape          */
   KS_PREC_FP32 = 1,     /* FP32 FFMA2 contraction (K <= 32, R == 1)          */
   KS_PREC_3XTF32 = 2,   /* tcgen05 tensor cores, TF32 hi/lo split, 3 products */
   KS_PREC_TF32 = 3,     /* tcgen05 tensor cores, single TF32 product         */

@@ -687,11 +687,12 @@ ks_status ks_set_sources(ks_ctx* ctx, const float* alpha, const float* W, int64_
   int prec = ctx->prec_req;
   int path;
   if (prec == KS_PREC_AUTO) {
-    // Measured on B200 (SS7): the tcgen05 3xTF32 kernel is faster for
-    // every configuration except tiny source sets (M <= 4096, K <= 32, R == 1),
-    // where the FP32 kernel's lower fixed cost wins.
-    path = (ctx->K <= 32 && R == 1 && M <= 4096) ? KS_PATH_FP32 : KS_PATH_TC;
-    prec = (path == KS_PATH_FP32) ? KS_PREC_FP32 : KS_PREC_3XF16;
+    // Measured on B200 (tools/msweep.py, SS7): the tcgen05 split-FP16 kernel is
+    // faster for every source-set size once the target set is not tiny (M = 512, N = 65,536:
+    // 0.044 vs 0.078 ms for set_sources + eval); the FP32 kernel only wins by ~8% when both
+    // sets are ~1,000 points, and N is unknown here -- so AUTO is always the tensor-core path.
+    path = KS_PATH_TC;
+    prec = KS_PREC_3XF16;
   } else if (prec == KS_PREC_FP32) {
     if (ctx->K > 32 || R != 1)
       return fail(KS_EUNSUPPORTED, "FP32 path needs K <= 32 and R == 1 (K=%d, R=%d)", ctx->K, R);
