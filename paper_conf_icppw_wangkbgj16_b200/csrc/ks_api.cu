@@ -386,8 +386,12 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   const bool use_wstat = (vcc == 1) && !(elw && elw[0] == '0');
   // FP16, R = 1: folded layout (norms + log-weights as 6 extra hi-plane K columns, reading
   // Q26; active on the device when c K amax^2 <= 2^12).  KS_TC_FOLD=0 disables (measurement knob)
+  // Measured (tools/fsweep.py, profiles/r01/policy_sweeps.txt): the fold pays up to K = 48 even
+  // when its columns need an operand chunk of their own, and costs ~1-4% beyond that when they do
+  // (K = 64, 96, 128, ...) -- then the norms stay in the epilogue.
   const char* efo = getenv("KS_TC_FOLD");
-  const int fold = (f16 && use_wstat && !(efo && efo[0] == '0')) ? 1 : 0;
+  const bool fold_fits = K <= 48 || round_up(K + 6, 2 * ks::kTcKC) == round_up(K, 2 * ks::kTcKC);
+  const int fold = (f16 && use_wstat && !(efo && efo[0] == '0') && (fold_fits || (efo && efo[0] == '1'))) ? 1 : 0;
   // k_pad in elements: one 64-byte row chunk per pipeline stage = 16 FP32 or 32 FP16
   const int k_pad = f16 ? (int)round_up(K + 6 * fold, 2 * ks::kTcKC) : tc_k_pad(K);
   const int aug = f16 ? 0 : tc_aug(K);  // FP16 mode: norms stay in FP32 in the epilogue (or fold)

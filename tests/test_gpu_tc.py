@@ -242,6 +242,17 @@ def test_r1_folded_norm_columns_placement(oracle_mod, K):
     check(oracle_mod, a, W, b, h)
 
 
+@pytest.mark.parametrize("K", [64, 100, 250])
+def test_r1_fold_policy_and_forced(oracle_mod, monkeypatch, K):
+    """Beyond K = 48 the norms are folded only when their six columns fit the last operand
+    chunk (K = 100: yes; K = 64, 250: no, measured 1-4% slower); KS_TC_FOLD=1 forces the fold.
+    Both layouts meet the bar."""
+    a, W, b, h = workloads.custom(1700, 500, K, 1, 0.3 * np.sqrt(K), wkind="pos", seed=300 + K)
+    check(oracle_mod, a, W, b, h)
+    monkeypatch.setenv("KS_TC_FOLD", "1")
+    check(oracle_mod, a, W, b, h)
+
+
 def test_r1_fold_inactive_for_wide_spread(oracle_mod):
     """c K amax^2 > 2^12 (h = 0.01 on the unit cube, K = 4): the folded layout
     is switched off on the device (the FP16 norm pieces would not hold the
