@@ -139,6 +139,42 @@ KS_API ks_status ks_set_sources_host(ks_ctx *ctx, const float *alpha, const floa
                               int64_t M, int R);
 KS_API ks_status ks_eval_host(ks_ctx *ctx, const float *beta, int64_t N, float *V);
 
+/* Tuning options.  Each selects among kernel variants that compute the same result
+ * within the path's tolerance (SS3-SS4); none drops work.  Defaults are the
+ * measured choices (SS7).  [sources] options take effect at the next
+ * ks_set_sources, [eval] ones at the next ks_eval.  The environment variable named
+ * beside an option, when set at ks_create, gives its initial value (read once there;
+ * later calls never read the environment). */
+typedef enum {
+  KS_OPT_R1_KERNEL = 1,       /* KS_R1: 1 (default) the dedicated R = 1 kernel where it applies
+                                 (split-FP16, K <= 58), 0 the general tcgen05 kernel [sources] */
+  KS_OPT_R1_EPILOGUE = 2,     /* KS_R1_MODE: 0 (default) log-weights when every W_i >= 0 (no
+                                 d^2 >= 0 clamp; any W_i < 0 takes mode 1), 1 weights with the
+                                 d^2 >= 0 clamp, 2 weights with d^2 -> |d^2|, 3 weights without
+                                 a clamp [sources] */
+  KS_OPT_EXP_POLY = 3,        /* KS_R1_POLY: exponential pairs of every 16 computed on the FMA
+                                 pipe instead of MUFU (0, 4..8; -1 default) [eval] */
+  KS_OPT_WEIGHTED_SUM = 4,    /* KS_TC_VCC: -1 auto, 0 tensor cores, 1 CUDA cores (R <= 16) [sources] */
+  KS_OPT_LOG_WEIGHTS = 5,     /* KS_TC_LOGW: general kernel, R = 1: 1 (default) / 0 [sources] */
+  KS_OPT_FOLD = 6,            /* KS_TC_FOLD: general kernel, R = 1: -1 auto, 0 off, 1 forced [sources] */
+  KS_OPT_AUG = 7,             /* KS_TC_AUG: TF32 modes: -1 auto, 0, 1 norms in 2 K columns [sources] */
+  KS_OPT_CLAMP = 8,           /* KS_TC_CLAMP: general kernel's log-weight epilogue: 0 (default),
+                                 1 exact d^2 >= 0 clamp [eval] */
+  KS_OPT_TARGET_RESIDENT = 9, /* KS_TC_ARES: general kernel: 1 (default) / 0 [eval] */
+  KS_OPT_STAGES = 10,         /* KS_TC_STAGES: general kernel operand ring: 0 default, 3..5 [eval] */
+  KS_OPT_AR_STAGES = 11,      /* KS_TC_AR_STAGES: 4 (default) / 5 [eval] */
+  KS_OPT_WSLOTS = 12,         /* KS_TC_WSLOTS: 0 default, 2..4 [eval] */
+  KS_OPT_PREP_LANES = 13,     /* KS_PREP_G: lanes per point in the prep kernels: 0 auto, 4, 8,
+                                 16, 32 [sources, eval] */
+  KS_OPT_EVAL_CHUNKS = 14,    /* KS_EVAL_CHUNKS: ks_eval_host target chunks: 0 auto, 1..4 [eval] */
+  KS_OPT_FP32_SPLIT = 15,     /* KS_FP32_SPLIT: FP32 kernel tile body: -1 auto, 0, 1 [eval] */
+  KS_OPT_COUNT_ = 16
+} ks_option;
+
+/* Set / read a tuning option.  KS_EINVAL for an unknown option or a value out of its range. */
+KS_API ks_status ks_set_option(ks_ctx *ctx, ks_option opt, int value);
+KS_API ks_status ks_get_option(const ks_ctx *ctx, ks_option opt, int *value);
+
 /* Pre-size the scratch for targets up to N_max so later ks_eval calls never
  * allocate (useful before CUDA-graph capture).  KS_EINVAL if N_max < 0. */
 KS_API ks_status ks_reserve(ks_ctx *ctx, int64_t N_max);

@@ -19,7 +19,9 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libks.so")
+# KS_LIB=libks_dbg.so selects a measurement build (KS_DEBUG / KS_PROF, tools only); the
+# shipped library is libks.so
+LIB_PATH = os.path.join(_HERE, os.path.basename(os.environ.get("KS_LIB", "libks.so")))
 
 KS_OK, KS_EINVAL, KS_ESTATE, KS_ENOMEM, KS_ECUDA, KS_EUNSUPPORTED = range(6)
 KS_PREC_AUTO, KS_PREC_FP32, KS_PREC_3XTF32, KS_PREC_TF32, KS_PREC_3XF16 = range(5)
@@ -30,7 +32,12 @@ PRECISIONS = {"auto": KS_PREC_AUTO, "fp32": KS_PREC_FP32, "3xtf32": KS_PREC_3XTF
 # every symbol include/ks.h declares (checked by tests/test_abi.py)
 EXPORTED = ("ks_create", "ks_destroy", "ks_set_precision", "ks_set_stream", "ks_set_sources", "ks_eval",
             "ks_set_sources_host", "ks_eval_host", "ks_reserve", "ks_get_info", "ks_timing_enable",
-            "ks_timing_read", "ks_status_str", "ks_last_error", "ks_version")
+            "ks_timing_read", "ks_set_option", "ks_get_option", "ks_status_str", "ks_last_error", "ks_version")
+
+# tuning options (include/ks.h ks_option): variants computing the same result, none drops work
+OPTIONS = {"r1_kernel": 1, "r1_epilogue": 2, "exp_poly": 3, "weighted_sum": 4, "log_weights": 5, "fold": 6,
+           "aug": 7, "clamp": 8, "target_resident": 9, "stages": 10, "ar_stages": 11, "wslots": 12,
+           "prep_lanes": 13, "eval_chunks": 14, "fp32_split": 15}
 
 
 class KsInfo(ctypes.Structure):
@@ -70,6 +77,8 @@ def _load():
         "ks_get_info": ([P, ctypes.POINTER(KsInfo)], I),
         "ks_timing_enable": ([P, I], I),
         "ks_timing_read": ([P, ctypes.POINTER(D), ctypes.POINTER(L), I], I),
+        "ks_set_option": ([P, I, I], I),
+        "ks_get_option": ([P, I, ctypes.POINTER(I)], I),
         "ks_status_str": ([I], ctypes.c_char_p),
         "ks_last_error": ([], ctypes.c_char_p),
         "ks_version": ([], ctypes.c_char_p),
@@ -167,6 +176,20 @@ def ks_get_info(ctx) -> dict:
     return info.as_dict()
 
 
+def ks_set_option(ctx, opt, value: int) -> None:
+    if isinstance(opt, str):
+        opt = OPTIONS[opt]
+    _check(_lib.ks_set_option(ctx, int(opt), int(value)), "ks_set_option")
+
+
+def ks_get_option(ctx, opt) -> int:
+    if isinstance(opt, str):
+        opt = OPTIONS[opt]
+    v = ctypes.c_int()
+    _check(_lib.ks_get_option(ctx, int(opt), ctypes.byref(v)), "ks_get_option")
+    return v.value
+
+
 def ks_timing_enable(ctx, on: bool) -> None:
     _check(_lib.ks_timing_enable(ctx, 1 if on else 0), "ks_timing_enable")
 
@@ -188,7 +211,7 @@ class KernelSum:
     CPU tensors and include the host<->device copies.
     """
 
-    def __init__(self, K: int, h: float, precision: str = "auto"):
+    def __init__(self, K: int, h: float, precision: str = "auto", options: dict | None = None):
         import torch
         load()
         self._torch = torch
@@ -196,10 +219,19 @@ class KernelSum:
             raise RuntimeError("KernelSum needs a CUDA device (no CPU fallback)")
         self.K = int(K)
         self.h = float(h)
+        self.device = torch.cuda.current_device()
         self.ctx = ks_create(self.K, self.h)
         ks_set_precision(self.ctx, precision)
+        for k, v in (options or {}).items():
+            ks_set_option(self.ctx, k, v)
         self.R = 1
         self.M = 0
+
+    def set_option(self, name, value: int):
+        ks_set_option(self.ctx, name, value)
+
+    def get_option(self, name) -> int:
+        return ks_get_option(self.ctx, name)
 
     def close(self):
         if getattr(self, "ctx", None):
@@ -221,23 +253,33 @@ class KernelSum:
     def _stream(self):
         ks_set_stream(self.ctx, self._torch.cuda.current_stream().cuda_stream)
 
-    def _dev(self, t, name, shape1):
+    def _dev(self, t, name, shape1, rows=None):
         torch = self._torch
         if not isinstance(t, torch.Tensor) or not t.is_cuda or t.dtype != torch.float32:
             raise TypeError(f"{name} must be a CUDA float32 tensor")
+        if t.device.index != self.device:
+            raise ValueError(f"{name} is on cuda:{t.device.index}, the context on cuda:{self.device}")
         if not t.is_contiguous():
             raise ValueError(f"{name} must be contiguous")
-        if t.dim() != 2 or t.shape[1] != shape1:
-            raise ValueError(f"{name} must be [n, {shape1}], got {tuple(t.shape)}")
+        if t.dim() != 2 or t.shape[1] != shape1 or (rows is not None and t.shape[0] != rows):
+            want = f"[{'n' if rows is None else rows}, {shape1}]"
+            raise ValueError(f"{name} must be {want}, got {tuple(t.shape)}")
         return t
+
+    @staticmethod
+    def _host(x, name, shape1, rows=None):
+        import numpy as np
+        a = np.ascontiguousarray(x, dtype=np.float32)
+        if a.ndim != 2 or a.shape[1] != shape1 or (rows is not None and a.shape[0] != rows):
+            want = f"[{'n' if rows is None else rows}, {shape1}]"
+            raise ValueError(f"{name} must be {want}, got {tuple(a.shape)}")
+        return a
 
     def set_sources(self, alpha, W):
         if W.dim() == 1:
             W = W.reshape(-1, 1)
         alpha = self._dev(alpha, "alpha", self.K)
-        W = self._dev(W, "W", W.shape[1])
-        if W.shape[0] != alpha.shape[0]:
-            raise ValueError("alpha and W must have the same number of rows")
+        W = self._dev(W, "W", W.shape[1], rows=alpha.shape[0])
         self._stream()
         ks_set_sources(self.ctx, alpha.data_ptr(), W.data_ptr(), alpha.shape[0], W.shape[1])
         self.M, self.R = alpha.shape[0], W.shape[1]
@@ -249,26 +291,30 @@ class KernelSum:
         if out is None:
             out = self._torch.empty((N, self.R), dtype=self._torch.float32, device=beta.device)
         else:
-            out = self._dev(out, "out", self.R)
+            out = self._dev(out, "out", self.R, rows=N)
         self._stream()
         ks_eval(self.ctx, beta.data_ptr(), N, out.data_ptr())
         return out
 
     def set_sources_host(self, alpha, W):
         import numpy as np
-        a = np.ascontiguousarray(alpha, dtype=np.float32)
-        w = np.ascontiguousarray(W, dtype=np.float32)
+        a = self._host(alpha, "alpha", self.K)
+        w = np.asarray(W, dtype=np.float32)
         if w.ndim == 1:
             w = w[:, None]
+        w = self._host(w, "W", w.shape[1] if w.ndim == 2 else -1, rows=a.shape[0])
         self._stream()
         ks_set_sources_host(self.ctx, a.ctypes.data, w.ctypes.data, a.shape[0], w.shape[1])
         self.M, self.R = a.shape[0], w.shape[1]
 
     def eval_host(self, beta, out=None):
         import numpy as np
-        b = np.ascontiguousarray(beta, dtype=np.float32)
+        b = self._host(beta, "beta", self.K)
         if out is None:
             out = np.empty((b.shape[0], self.R), dtype=np.float32)
+        elif (not isinstance(out, np.ndarray) or out.dtype != np.float32 or out.shape != (b.shape[0], self.R)
+              or not out.flags["C_CONTIGUOUS"]):
+            raise ValueError(f"out must be a C-contiguous float32 array of shape {(b.shape[0], self.R)}")
         self._stream()
         ks_eval_host(self.ctx, b.ctypes.data, b.shape[0], out.ctypes.data)
         return out

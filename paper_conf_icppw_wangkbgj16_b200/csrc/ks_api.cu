@@ -23,6 +23,10 @@
 #include "../../include/ks.h"
 #include "ks_internal.h"
 
+#ifndef KS_DEBUG
+#define KS_DEBUG 0
+#endif
+
 namespace {
 
 thread_local std::string g_err;
@@ -114,6 +118,8 @@ struct ks_ctx {
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t ev_copied = nullptr;
   cudaEvent_t ev_bc[4] = {}, ev_v[4] = {};  // chunked ks_eval_host: chunk uploaded / evaluated
+  cudaEvent_t ev_stream = nullptr;          // ks_set_stream: new stream waits for the old one
+  int64_t reserve_n = 0;                    // ks_reserve: target count the scratch is sized for
 
   // current sources
   bool have_src = false;
@@ -135,6 +141,8 @@ struct ks_ctx {
   int tc_fold = 0;  // FP16 R = 1 folded layout (6 extra hi-plane K columns)
   int tc_kcols = 0, tc_kdims = 0;  // live operand columns / columns needing every split product
   int tc_vcc = 0;  // RV: weighted sum on CUDA cores over RV padded columns (0: tensor-core V path)
+  int r1 = 0;      // R = 1 folded kernel (ks_fused_r1.cu): 2 = log-weight mode allowed, 3 = weight mode only
+  int r1_clamp = 0;
   CUtensorMap tmB_hi, tmB_lo;
   DBuf<float> mu;         // [k_pad]
   DBuf<double> mean_part; // [nparts][K]
@@ -153,6 +161,11 @@ struct ks_ctx {
   // host staging (ks_*_host)
   DBuf<float> h_alpha, h_W, h_beta, h_V;
 
+  // tuning options (ks_set_option; initial values from the environment at ks_create) and the
+  // debug trace file (KS_CTA_TIMES, read at ks_create)
+  ks::Opts opts;
+  std::string cta_times_path;
+
   // accounting / timing
   int64_t launches = 0, fused_launches = 0;
   bool timing = false;
@@ -160,7 +173,56 @@ struct ks_ctx {
   size_t ev_used = 0;           // pairs in use
 };
 
+namespace ks {
+thread_local const Opts* tl_opts = nullptr;
+}
+
 namespace {
+
+// The context's options are visible to the launchers for the duration of one API call.
+struct OptScope {
+  const ks::Opts* prev;
+  explicit OptScope(const ks_ctx* ctx) : prev(ks::tl_opts) { ks::tl_opts = &ctx->opts; }
+  ~OptScope() { ks::tl_opts = prev; }
+};
+
+struct OptSpec {
+  const char* env;
+  int dflt, lo, hi;
+};
+// [option id] = {environment variable, default, valid range}
+const OptSpec kOpt[KS_OPT_COUNT_] = {
+    {nullptr, 0, 0, 0},
+    {"KS_R1", 1, 0, 1},
+    {"KS_R1_MODE", 0, 0, 3},
+    {"KS_R1_POLY", -1, -1, 8},
+    {"KS_TC_VCC", -1, -1, 1},
+    {"KS_TC_LOGW", 1, 0, 1},
+    {"KS_TC_FOLD", -1, -1, 1},
+    {"KS_TC_AUG", -1, -1, 1},
+    {"KS_TC_CLAMP", 0, 0, 1},
+    {"KS_TC_ARES", 1, 0, 1},
+    {"KS_TC_STAGES", 0, 0, 5},
+    {"KS_TC_AR_STAGES", 4, 4, 5},
+    {"KS_TC_WSLOTS", 0, 0, 4},
+    {"KS_PREP_G", 0, 0, 32},
+    {"KS_EVAL_CHUNKS", 0, 0, 4},
+    {"KS_FP32_SPLIT", -1, -1, 1},
+};
+
+void init_opts(ks_ctx* ctx) {
+  for (int i = 0; i < KS_OPT_COUNT_; ++i) {
+    ctx->opts.v[i] = kOpt[i].dflt;
+    if (!kOpt[i].env) continue;
+    const char* e = getenv(kOpt[i].env);
+    if (!e || !*e) continue;
+    char* end = nullptr;
+    const long v = strtol(e, &end, 10);
+    if (end != e && v >= kOpt[i].lo && v <= kOpt[i].hi) ctx->opts.v[i] = (int)v;
+  }
+  const char* t = getenv("KS_CTA_TIMES");
+  if (t && *t) ctx->cta_times_path = t;
+}
 
 ks_status check_ctx(const ks_ctx* ctx) {
   if (!ctx) return fail(KS_EINVAL, "ctx is NULL");
@@ -277,9 +339,9 @@ ks_status eval_fp32(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.counters = ctx->counters.p;
   a.sk = sk;
   a.cta_times = nullptr;
-  // debug knob: KS_CTA_TIMES=<file> appends per-CTA start/end globaltimer (ns) of each launch
-  const char* dbg = getenv("KS_CTA_TIMES");
-  if (dbg && *dbg) {
+  // debug trace: KS_CTA_TIMES=<file> (at ks_create) appends per-CTA start/end globaltimer (ns)
+  const char* dbg = ctx->cta_times_path.empty() ? nullptr : ctx->cta_times_path.c_str();
+  if (dbg) {
     KS_CUDA(ctx->dbg_times.reserve((size_t)sk.grid * 2, st, true), "allocate debug timers");
     a.cta_times = ctx->dbg_times.p;
   }
@@ -361,8 +423,8 @@ ks_status encode_wcat(CUtensorMap* map, const void* base, int64_t m_pad, int r_p
 // Fold the norms into the MMA (two extra K columns) when that costs no extra K chunk.
 // KS_TC_AUG=0/1 overrides (measurement knob).
 int tc_aug(int K) {
-  const char* e = getenv("KS_TC_AUG");
-  if (e && (e[0] == '0' || e[0] == '1')) return e[0] - '0';
+  const int o = ks::opt(KS_OPT_AUG, -1);
+  if (o == 0 || o == 1) return o;
   return (round_up(K + 2, ks::kTcKC) == round_up(K, ks::kTcKC)) ? 1 : 0;  // measured: an extra chunk costs more than it saves
 }
 int tc_k_pad(int K) { return (int)round_up(K + 2 * tc_aug(K), ks::kTcKC); }
@@ -374,28 +436,40 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   // MMA (vcc = 0).  Split-FP16 crossover measured at M = N = 65,536 (tools/vsweep.py, DESIGN.md
   // SS7): the tensor-core V costs the same for any R, the CUDA-core V grows with R -- CUDA cores
   // for R <= 4, and for R <= 8 when K > 48; TF32 modes keep CUDA cores up to R = 16.
-  // KS_TC_VCC=0 / 1 forces the tensor-core / CUDA-core (R <= 16) variant (measurement knob).
-  const char* ev = getenv("KS_TC_VCC");
+  // KS_OPT_WEIGHTED_SUM = 0 / 1 forces the tensor-core / CUDA-core (R <= 16) variant.
+  const int ovs = ks::opt(KS_OPT_WEIGHTED_SUM, -1);
   int vcc = ks::fused_tc_rv(R);
   if (f16 && (R > 8 || (R > 4 && K <= 48))) vcc = 0;
-  if (ev && ev[0] == '0') vcc = 0;
-  if (ev && ev[0] == '1') vcc = ks::fused_tc_rv(R);
+  if (ovs == 0) vcc = 0;
+  if (ovs == 1) vcc = ks::fused_tc_rv(R);
   // R = 1 with W >= 0: log-weights in na (decided on the device, no host sync);
-  // KS_TC_LOGW=0 disables (measurement knob)
-  const char* elw = getenv("KS_TC_LOGW");
-  const bool use_wstat = (vcc == 1) && !(elw && elw[0] == '0');
+  // KS_OPT_LOG_WEIGHTS = 0 disables (general kernel)
+  const bool use_wstat = (vcc == 1) && ks::opt(KS_OPT_LOG_WEIGHTS, 1) != 0;
   // FP16, R = 1: folded layout (norms + log-weights as 6 extra hi-plane K columns, reading
   // Q26; active on the device when c K amax^2 <= 2^12).  KS_TC_FOLD=0 disables (measurement knob)
   // Measured (tools/fsweep.py, profiles/r01/policy_sweeps.txt): the fold pays up to K = 48 even
   // when its columns need an operand chunk of their own, and costs ~1-4% beyond that when they do
   // (K = 64, 96, 128, ...) -- then the norms stay in the epilogue.
-  const char* efo = getenv("KS_TC_FOLD");
+  const int ofo = ks::opt(KS_OPT_FOLD, -1);
   const bool fold_fits = K <= 48 || round_up(K + 6, 2 * ks::kTcKC) == round_up(K, 2 * ks::kTcKC);
-  const int fold = (f16 && use_wstat && !(efo && efo[0] == '0') && (fold_fits || (efo && efo[0] == '1'))) ? 1 : 0;
+  int fold = (f16 && use_wstat && ofo != 0 && (fold_fits || ofo == 1)) ? 1 : 0;
+  // R = 1, split-FP16, K + 6 <= 64: the dedicated folded kernel (ks_fused_r1.cu;
+  // KS_OPT_R1_KERNEL = 0 selects the general kernel), fold mode 2 (always folded, fold shift,
+  // reading Q28).  KS_OPT_R1_EPILOGUE: 0 = log-weights when every W_i >= 0 (decided on the
+  // device), else the weight mode with the clamp; 1 = weight mode with the d^2 >= 0 clamp for any
+  // W; 2 = weight mode with |d^2|; 3 = weight mode without a clamp.
+  int r1 = 0, r1_clamp = 0;
+  if (f16 && vcc == 1 && K + 6 <= 2 * 2 * ks::kTcKC && ks::opt(KS_OPT_R1_KERNEL, 1) != 0) {
+    const int mode = ks::opt(KS_OPT_R1_EPILOGUE, 0);
+    r1 = mode == 0 ? 2 : 3;
+    r1_clamp = mode == 3 ? 0 : mode == 2 ? 2 : 1;
+    fold = r1;
+  }
   // k_pad in elements: one 64-byte row chunk per pipeline stage = 16 FP32 or 32 FP16
-  const int k_pad = f16 ? (int)round_up(K + 6 * fold, 2 * ks::kTcKC) : tc_k_pad(K);
+  const int k_pad = f16 ? (int)round_up(K + 6 * (fold ? 1 : 0), 2 * ks::kTcKC) : tc_k_pad(K);
   const int aug = f16 ? 0 : tc_aug(K);  // FP16 mode: norms stay in FP32 in the epilogue (or fold)
   const int tile_s = ks::fused_tc_tile_s(vcc);
+  const int box_s = r1 ? 128 : tile_s;  // sources per operand tile of the kernel
   const int64_t m_pad = round_up(M > 0 ? M : 1, tile_s);
   const int r_pad = (int)round_up(R, 16);
   cudaStream_t st = ctx->stream;
@@ -408,8 +482,9 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(ctx->wv.reserve((size_t)m_pad * (vcc ? vcc : 1), st, false), "allocate W rows");
   KS_CUDA(ctx->mu.reserve(k_pad, st, false), "allocate mean buffer");
   // mean, max |alpha - mu| (FP16 scaling) and the R = 1 weight statistics in one launch
-  KS_CUDA(source_stats(ctx, alpha, W, use_wstat, M, k_pad, f16), "source statistics");
-  const unsigned* wst = use_wstat ? ctx->wstat.p : nullptr;
+  const bool want_wstat = use_wstat || r1;  // the R = 1 kernel decides its epilogue from wstat
+  KS_CUDA(source_stats(ctx, alpha, W, want_wstat, M, k_pad, f16), "source statistics");
+  const unsigned* wst = want_wstat ? ctx->wstat.p : nullptr;
   if (f16) {
     KS_CUDA(ks::launch_prep_f16_sources(alpha, W, M, m_pad, K, k_pad, R, 0, ctx->mu.p, ctx->c,
                                         ctx->amax.p, fold, ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p,
@@ -433,20 +508,92 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
             "source prep (TC)");
   }
   ctx->launches += 1;
-  ks_status s = encode_2d_sw64(&ctx->tmB_hi, ctx->src_hi.p, k_pad, m_pad, tile_s, f16);
+  ks_status s = encode_2d_sw64(&ctx->tmB_hi, ctx->src_hi.p, k_pad, m_pad, box_s, f16);
   if (s != KS_OK) return s;
-  s = encode_2d_sw64(&ctx->tmB_lo, ctx->src_lo.p, k_pad, m_pad, tile_s, f16);
+  s = encode_2d_sw64(&ctx->tmB_lo, ctx->src_lo.p, k_pad, m_pad, box_s, f16);
   if (s != KS_OK) return s;
   ctx->k_pad = k_pad;
   ctx->m_pad = m_pad;
   ctx->r_pad = r_pad;
   ctx->tc_aug = aug;
-  ctx->tc_fold = fold;
-  ctx->tc_kcols = f16 ? K + 6 * fold : K + 2 * aug;
+  ctx->tc_fold = fold;  // 1: general kernel (device-side f16_fold_ok); 2, 3: R = 1 kernel (fold shift)
+  ctx->r1 = r1;
+  ctx->r1_clamp = r1_clamp;
+  ctx->tc_kcols = f16 ? K + 6 * (fold ? 1 : 0) : K + 2 * aug;
   ctx->tc_kdims = f16 ? K : K + 2 * aug;
   ctx->tc_vcc = vcc;
   ctx->tc_f16 = f16 ? 1 : 0;
-  ctx->tc_wstat = use_wstat;
+  ctx->tc_wstat = want_wstat;
+  return KS_OK;
+}
+
+// R = 1 folded kernel (ks_fused_r1.cu): 128-source units, one launch.
+ks_status eval_r1(ks_ctx* ctx, const CUtensorMap* maps, int64_t N, float* V) {
+  cudaStream_t st = ctx->stream;
+  ks::StreamK sk;
+  sk.n_t = round_up(N, ks::kTcTileT) / ks::kTcTileT;
+  sk.n_s = (int32_t)(ctx->m_pad / 128);
+  sk.units = sk.n_t * (int64_t)sk.n_s;
+  int64_t g = ctx->num_sms;
+  if (g > sk.units) g = sk.units;
+  sk.grid = (int32_t)g;
+  KS_CUDA(ctx->partial.reserve((size_t)sk.grid * 2 * 128, st, false), "allocate partials");
+  KS_CUDA(ctx->counters.reserve((size_t)sk.n_t, st, true), "allocate tile counters");
+  ks::R1Args a;
+  a.N = N;
+  a.n_kc = ctx->k_pad / 32;
+  a.kdims = ctx->tc_kdims;
+  a.kcols = ctx->tc_kcols;
+  a.logw = ctx->r1 == 2 ? 1 : 0;
+  a.clamp = ctx->r1_clamp;
+  a.wstat = ctx->wstat.p;
+  a.wv = ctx->wv.p;
+  a.V = V;
+  a.partial = ctx->partial.p;
+  a.counters = ctx->counters.p;
+  a.sk = sk;
+  a.cta_times = nullptr;
+  a.dbg = 0;
+#if KS_DEBUG
+  {
+    const char* e = getenv("KS_R1_DEBUG");  // measurement builds only: drops work, wrong results
+    a.dbg = e ? atoi(e) : 0;
+  }
+#endif
+  const char* dbg = ctx->cta_times_path.empty() ? nullptr : ctx->cta_times_path.c_str();
+  const size_t n_dbg = (size_t)sk.grid * (4 + 20 * 4) + 4 * 4096;  // + KS_TRACE unit clocks of CTA 0
+  if (dbg) {
+    KS_CUDA(ctx->dbg_times.reserve(n_dbg, st, true), "allocate debug timers");
+    a.cta_times = ctx->dbg_times.p;
+  }
+  cudaEvent_t stop;
+  ks_status s = timed_begin(ctx, &stop);
+  if (s != KS_OK) return s;
+  KS_CUDA(ks::launch_fused_r1(maps, a, ks::r1_poly(), st), "fused R = 1 kernel launch");
+  ctx->launches++;
+  ctx->fused_launches++;
+  ctx->last_grid = sk.grid;
+  s = timed_end(ctx, stop);
+  if (s != KS_OK) return s;
+  if (a.cta_times) {  // "r1 <cta> <t0 ns> <t1 ns> <clock0> <clock1> [20 x 4 phase clocks]" per CTA
+    std::vector<unsigned long long> h(n_dbg);
+    KS_CUDA(cudaMemcpyAsync(h.data(), a.cta_times, h.size() * 8, cudaMemcpyDeviceToHost, st), "copy debug timers");
+    KS_CUDA(cudaStreamSynchronize(st), "synchronize");
+    FILE* f = fopen(dbg, "a");
+    if (f) {
+      for (int i = 0; i < sk.grid; ++i) {
+        fprintf(f, "r1 %d %llu %llu %llu %llu", i, h[4 * i], h[4 * i + 2], h[4 * i + 1], h[4 * i + 3]);
+        for (int k = 0; k < 80; ++k) fprintf(f, " %llu", h[4 * (size_t)sk.grid + (size_t)i * 80 + k]);
+        fprintf(f, "\n");
+      }
+      const size_t t0 = (size_t)sk.grid * 84;
+      for (int q = 0; q < 4096 && h[t0 + 4 * q] != 0; ++q)
+        fprintf(f, "trace %d %llu %llu %llu %llu\n", q, h[t0 + 4 * q], h[t0 + 4 * q + 1], h[t0 + 4 * q + 2],
+                h[t0 + 4 * q + 3]);
+      fprintf(f, "--\n");
+      fclose(f);
+    }
+  }
   return KS_OK;
 }
 
@@ -477,6 +624,7 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   if (s != KS_OK) return s;
   maps[2] = ctx->tmB_hi;
   maps[3] = ctx->tmB_lo;
+  if (ctx->r1) return eval_r1(ctx, maps, N, V);
 
   ks::StreamK sk;
   sk.n_t = n_pad / ks::kTcTileT;
@@ -499,30 +647,29 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.aug = ctx->tc_aug;
   a.kcols = ctx->tc_kcols;
   a.kdims = ctx->tc_kdims;
-  a.fold = ctx->tc_fold;
+  a.fold = ctx->tc_fold ? 1 : 0;
   a.amax = f16 ? ctx->amax.p : nullptr;
   a.c = ctx->c;
   a.K = ctx->K;
   a.wv = ctx->wv.p;
   a.wcol = ctx->wcol.p;
   a.vcc = ctx->tc_vcc;
+  a.ares = ks::opt(KS_OPT_TARGET_RESIDENT, 1) ? 1 : 0;  // 0: reload the target operand per unit
+  a.ar_stages = ks::opt(KS_OPT_AR_STAGES, 4) == 5 ? 5 : 4;
   {
-    const char* e = getenv("KS_TC_ARES");  // measurement knob: 0 = reload the target operand per unit
-    a.ares = (e && e[0] == '0') ? 0 : 1;
-    const char* es = getenv("KS_TC_AR_STAGES");  // measurement knob: 5 = one source stage more
-    a.ar_stages = (es && es[0] == '5') ? 5 : 4;
+    const int w = ks::opt(KS_OPT_WSLOTS, 0);
+    a.wslots = (w >= 2 && w <= 4) ? w : 0;
   }
-  {
-    const char* e = getenv("KS_TC_WSLOTS");  // measurement knob
-    a.wslots = (e && e[0] >= '2' && e[0] <= '4') ? (e[0] - '0') : 0;
-  }
+  a.dbg_skip_v = 0;
+#if KS_DEBUG
   {
     const char* e = getenv("KS_TC_DEBUG_SKIP_V");
-    // 1 no epilogue math, 4 W/na loaded once, 5 no S MMAs, 6 one product, 7 no MMAs and no operand
-    // loads, 8 = 1 + 5, 9 = 1 + no operand loads, 10 = 1 + 7 (measurement only: wrong results)
+    // measurement builds only (wrong results): 1 no epilogue math, 4 W/na loaded once, 5 no S MMAs,
+    // 6 one product, 7 no MMAs and no operand loads, 8 = 1 + 5, 9 = 1 + no operand loads, 10 = 1 + 7
     a.dbg_skip_v = e ? atoi(e) : 0;
     if (a.dbg_skip_v < 0 || a.dbg_skip_v > 10) a.dbg_skip_v = 0;
   }
+#endif
   a.na = ctx->na.p;
   a.nb = ctx->nb.p;
   a.V = V;
@@ -530,9 +677,9 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   a.counters = ctx->counters.p;
   a.sk = sk;
   a.cta_times = nullptr;
-  const char* dbg = getenv("KS_CTA_TIMES");
+  const char* dbg = ctx->cta_times_path.empty() ? nullptr : ctx->cta_times_path.c_str();
   const size_t n_dbg = (size_t)sk.grid * (2 + 20 * 5);  // CTA start/end + (KS_PROF builds) per-warp phase clocks
-  if (dbg && *dbg) {
+  if (dbg) {
     KS_CUDA(ctx->dbg_times.reserve(n_dbg, st, true), "allocate debug timers");
     a.cta_times = ctx->dbg_times.p;
   }
@@ -580,6 +727,21 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   return KS_OK;
 }
 
+// The TC path's per-eval target buffers for ctx->reserve_n targets at the current operand
+// layout (ks_reserve; re-applied by ks_set_sources when the layout changes), so that no later
+// ks_eval with N <= reserve_n allocates (CUDA-graph capture).
+ks_status reserve_targets(ks_ctx* ctx) {
+  if (ctx->reserve_n <= 0 || !ctx->have_src || ctx->path != KS_PATH_TC) return KS_OK;
+  const int64_t n_pad = round_up(ctx->reserve_n, ks::kTcTileT);
+  const size_t ntg = ctx->tc_f16 ? ((size_t)n_pad * ctx->k_pad + 1) / 2 : (size_t)n_pad * ctx->k_pad;
+  cudaStream_t st = ctx->stream;
+  KS_CUDA(ctx->tgt_hi.reserve(ntg, st, false), "allocate target hi");
+  KS_CUDA(ctx->tgt_lo.reserve(ntg, st, false), "allocate target lo");
+  KS_CUDA(ctx->nb.reserve((size_t)n_pad, st, false), "allocate target norms");
+  KS_CUDA(ctx->tsc.reserve((size_t)n_pad, st, false), "allocate target scales");
+  return KS_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -621,6 +783,7 @@ ks_status ks_create(int K, float h, ks_ctx** out) {
   ks_ctx* ctx = new (std::nothrow) ks_ctx();
   if (!ctx) return fail(KS_ENOMEM, "host allocation of the context failed");
   ctx->device = dev;
+  init_opts(ctx);
   ctx->num_sms = prop.multiProcessorCount;
   ctx->K = K;
   ctx->h = h;
@@ -656,6 +819,7 @@ ks_status ks_destroy(ks_ctx* ctx) {
   ctx->h_V.release();
   for (cudaEvent_t ev : ctx->ev) cudaEventDestroy(ev);
   if (ctx->ev_copied) cudaEventDestroy(ctx->ev_copied);
+  if (ctx->ev_stream) cudaEventDestroy(ctx->ev_stream);
   for (int c = 0; c < 4; ++c) {
     if (ctx->ev_bc[c]) cudaEventDestroy(ctx->ev_bc[c]);
     if (ctx->ev_v[c]) cudaEventDestroy(ctx->ev_v[c]);
@@ -676,14 +840,44 @@ ks_status ks_set_precision(ks_ctx* ctx, ks_precision p) {
   return KS_OK;
 }
 
+ks_status ks_set_option(ks_ctx* ctx, ks_option o, int value) {
+  if (check_ctx(ctx)) return KS_EINVAL;
+  const int i = (int)o;
+  if (i < 1 || i >= KS_OPT_COUNT_) return fail(KS_EINVAL, "unknown option %d", i);
+  if (value < kOpt[i].lo || value > kOpt[i].hi)
+    return fail(KS_EINVAL, "option %d value %d outside [%d, %d]", i, value, kOpt[i].lo, kOpt[i].hi);
+  ctx->opts.v[i] = value;
+  return KS_OK;
+}
+
+ks_status ks_get_option(const ks_ctx* ctx, ks_option o, int* value) {
+  if (check_ctx(ctx)) return KS_EINVAL;
+  const int i = (int)o;
+  if (!value) return fail(KS_EINVAL, "value is NULL");
+  if (i < 1 || i >= KS_OPT_COUNT_) return fail(KS_EINVAL, "unknown option %d", i);
+  *value = ctx->opts.v[i];
+  return KS_OK;
+}
+
 ks_status ks_set_stream(ks_ctx* ctx, void* cuda_stream) {
   if (check_ctx(ctx)) return KS_EINVAL;
-  ctx->stream = reinterpret_cast<cudaStream_t>(cuda_stream);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(cuda_stream);
+  if (st != ctx->stream) {
+    // order the new stream after everything already enqueued on the old one (prepared sources,
+    // buffers a later growth may free), so mixing streams across calls is safe
+    ks_status s = set_device(ctx);
+    if (s != KS_OK) return s;
+    if (!ctx->ev_stream) KS_CUDA(cudaEventCreateWithFlags(&ctx->ev_stream, cudaEventDisableTiming), "create event");
+    KS_CUDA(cudaEventRecord(ctx->ev_stream, ctx->stream), "cudaEventRecord");
+    KS_CUDA(cudaStreamWaitEvent(st, ctx->ev_stream, 0), "cudaStreamWaitEvent");
+    ctx->stream = st;
+  }
   return KS_OK;
 }
 
 ks_status ks_set_sources(ks_ctx* ctx, const float* alpha, const float* W, int64_t M, int R) {
   if (check_ctx(ctx)) return KS_EINVAL;
+  OptScope opt_scope(ctx);
   if (M < 0) return fail(KS_EINVAL, "M=%lld < 0", (long long)M);
   if (R < 1 || R > 256) return fail(KS_EINVAL, "R=%d outside [1, 256]", R);
   if (M > 0 && (!alpha || !W)) return fail(KS_EINVAL, "alpha/W is NULL with M=%lld", (long long)M);
@@ -715,11 +909,12 @@ ks_status ks_set_sources(ks_ctx* ctx, const float* alpha, const float* W, int64_
   ctx->M = M;
   ctx->R = R;
   ctx->have_src = true;
-  return KS_OK;
+  return reserve_targets(ctx);
 }
 
 ks_status ks_eval(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   if (check_ctx(ctx)) return KS_EINVAL;
+  OptScope opt_scope(ctx);
   if (N < 0) return fail(KS_EINVAL, "N=%lld < 0", (long long)N);
   if (!ctx->have_src) return fail(KS_ESTATE, "ks_eval before ks_set_sources");
   if (N == 0) return KS_OK;
@@ -736,6 +931,7 @@ ks_status ks_eval(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
 
 ks_status ks_reserve(ks_ctx* ctx, int64_t N_max) {
   if (check_ctx(ctx)) return KS_EINVAL;
+  OptScope opt_scope(ctx);
   if (N_max < 0) return fail(KS_EINVAL, "N_max < 0");
   ks_status s = set_device(ctx);
   if (s != KS_OK) return s;
@@ -744,7 +940,8 @@ ks_status ks_reserve(ks_ctx* ctx, int64_t N_max) {
   const size_t per_cta = std::max((size_t)2 * ks::kTileT, (size_t)2 * ks::kTcTileT * 32);
   KS_CUDA(ctx->partial.reserve((size_t)g * per_cta, ctx->stream, false), "allocate partials");
   KS_CUDA(ctx->counters.reserve((size_t)(n_t > 0 ? n_t : 1), ctx->stream, true), "allocate tile counters");
-  return KS_OK;
+  if (N_max > ctx->reserve_n) ctx->reserve_n = N_max;
+  return reserve_targets(ctx);
 }
 
 namespace {
@@ -762,6 +959,7 @@ ks_status host_api_init(ks_ctx* ctx) {
 
 ks_status ks_set_sources_host(ks_ctx* ctx, const float* alpha, const float* W, int64_t M, int R) {
   if (check_ctx(ctx)) return KS_EINVAL;
+  OptScope opt_scope(ctx);
   if (M < 0) return fail(KS_EINVAL, "M=%lld < 0", (long long)M);
   if (R < 1 || R > 256) return fail(KS_EINVAL, "R=%d outside [1, 256]", R);
   if (M > 0 && (!alpha || !W)) return fail(KS_EINVAL, "alpha/W is NULL with M=%lld", (long long)M);
@@ -787,6 +985,7 @@ ks_status ks_set_sources_host(ks_ctx* ctx, const float* alpha, const float* W, i
 
 ks_status ks_eval_host(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   if (check_ctx(ctx)) return KS_EINVAL;
+  OptScope opt_scope(ctx);
   if (N < 0) return fail(KS_EINVAL, "N=%lld < 0", (long long)N);
   if (!ctx->have_src) return fail(KS_ESTATE, "ks_eval before ks_set_sources");
   if (N == 0) return KS_OK;
@@ -801,13 +1000,13 @@ ks_status ks_eval_host(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   // The uploads run on the copy stream (overlapping a source prep still in flight on `stream`;
   // the staging buffer's previous readers finished before the previous ks_eval_host returned).
   // Large N: up to 4 chunks of >= half a wave of 128-target tiles each; chunk c is evaluated
-  // while chunk c + 1 uploads and its V downloads while chunk c + 1 evaluates (KS_EVAL_CHUNKS=n
-  // forces n; measured at cfg3, same box: 1 / 2 / 3 / 4 chunks 1.455 / 1.383 / 1.386 / 1.363 ms
+  // while chunk c + 1 uploads and its V downloads while chunk c + 1 evaluates (KS_OPT_EVAL_CHUNKS
+  // = n forces n; measured at cfg3, same box: 1 / 2 / 3 / 4 chunks 1.455 / 1.383 / 1.386 / 1.363 ms
   // per host-API step).
-  const char* ec = getenv("KS_EVAL_CHUNKS");
+  const int och = ctx->opts.v[KS_OPT_EVAL_CHUNKS];
   const int64_t half_wave = (int64_t)ctx->num_sms * 64;
   int nch = (int)(N / half_wave);
-  if (ec && ec[0] >= '1' && ec[0] <= '4') nch = ec[0] - '0';
+  if (och >= 1 && och <= 4) nch = och;
   if (nch > 4) nch = 4;
   if (nch < 1) nch = 1;
   int64_t off[4] = {0, 0, 0, 0}, cnt[4] = {0, 0, 0, 0};
@@ -853,9 +1052,10 @@ ks_status ks_get_info(const ks_ctx* ctx, ks_info* out) {
   out->k_pad = ctx->k_pad;
   const bool tc = ctx->have_src && ctx->path == KS_PATH_TC;
   out->tile_t = tc ? ks::kTcTileT : ks::kTileT;
-  out->tile_s = tc ? ks::fused_tc_tile_s(ctx->tc_vcc) : ks::kTileS;
+  out->tile_s = tc ? (ctx->r1 ? 128 : ks::fused_tc_tile_s(ctx->tc_vcc)) : ks::kTileS;
   out->num_ctas = ctx->last_grid;
   out->stages = !ctx->k_pad ? 0
+                : tc && ctx->r1 ? ks::fused_r1_stages(ctx->K)
                 : (tc ? ks::fused_tc_stages(ctx->tc_vcc, ctx->tc_f16 != 0, ctx->tc_f16 ? ctx->k_pad / 2 : ctx->k_pad,
                                             ctx->r_pad >= 32 ? 32 : 16)
                       : ks::fused_fp32_stages(ctx->k_pad));

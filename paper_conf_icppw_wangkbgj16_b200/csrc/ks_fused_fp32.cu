@@ -391,15 +391,11 @@ __global__ void __launch_bounds__(kFp32Threads, 1)
 // Tile-body variant.  Measured on B200 (SS7): at K = 32 the split
 // halves with the interleaved epilogue are faster (76% vs 74% of the FP32
 // roofline); at K <= 16 the full 8x8 tile (half the LDS per FMA) wins.
-// KS_FP32_SPLIT=0/1 overrides (measurement knob).
+// KS_OPT_FP32_SPLIT=0/1 overrides (tuning option).
 template <int KP>
 static bool fp32_split() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("KS_FP32_SPLIT");
-    v = (e && (e[0] == '0' || e[0] == '1')) ? (e[0] - '0') : (KP >= 32 ? 1 : 0);
-  }
-  return v == 1;
+  const int o = opt(KS_OPT_FP32_SPLIT, -1);
+  return (o == 0 || o == 1) ? o == 1 : KP >= 32;
 }
 
 template <int KP, bool SPLIT>

@@ -126,6 +126,17 @@ __device__ __forceinline__ bool f16_fold_ok(const unsigned* amax, double c, int 
   const double a = (double)__uint_as_float(*amax);
   return c * (double)K * a * a <= 4096.0;
 }
+// Fold shift (reading Q28; the R = 1 kernel of ks_fused_r1.cu, fold modes 2 and 3): beyond
+// c K amax^2 = 2^12 the norm pieces are stored as n 2^-s and the opposite operand's unit
+// columns hold 2^s (exact), s = ceil(log2(c K amax^2 / 2^12)) <= 15, so the folded layout is
+// valid for every input and needs no device-side fallback.
+__device__ __forceinline__ int f16_fold_shift(const unsigned* amax, double c, int K) {
+  const double a = (double)__uint_as_float(*amax);
+  const double v = c * (double)K * a * a / 4096.0;
+  if (!(v > 1.0)) return 0;  // (NaN: 0)
+  const int s = (int)ceil(log2(v));
+  return s > 15 ? 15 : s;
+}
 // balanced scaling: |2c x 2^eF| ~ |x 2^-eF| for coordinates of equal spread
 __device__ __forceinline__ int f16_fold_exp(double c) {
   const int e = (int)rint(-0.5 * log2(2.0 * c));
@@ -1306,10 +1317,9 @@ __device__ __forceinline__ float group_max(float v) {
   for (int o = G / 2; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
   return v;
 }
-// KS_PREP_G = 4, 8, 16 or 32 overrides (measurement knob)
+// KS_OPT_PREP_LANES = 4, 8, 16 or 32 overrides (tuning option)
 int prep_group(int K) {
-  const char* e = getenv("KS_PREP_G");
-  const int g = e ? atoi(e) : 0;
+  const int g = opt(KS_OPT_PREP_LANES, 0);
   if (g == 4 || g == 8 || g == 16 || g == 32) return g;
   return K <= 8 ? 4 : 8;
 }
@@ -1337,17 +1347,22 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
   n = group_sum<G>(n);
   const float nai = live ? (float)(-c * n) : 0.f;
   const double c2 = 2.0 * c;
-  const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u;
+  // aug (FP16): 1 folded layout when f16_fold_ok, 2 always folded (fold shift), 3 the same
+  // without log-weights (the R = 1 kernel's weight mode)
+  const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && !(F16 && aug == 3);
   // log2(W_i / Wmax) (R = 1, W >= 0; -inf for W_i = 0 and padding)
   const double wl = !logw ? 0.0 : live ? log2((double)W[i]) - log2((double)__uint_as_float(wstat[0])) : -INFINITY;
   float sA = 1.f;
   bool fa = false;  // folded layout active
   __half np[3] = {__float2half(0.f), __float2half(0.f), __float2half(0.f)};
+  __half one = __float2half(1.f);  // unit columns (times the target's norm pieces): 2^s
   if constexpr (F16) {
-    fa = aug && f16_fold_ok(amax, c, K);
+    fa = aug >= 2 || (aug == 1 && f16_fold_ok(amax, c, K));
     if (fa) {
+      const int fsh = aug >= 2 ? f16_fold_shift(amax, c, K) : 0;
+      one = __float2half(ldexpf(1.f, fsh));
       sA = ldexpf(1.f, f16_fold_exp(c));
-      const double nf = -c * n + wl;  // finite unless W_i = 0: then the FP16 stand-in for -inf
+      const double nf = ldexp(-c * n + wl, -fsh);  // finite unless W_i = 0: then the FP16 stand-in for -inf
       if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
       else split3_f16(nf, np);
     } else {
@@ -1370,11 +1385,11 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
       split_f16(a0 * sA, h0, l0);  // exact power-of-2 scaling
       split_f16(a1 * sA, h1, l1);
       if (fa && d >= K && d < K + 6) {  // folded norm columns: hi planes only
-        h0 = d < K + 3 ? np[d - K] : __float2half(1.f);
+        h0 = d < K + 3 ? np[d - K] : one;
         l0 = __float2half(0.f);
       }
       if (fa && d + 1 >= K && d + 1 < K + 6) {
-        h1 = d + 1 < K + 3 ? np[d + 1 - K] : __float2half(1.f);
+        h1 = d + 1 < K + 3 ? np[d + 1 - K] : one;
         l1 = __float2half(0.f);
       }
       static_cast<__half2*>(src_hi)[(i * k_pad + d) >> 1] = __halves2half2(h0, h1);
@@ -1434,13 +1449,16 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
   float sB = 1.f, rj = 1.f;
   bool fa = false, far = false;  // folded layout active; row beyond every source (kernel row 0)
   __half mp[3] = {__float2half(0.f), __float2half(0.f), __float2half(0.f)};
+  __half one = __float2half(1.f);  // unit columns (times the source's norm pieces): 2^s
   if constexpr (F16) {
-    fa = aug && f16_fold_ok(amax, c, K);
+    fa = aug >= 2 || (aug == 1 && f16_fold_ok(amax, c, K));
     if (fa) {
+      const int fsh = aug >= 2 ? f16_fold_shift(amax, c, K) : 0;
+      one = __float2half(ldexpf(1.f, fsh));
       sB = ldexpf(1.f, -f16_fold_exp(c));
-      far = c * n > kFoldFar;
+      far = c * n > ldexp(kFoldFar, fsh);
       if (far) mp[0] = __float2half(kFoldNegInf);
-      else split3_f16(-c * n, mp);
+      else split3_f16(ldexp(-c * n, -fsh), mp);
     } else {
       bmax = group_max<G>(bmax);
       const int eA = f16_scale_exp((float)(2.0 * c * (double)__uint_as_float(*amax)));
@@ -1462,11 +1480,11 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
       split_f16(x0 * sB, h0, l0);
       split_f16(x1 * sB, h1, l1);
       if (fa && d >= K && d < K + 6) {  // folded norm columns: hi planes only
-        h0 = d < K + 3 ? __float2half(1.f) : mp[d - K - 3];
+        h0 = d < K + 3 ? one : mp[d - K - 3];
         l0 = __float2half(0.f);
       }
       if (fa && d + 1 >= K && d + 1 < K + 6) {
-        h1 = d + 1 < K + 3 ? __float2half(1.f) : mp[d + 1 - K - 3];
+        h1 = d + 1 < K + 3 ? one : mp[d + 1 - K - 3];
         l1 = __float2half(0.f);
       }
       static_cast<__half2*>(tgt_hi)[(j * k_pad + d) >> 1] = __halves2half2(h0, h1);
@@ -1478,7 +1496,8 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
     }
   }
   if (gl == 0) {
-    nb[j] = aug ? 0.f : nbj;  // aug (TF32) / folded (FP16): the norm rides in the contraction
+    // aug (TF32) / folded (FP16, when active on the device): the norm rides in the contraction
+    nb[j] = (fa || (!F16 && aug)) ? 0.f : nbj;
     tsc[j] = rj;
   }
 }
@@ -1614,10 +1633,10 @@ cudaError_t launch_prep_f16_targets(const float* beta, int64_t N, int64_t n_pad,
   return launch_prep_targets<true>(beta, N, n_pad, K, k_pad, mu, c, fold, amax, tgt_hi, tgt_lo, nb, tsc, st);
 }
 
-// Pipeline depth: KS_TC_STAGES (3..6) overrides the default (measurement knob).
+// Pipeline depth: KS_OPT_STAGES (3..5) overrides the default (tuning option).
 static int tc_stages(int r_c) {
-  const char* e = getenv("KS_TC_STAGES");
-  int v = (e && e[0] >= '3' && e[0] <= '5') ? (e[0] - '0') : 5;
+  const int o = opt(KS_OPT_STAGES, 0);
+  int v = (o >= 3 && o <= 5) ? o : 5;
   if (r_c > 16 && v > 4) v = 4;  // shared-memory budget (227 KB per CTA)
   return v;
 }
@@ -1666,13 +1685,12 @@ cudaError_t launch_fused_tc(const CUtensorMap* maps, const TcArgs& a, cudaStream
   // CUDA-core weighted sum (256-source tiles): 48 KB stages, 4 fit (3 with the 16 KB weight slots)
   switch (a.vcc) {
     case 1: {
-      // R = 1: exponential pairs of 16 on the FMA pipe (KS_TC_POLY = 0, 4, 6 or 8)
-      // and the exact d^2 >= 0 clamp of the log-weight epilogue (KS_TC_CLAMP=1; costs 15% at cfg3)
+      // R = 1: exponential pairs of 16 on the FMA pipe (KS_OPT_EXP_POLY = 0, 4, 6 or 8)
+      // and the exact d^2 >= 0 clamp of the log-weight epilogue (KS_OPT_CLAMP=1; costs 15% at cfg3)
       // one operand chunk (K <= 26 folded): the contraction is shorter, 7 of 16 on the FMA pipe
-      const char* e = getenv("KS_TC_POLY");
-      const int pp = e ? atoi(e) : (a.ares && a.f16 && a.k_pad <= kTcKC ? 7 : kTcPolyDefault);
-      const char* ec = getenv("KS_TC_CLAMP");
-      const bool clamp = ec && ec[0] == '1';
+      const int po = opt(KS_OPT_EXP_POLY, -1);
+      const int pp = po >= 0 ? po : (a.ares && a.f16 && a.k_pad <= kTcKC ? 7 : kTcPolyDefault);
+      const bool clamp = opt(KS_OPT_CLAMP, 0) == 1;
       if (clamp) return pp == 0 ? launch_rcsv<16, 4, 1, 16>(maps, a, st) : launch_rcsv<16, 4, 1, 20>(maps, a, st);
       if (a.ares && a.f16 && a.k_pad <= 2 * kTcKC) {  // split-FP16, target operand resident (<= 2 chunks)
         switch (pp) {

@@ -7,6 +7,8 @@
 #include <atomic>
 #include <cstdint>
 
+#include "ks.h"
+
 namespace ks {
 
 // Programmatic dependent launch (PDL): kernels of the TC path after the source statistics are
@@ -46,6 +48,14 @@ inline cudaError_t smem_optin_once(std::atomic<uint64_t>& done, const void* fn, 
   if (e == cudaSuccess && bit) done.fetch_or(bit, std::memory_order_acq_rel);
   return e;
 }
+
+// Tuning options of the context making the current API call (ks_set_option, include/ks.h),
+// visible to the kernel launchers for the duration of that call.
+struct Opts {
+  int v[16];
+};
+extern thread_local const Opts* tl_opts;
+inline int opt(int id, int dflt) { return tl_opts ? tl_opts->v[id] : dflt; }
 
 constexpr int kTileT = 256;   // targets per CTA tile (FP32 path)
 constexpr int kTileS = 128;   // sources per pipeline stage (FP32 path)
@@ -142,6 +152,30 @@ struct TcArgs {
   StreamK sk;
   unsigned long long* cta_times;
 };
+
+// ---------------------------------------------------------------- R = 1 folded kernel (ks_fused_r1.cu)
+// Split-FP16 operands with the norms folded into the contraction (K + 6 <= 64), one weight
+// column.  Sources in 128-row tiles (box rows 128 for both operand maps).
+struct R1Args {
+  int64_t N;              // targets
+  int n_kc;               // 64-byte operand chunks (32 halves each): 1 or 2
+  int kdims;              // coordinate columns (= K): K steps below need all three split products
+  int kcols;              // K + 6: steps at or past it are zero padding
+  int logw;               // host allows the log-weight mode (decided on the device from wstat)
+  int clamp;              // weight mode: 1 clamp t <= 0 (d^2 >= 0) before the exponential, 2 t -> -|t|
+  const unsigned* wstat;  // {bits of max |W|, any W < 0 or NaN}
+  const float* wv;        // [m_pad] raw weights, zero padded (weight mode)
+  float* V;               // [N]
+  float* partial;         // [grid][2][128]
+  int* counters;          // [n_t], zero on entry, left zero
+  StreamK sk;             // n_s = m_pad / 128
+  unsigned long long* cta_times;  // debug: [grid][4] globaltimer, clock64 at CTA start; the same at the end
+                                  // (KS_PROF builds: then [grid][20 warps][4] per-warp phase clocks)
+  int dbg;                // KS_DEBUG builds only (KS_R1_DEBUG): 1 no epilogue math, 2 no MMAs, 3 neither, 4 + no source loads
+};
+cudaError_t launch_fused_r1(const CUtensorMap* maps, const R1Args& a, int npoly, cudaStream_t st);
+int fused_r1_stages(int K);
+int r1_poly();
 
 // sources: src_hi/lo [m_pad][k_pad] = TF32 split of RN(2c (alpha - mu)),
 // na [m_pad], W^T split wt_hi/lo [r_pad][m_pad] (zero padded)

@@ -20,21 +20,27 @@ import paper_conf_icppw_wangkbgj16_b200 as ks  # noqa: E402
 _PREC = {"p": "auto"}
 
 
-@pytest.fixture(autouse=True, params=["3xf16", "3xtf32"])
+@pytest.fixture(autouse=True, params=["3xf16", "3xf16-general", "3xtf32"])
 def _split_precision(request):
     """Every test below runs on both split-operand MMA kinds (kind::f16 with
     power-of-2 scaled FP16 hi/lo operands -- the KS_PREC_AUTO choice -- and
-    kind::tf32 with TF32 hi/lo), unless it names a precision itself."""
+    kind::tf32 with TF32 hi/lo), unless it names a precision itself.  At R = 1 and
+    K <= 58 split-FP16 runs the dedicated R = 1 kernel (ks_fused_r1.cu);
+    "3xf16-general" sets KS_OPT_R1_KERNEL = 0 so the general kernel's R = 1 epilogues
+    (and the knobs the tests below set for them) stay covered."""
     _PREC["p"] = request.param
     yield
 
 
 def gpu_eval(alpha, W, beta, h, precision=None):
     precision = precision or _PREC["p"]
+    opts = {}
+    if precision == "3xf16-general":
+        precision, opts = "3xf16", {"r1_kernel": 0}
     W = np.asarray(W, np.float32)
     if W.ndim == 1:
         W = W[:, None]
-    with ks.KernelSum(alpha.shape[1], float(h), precision) as plan:
+    with ks.KernelSum(alpha.shape[1], float(h), precision, options=opts) as plan:
         plan.set_sources(torch.from_numpy(np.ascontiguousarray(alpha)).cuda(),
                          torch.from_numpy(np.ascontiguousarray(W)).cuda())
         V = plan.eval(torch.from_numpy(np.ascontiguousarray(beta)).cuda())
@@ -254,9 +260,10 @@ def test_r1_fold_policy_and_forced(oracle_mod, monkeypatch, K):
 
 
 def test_r1_fold_inactive_for_wide_spread(oracle_mod):
-    """c K amax^2 > 2^12 (h = 0.01 on the unit cube, K = 4): the folded layout
-    is switched off on the device (the FP16 norm pieces would not hold the
-    norms) and the epilogue adds them in FP32; same bar."""
+    """c K amax^2 > 2^12 (h = 0.01 on the unit cube, K = 4): the general kernel switches
+    the folded layout off on the device (the FP16 norm pieces would not hold the norms)
+    and adds the norms in FP32; the R = 1 kernel keeps it with the fold shift (reading
+    Q28: pieces of n 2^-s against unit columns 2^s).  Same bar."""
     a, W, b, h = workloads.custom(2000, 600, 4, 1, 0.01, wkind="pos", seed=5, same_points=True)
     check(oracle_mod, a, W, b, h)
 
