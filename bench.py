@@ -65,7 +65,8 @@ def parse():
     p.add_argument("--energy-seconds", type=float, default=1.0,
                    help="length of the NVML energy loop after the timed region (0: skip)")
     p.add_argument("--no-cpu-baseline", action="store_true")
-    p.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
+    p.add_argument("--cpu-seconds", type=float, default=16.0,
+                   help="target CPU time of the oracle sample (cfg3 on 16 cores: every target)")
     p.add_argument("--no-flush", action="store_true")
     p.add_argument("--precision", default="auto", choices=["auto", "fp32", "3xtf32", "3xf16", "tf32"],
                    help="ks_set_precision (auto: FP32 path for K<=32 and R=1, else 3xTF32 tensor cores)")
@@ -277,7 +278,7 @@ def run_ours(args):
     M, N, K, R = c.M, c.N, c.K, c.R
     lo, hi = shard_bounds(N, world, rank)
 
-    plan = ks.KernelSum(K, float(h), args.precision)
+    plan = ks.KernelSum(K, float(h), args.precision, options={"measure_clock": 1})
     ta = torch.from_numpy(a).to(dev) if rank == 0 or world == 1 else torch.empty((M, K), device=dev)
     tw = torch.from_numpy(W).to(dev) if rank == 0 or world == 1 else torch.empty((M, R), device=dev)
     tb = torch.from_numpy(b[lo:hi].copy()).to(dev)
@@ -327,6 +328,10 @@ def run_ours(args):
     ks.ks_timing_enable(plan.ctx, False)
     kern_ms, kern_n = ks.ks_timing_read(plan.ctx, reset=True)
     info1 = plan.info()
+    try:  # effective SM clock of the last timed fused launch (clock64 / globaltimer per CTA)
+        kern_ghz = ks.ks_clock_read(plan.ctx)[0]
+    except ks.KsError:
+        kern_ghz = None
     ms_steps = [s.elapsed_time(e) for s, e in zip(ev0, ev1)]
     ms_local = sum(ms_steps) / n_ev
     t = torch.tensor([ms_local], dtype=torch.float64, device=dev)
@@ -354,7 +359,7 @@ def run_ours(args):
         nprod = 3 if info1["precision"] in (ks.KS_PREC_3XTF32, ks.KS_PREC_3XF16) else 1
         # R <= 16 (256-source tiles): the weighted sum runs on CUDA cores and the
         # tensor work is the 2K contraction; R > 16: a second MMA adds 2R per pair
-        vcc = info1["tile_s"] == 256
+        vcc = info1["tile_s"] == 256 or info1["kernel"] == 3
         # burst peak for a kernel timed alone; the sustained (power-capped) one inside a long step
         long_step = ms_per_step >= 20.0
         pk = load_peaks()
@@ -379,18 +384,34 @@ def run_ours(args):
         achieved = pairs_launch * flops_pair / (kms / 1e3) / 1e12
         tensor = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": unit, "frac": achieved / peak,
                   "peak_derivation": deriv}
-        # the exponential: one 2^t per pair on MUFU.EX2 (16 / clk / SM), except the R = 1
-        # epilogue's 6 of 16 (folded layout; 4 of 16 unfolded) that run as a polynomial on the FMA pipe
-        sfu_peak = 16 * sms * max_mhz * 1e6
+        # the exponential: one 2^t per pair, NPOLY of every 16 pairs as a degree-5 polynomial on
+        # the FMA pipe (R = 1), the rest on MUFU.EX2.  Ceiling per SM per clock (SS6):
+        # MUFU 16 / (1 - p); FMA pipe 128 / (8.5 p + 1) lane-ops (8 per polynomial exponential,
+        # 0.5 IMAD, 1 accumulate per exponential); issue 128 / (1.5 + 5 p) (4 SMSPs x 32 lanes);
+        # p = NPOLY / 16.  At the design's best split (p = 0.424) the ceiling is 27.8 /clk/SM.
+        p = (info1["exp_poly"] / 16.0) if R == 1 else 0.0
+        lim = {"mufu": 16.0 / (1.0 - p), "fma": 128.0 / (8.5 * p + 1.0), "issue": 128.0 / (1.5 + 5.0 * p)}
+        per_clk = min(lim.values())
+        best = max(min(16.0 / (1.0 - q), 128.0 / (8.5 * q + 1.0), 128.0 / (1.5 + 5.0 * q))
+                   for q in np.linspace(0.0, 0.75, 301))
         ex2_rate = pairs_launch / (kms / 1e3)
-        sfu = {"bound": "alu", "achieved": ex2_rate / 1e9, "peak": sfu_peak / 1e9, "frac": ex2_rate / sfu_peak,
-               "unit": "G exponentials/s (MUFU.EX2 peak; R = 1 computes 6/16 of them on the FMA pipe)",
-               "peak_derivation": f"16 ex2/clk/SM x {sms} SMs x {max_mhz} MHz (sm_max)"}
+        exp_peak = per_clk * sms * max_mhz * 1e6
+        sfu = {"bound": "alu", "achieved": ex2_rate / 1e9, "peak": exp_peak / 1e9, "frac": ex2_rate / exp_peak,
+               "unit": "G exponentials/s (one 2^t per pair; %d of 16 pairs on the FMA pipe)" % info1["exp_poly"],
+               "peak_derivation": "min(MUFU 16/(1-p), FMA 128/(8.5p+1), issue 128/(1.5+5p)) = %.1f exp/clk/SM "
+                                  "(p = %d/16; %s-bound) x %d SMs x %d MHz (sm_max)"
+                                  % (per_clk, info1["exp_poly"], min(lim, key=lim.get), sms, max_mhz),
+               "mufu_only_frac": ex2_rate * (1.0 - p) / (16 * sms * max_mhz * 1e6),
+               "design_best_split_frac": ex2_rate / (best * sms * max_mhz * 1e6)}
+        if kern_ghz:
+            sfu["frac_at_kernel_clock"] = ex2_rate / (per_clk * sms * kern_ghz * 1e9)
+            tensor["frac_at_kernel_clock"] = achieved / (peak * kern_ghz * 1e3 / max_mhz)
         # the binding resource is the primary roofline, the other the co-bound
         prim, co = (sfu, tensor) if sfu["frac"] >= tensor["frac"] else (tensor, sfu)
         roof = dict(prim)
-        roof.update({"kernel": "ks_fused_tc_kernel", "traffic": load_traffic(args.cfg, args.precision),
-                     "co_bound": co})
+        roof.update({"kernel": "ks_fused_r1_kernel" if info1["kernel"] == 3 else "ks_fused_tc_kernel",
+                     "traffic": load_traffic(args.cfg, args.precision), "co_bound": co,
+                     "kernel_sm_ghz": kern_ghz})
         if vcc:
             # CUDA-core epilogue, R FFMA (weighted sum) + 1 FADD (exponent) per pair
             ops = pairs_launch * (R + 1) / (kms / 1e3) / 1e12
@@ -419,21 +440,50 @@ def run_ours(args):
         if energy and "j_per_step" in energy:
             energy["pairs_per_joule"] = pairs_per_step / energy["j_per_step"]
 
-    # ---- e2e through the C-ABI host entry points (pinned buffers, copies timed)
-    ha = torch.from_numpy(a).pin_memory()
-    hw = torch.from_numpy(W).pin_memory()
+    # ---- e2e: inputs from pinned host memory, copies inside the timed region.  N = 1: the C-ABI
+    # host entry points (ks_set_sources_host + ks_eval_host).  N > 1: rank 0 uploads alpha and W and
+    # broadcasts them over NCCL, every rank uploads its target shard, evaluates, the shards'
+    # V are all-gathered and rank 0 downloads V.
+    ha = torch.from_numpy(a).pin_memory() if rank == 0 or world == 1 else None
+    hw = torch.from_numpy(W).pin_memory() if rank == 0 or world == 1 else None
     hb = torch.from_numpy(b[lo:hi].copy()).pin_memory()
     hv = torch.empty((max(hi - lo, 1), R), dtype=torch.float32).pin_memory()
-    an, wn, bn, vn = ha.numpy(), hw.numpy(), hb.numpy(), hv.numpy()
+    hall = torch.empty((S * world, R), dtype=torch.float32).pin_memory() if (world > 1 and rank == 0) else None
     e2e_plan = ks.KernelSum(K, float(h), args.precision)
 
-    def e2e_step():
-        if world > 1:
-            dist.broadcast(ta, src=0)
-            dist.broadcast(tw, src=0)
-        e2e_plan.set_sources_host(an, wn)
-        if hi > lo:
+    if world == 1:
+        an, wn, bn, vn = ha.numpy(), hw.numpy(), hb.numpy(), hv.numpy()
+
+        def e2e_step():
+            e2e_plan.set_sources_host(an, wn)
             e2e_plan.eval_host(bn, out=vn[: hi - lo])
+        api = "ks_set_sources_host + ks_eval_host (pinned host buffers)"
+        h2d = 4 * (M * K + M * R + (hi - lo) * K)
+        d2h = 4 * (hi - lo) * R
+    else:
+        ea = torch.empty((M, K), device=dev)
+        ew = torch.empty((M, R), device=dev)
+        eb = torch.empty((max(hi - lo, 1), K), device=dev)
+        ev = torch.empty((max(hi - lo, 1), R), device=dev)
+
+        def e2e_step():
+            if rank == 0:
+                ea.copy_(ha, non_blocking=True)
+                ew.copy_(hw, non_blocking=True)
+            dist.broadcast(ea, src=0)
+            dist.broadcast(ew, src=0)
+            e2e_plan.set_sources(ea, ew)
+            if hi > lo:
+                eb[: hi - lo].copy_(hb, non_blocking=True)
+                e2e_plan.eval(eb[: hi - lo], out=ev[: hi - lo])
+                Vpad[: hi - lo].copy_(ev[: hi - lo])
+            dist.all_gather_into_tensor(Vall, Vpad)
+            if rank == 0:
+                hall.copy_(Vall, non_blocking=True)
+        api = "rank 0: pinned H2D of alpha, W + NCCL broadcast; per rank: pinned H2D of its beta shard, " \
+              "ks_set_sources + ks_eval; NCCL all-gather of V; rank 0: D2H of V"
+        h2d = 4 * (M * K + M * R + N * K)
+        d2h = 4 * N * R
 
     for _ in range(max(1, args.warmup)):
         e2e_step()
@@ -445,20 +495,18 @@ def run_ours(args):
         if flush is not None:
             l2_flush(flush)
         torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
         t0 = time.perf_counter()
         e2e_step()
         torch.cuda.synchronize()
         e_ms.append(1e3 * (time.perf_counter() - t0))
-    if os.environ.get("KS_BENCH_E2E_DEBUG"):
-        print("e2e per-step ms:", " ".join("%.3f" % x for x in e_ms), file=sys.stderr)
     t = torch.tensor([sum(e_ms) / len(e_ms)], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     e2e_ms = float(t.item())
     e2e = {"value": pairs_per_step / (e2e_ms / 1e3), "unit": UNIT,
-           "h2d_bytes_per_step": int(4 * (M * K + M * R + (hi - lo) * K)),
-           "d2h_bytes_per_step": int(4 * (hi - lo) * R), "ms_per_step": e2e_ms,
-           "api": "ks_set_sources_host + ks_eval_host (pinned host buffers)"}
+           "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "ms_per_step": e2e_ms, "api": api}
     e2e_plan.close()
 
     out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -475,7 +523,15 @@ def run_ours(args):
                       "path": {1: "fp32", 2: "tcgen05"}.get(info1["path"], info1["path"]),
                       "precision": {1: "fp32", 2: "3xtf32", 3: "tf32", 4: "3xf16"}.get(info1["precision"]),
                       "k_pad": info1["k_pad"], "ctas": info1["num_ctas"],
-                      "stages": info1["stages"]},
+                      "stages": info1["stages"],
+                      "kernel": {1: "ks_fused_fp32_kernel", 2: "ks_fused_tc_kernel",
+                                 3: "ks_fused_r1_kernel"}.get(info1["kernel"], "?"),
+                      # north_star's d^2 >= 0 clamp: the FP32 kernel and the R > 1 / weight-mode
+                      # epilogues clamp; the default R = 1 log-weight epilogue does not (DESIGN.md
+                      # Q8: overshoot bounded by the Eq.3 rounding, tests/test_gpu_r1.py)
+                      "clamp": ("off (log-weight epilogue, DESIGN.md Q8)" if info1["kernel"] == 3 and
+                                info1["r1_epilogue"] == 0 else
+                                {1: "on", 2: "on (|d^2|)", 3: "off"}.get(info1["r1_epilogue"], "on"))},
            "roofline": roof, "e2e": e2e, "clocks": clk_sum, "gpu_launches": launches,
            "gpu": torch.cuda.get_device_name(dev)}
     if energy is not None:
@@ -487,7 +543,8 @@ def run_ours(args):
         out["cpu_baseline"] = cb
         Vg = Vloc.cpu().numpy().astype(np.float64)[J]
         out["parity_sampled"] = {"e_norm": float(np.max(np.abs(Vg - Vr)) / np.abs(W).sum()),
-                                 "targets": int(len(J)), "bar": 1e-5}
+                                 "targets": int(len(J)), "of": int(N), "bar": 1e-5,
+                                 "sampling": "distinct targets (without replacement)"}
     if rank == 0:
         print(json.dumps(out), flush=True)
     plan.close()

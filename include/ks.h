@@ -83,6 +83,11 @@ typedef struct {
   int64_t launches;     /* cumulative kernels launched by this context       */
   int64_t fused_launches; /* cumulative launches of the fused kernel         */
   double c_log2;        /* c = log2(e) / (2 h^2), the ex2 prescale           */
+  int kernel;           /* 0 none, 1 FP32 kernel, 2 general tcgen05 kernel,
+                           3 R = 1 tcgen05 kernel (ks_fused_r1.cu)            */
+  int exp_poly;         /* exponential pairs of every 16 on the FMA pipe      */
+  int r1_epilogue;      /* R = 1 kernel: KS_OPT_R1_EPILOGUE in effect (0 log-
+                           weights, no d^2 clamp; 1 clamp; 2 |d^2|; 3 none)  */
 } ks_info;
 
 /* Create a context for dimension K (1 <= K <= 4096) and bandwidth h (finite,
@@ -168,7 +173,9 @@ typedef enum {
                                  16, 32 [sources, eval] */
   KS_OPT_EVAL_CHUNKS = 14,    /* KS_EVAL_CHUNKS: ks_eval_host target chunks: 0 auto, 1..4 [eval] */
   KS_OPT_FP32_SPLIT = 15,     /* KS_FP32_SPLIT: FP32 kernel tile body: -1 auto, 0, 1 [eval] */
-  KS_OPT_COUNT_ = 16
+  KS_OPT_MEASURE_CLOCK = 16,  /* 1: the R = 1 kernel records globaltimer and clock64 at every CTA's
+                                 start and end, for ks_clock_read (measurement, 0 default) [eval] */
+  KS_OPT_COUNT_ = 17
 } ks_option;
 
 /* Set / read a tuning option.  KS_EINVAL for an unknown option or a value out of its range. */
@@ -188,6 +195,11 @@ KS_API ks_status ks_get_info(const ks_ctx *ctx, ks_info *out);
  * (ms) and number of timed launches since the last reset. */
 KS_API ks_status ks_timing_enable(ks_ctx *ctx, int on);
 KS_API ks_status ks_timing_read(ks_ctx *ctx, double *total_ms, int64_t *launches, int reset);
+
+/* Effective SM clock of the last fused launch (KS_OPT_MEASURE_CLOCK = 1, R = 1 kernel): the mean
+ * over its CTAs of elapsed SM cycles (clock64) / elapsed time (globaltimer), in GHz, and the CTA
+ * count.  Synchronises the context's stream.  KS_ESTATE when no such launch was measured. */
+KS_API ks_status ks_clock_read(ks_ctx *ctx, double *sm_ghz, int *ctas);
 
 /* Human-readable status name; never NULL. */
 KS_API const char *ks_status_str(ks_status s);

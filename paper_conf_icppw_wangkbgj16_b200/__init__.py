@@ -32,12 +32,13 @@ PRECISIONS = {"auto": KS_PREC_AUTO, "fp32": KS_PREC_FP32, "3xtf32": KS_PREC_3XTF
 # every symbol include/ks.h declares (checked by tests/test_abi.py)
 EXPORTED = ("ks_create", "ks_destroy", "ks_set_precision", "ks_set_stream", "ks_set_sources", "ks_eval",
             "ks_set_sources_host", "ks_eval_host", "ks_reserve", "ks_get_info", "ks_timing_enable",
-            "ks_timing_read", "ks_set_option", "ks_get_option", "ks_status_str", "ks_last_error", "ks_version")
+            "ks_timing_read", "ks_set_option", "ks_get_option", "ks_clock_read", "ks_status_str", "ks_last_error",
+            "ks_version")
 
 # tuning options (include/ks.h ks_option): variants computing the same result, none drops work
 OPTIONS = {"r1_kernel": 1, "r1_epilogue": 2, "exp_poly": 3, "weighted_sum": 4, "log_weights": 5, "fold": 6,
            "aug": 7, "clamp": 8, "target_resident": 9, "stages": 10, "ar_stages": 11, "wslots": 12,
-           "prep_lanes": 13, "eval_chunks": 14, "fp32_split": 15}
+           "prep_lanes": 13, "eval_chunks": 14, "fp32_split": 15, "measure_clock": 16}
 
 
 class KsInfo(ctypes.Structure):
@@ -45,7 +46,8 @@ class KsInfo(ctypes.Structure):
                 ("tile_t", ctypes.c_int), ("tile_s", ctypes.c_int), ("num_ctas", ctypes.c_int),
                 ("stages", ctypes.c_int), ("num_sms", ctypes.c_int), ("m", ctypes.c_int64),
                 ("m_pad", ctypes.c_int64), ("r", ctypes.c_int), ("launches", ctypes.c_int64),
-                ("fused_launches", ctypes.c_int64), ("c_log2", ctypes.c_double)]
+                ("fused_launches", ctypes.c_int64), ("c_log2", ctypes.c_double), ("kernel", ctypes.c_int),
+                ("exp_poly", ctypes.c_int), ("r1_epilogue", ctypes.c_int)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -79,6 +81,7 @@ def _load():
         "ks_timing_read": ([P, ctypes.POINTER(D), ctypes.POINTER(L), I], I),
         "ks_set_option": ([P, I, I], I),
         "ks_get_option": ([P, I, ctypes.POINTER(I)], I),
+        "ks_clock_read": ([P, ctypes.POINTER(D), ctypes.POINTER(I)], I),
         "ks_status_str": ([I], ctypes.c_char_p),
         "ks_last_error": ([], ctypes.c_char_p),
         "ks_version": ([], ctypes.c_char_p),
@@ -188,6 +191,14 @@ def ks_get_option(ctx, opt) -> int:
     v = ctypes.c_int()
     _check(_lib.ks_get_option(ctx, int(opt), ctypes.byref(v)), "ks_get_option")
     return v.value
+
+
+def ks_clock_read(ctx):
+    """(effective SM GHz, CTAs) of the last fused launch measured with option measure_clock=1."""
+    g = ctypes.c_double()
+    n = ctypes.c_int()
+    _check(_lib.ks_clock_read(ctx, ctypes.byref(g), ctypes.byref(n)), "ks_clock_read")
+    return g.value, n.value
 
 
 def ks_timing_enable(ctx, on: bool) -> None:

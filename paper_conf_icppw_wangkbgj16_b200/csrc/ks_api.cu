@@ -152,6 +152,10 @@ struct ks_ctx {
   DBuf<unsigned> wcol, wcol_part; // FP16 V-MMA: per-column max |W| bits [r_pad], block partials
   CUtensorMap tmap_src;
 
+  // KS_OPT_MEASURE_CLOCK: per-CTA {globaltimer, clock64} x {start, end} of the last R = 1 launch
+  DBuf<unsigned long long> clk_buf;
+  int clk_ctas = 0;
+
   // eval scratch
   DBuf<float> partial;
   DBuf<int> counters;
@@ -208,6 +212,7 @@ const OptSpec kOpt[KS_OPT_COUNT_] = {
     {"KS_PREP_G", 0, 0, 32},
     {"KS_EVAL_CHUNKS", 0, 0, 4},
     {"KS_FP32_SPLIT", -1, -1, 1},
+    {"KS_MEASURE_CLOCK", 0, 0, 1},
 };
 
 void init_opts(ks_ctx* ctx) {
@@ -565,6 +570,10 @@ ks_status eval_r1(ks_ctx* ctx, const CUtensorMap* maps, int64_t N, float* V) {
   if (dbg) {
     KS_CUDA(ctx->dbg_times.reserve(n_dbg, st, true), "allocate debug timers");
     a.cta_times = ctx->dbg_times.p;
+  } else if (ctx->opts.v[KS_OPT_MEASURE_CLOCK]) {
+    KS_CUDA(ctx->clk_buf.reserve((size_t)ctx->num_sms * 4, st, false), "allocate clock buffer");
+    a.cta_times = ctx->clk_buf.p;
+    ctx->clk_ctas = sk.grid;
   }
   cudaEvent_t stop;
   ks_status s = timed_begin(ctx, &stop);
@@ -575,7 +584,7 @@ ks_status eval_r1(ks_ctx* ctx, const CUtensorMap* maps, int64_t N, float* V) {
   ctx->last_grid = sk.grid;
   s = timed_end(ctx, stop);
   if (s != KS_OK) return s;
-  if (a.cta_times) {  // "r1 <cta> <t0 ns> <t1 ns> <clock0> <clock1> [20 x 4 phase clocks]" per CTA
+  if (dbg) {  // "r1 <cta> <t0 ns> <t1 ns> <clock0> <clock1> [20 x 4 phase clocks]" per CTA
     std::vector<unsigned long long> h(n_dbg);
     KS_CUDA(cudaMemcpyAsync(h.data(), a.cta_times, h.size() * 8, cudaMemcpyDeviceToHost, st), "copy debug timers");
     KS_CUDA(cudaStreamSynchronize(st), "synchronize");
@@ -813,6 +822,7 @@ ks_status ks_destroy(ks_ctx* ctx) {
   ctx->partial.release();
   ctx->counters.release();
   ctx->dbg_times.release();
+  ctx->clk_buf.release();
   ctx->h_alpha.release();
   ctx->h_W.release();
   ctx->h_beta.release();
@@ -1066,6 +1076,34 @@ ks_status ks_get_info(const ks_ctx* ctx, ks_info* out) {
   out->launches = ctx->launches;
   out->fused_launches = ctx->fused_launches;
   out->c_log2 = ctx->c;
+  out->kernel = !ctx->have_src ? 0 : ctx->path == KS_PATH_FP32 ? 1 : ctx->r1 ? 3 : 2;
+  out->exp_poly = ctx->r1 ? ks::r1_poly_for(ctx->opts.v[KS_OPT_EXP_POLY]) : ctx->opts.v[KS_OPT_EXP_POLY];
+  out->r1_epilogue = ctx->r1 ? ctx->opts.v[KS_OPT_R1_EPILOGUE] : -1;
+  return KS_OK;
+}
+
+ks_status ks_clock_read(ks_ctx* ctx, double* sm_ghz, int* ctas) {
+  if (check_ctx(ctx)) return KS_EINVAL;
+  if (!sm_ghz || !ctas) return fail(KS_EINVAL, "sm_ghz/ctas is NULL");
+  if (ctx->clk_ctas <= 0 || !ctx->clk_buf.p) return fail(KS_ESTATE, "no measured launch (KS_OPT_MEASURE_CLOCK)");
+  ks_status s = set_device(ctx);
+  if (s != KS_OK) return s;
+  std::vector<unsigned long long> h((size_t)ctx->clk_ctas * 4);
+  KS_CUDA(cudaMemcpyAsync(h.data(), ctx->clk_buf.p, h.size() * 8, cudaMemcpyDeviceToHost, ctx->stream),
+          "copy clock records");
+  KS_CUDA(cudaStreamSynchronize(ctx->stream), "synchronize");
+  double acc = 0.0;
+  int n = 0;
+  for (int b = 0; b < ctx->clk_ctas; ++b) {
+    const double dt = (double)(h[4 * b + 2] - h[4 * b]), dc = (double)(h[4 * b + 3] - h[4 * b + 1]);
+    if (dt > 0.0) {
+      acc += dc / dt;
+      ++n;
+    }
+  }
+  if (n == 0) return fail(KS_ESTATE, "empty clock records");
+  *sm_ghz = acc / n;
+  *ctas = n;
   return KS_OK;
 }
 

@@ -562,10 +562,8 @@ __global__ void __launch_bounds__(kR1Threads, 1)
 }
 
 // exponential pairs of 16 on the FMA pipe (KS_OPT_EXP_POLY tuning option; default measured)
-int r1_poly() {
-  const int v = opt(KS_OPT_EXP_POLY, -1);
-  return (v == 0 || v == 4 || v == 5 || v == 6 || v == 7 || v == 8) ? v : 6;
-}
+int r1_poly_for(int v) { return (v == 0 || v == 4 || v == 5 || v == 6 || v == 7 || v == 8) ? v : 6; }
+int r1_poly() { return r1_poly_for(opt(KS_OPT_EXP_POLY, -1)); }
 
 template <int NPOLY, int CLAMP>
 static cudaError_t launch_r1_t(const CUtensorMap* m, const R1Args& a, cudaStream_t st) {

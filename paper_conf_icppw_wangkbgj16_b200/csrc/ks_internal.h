@@ -52,7 +52,7 @@ inline cudaError_t smem_optin_once(std::atomic<uint64_t>& done, const void* fn, 
 // Tuning options of the context making the current API call (ks_set_option, include/ks.h),
 // visible to the kernel launchers for the duration of that call.
 struct Opts {
-  int v[16];
+  int v[KS_OPT_COUNT_];
 };
 extern thread_local const Opts* tl_opts;
 inline int opt(int id, int dflt) { return tl_opts ? tl_opts->v[id] : dflt; }
@@ -176,6 +176,7 @@ struct R1Args {
 cudaError_t launch_fused_r1(const CUtensorMap* maps, const R1Args& a, int npoly, cudaStream_t st);
 int fused_r1_stages(int K);
 int r1_poly();
+int r1_poly_for(int opt_value);  // the NPOLY the R = 1 kernel runs for a KS_OPT_EXP_POLY value
 
 // sources: src_hi/lo [m_pad][k_pad] = TF32 split of RN(2c (alpha - mu)),
 // na [m_pad], W^T split wt_hi/lo [r_pad][m_pad] (zero padded)

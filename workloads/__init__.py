@@ -155,10 +155,11 @@ def separable_grid(K: int, G: int, seed: int):
 
 
 def sample_targets(N: int, n: int, seed: int, tile: int = 128, extra=()):
-    """Seeded target subset for sampled parity: n uniform indices plus the
-    first/last target of the range and of tile boundaries, plus `extra`."""
+    """Seeded target subset for sampled parity: n distinct uniform indices (drawn
+    without replacement, so n = N covers every target) plus the first/last target
+    of the range and of tile boundaries, plus `extra`."""
     g = rng(seed)
-    pick = set(int(x) for x in g.integers(0, N, size=min(n, N)))
+    pick = set(int(x) for x in g.choice(N, size=min(n, N), replace=False)) if N > 0 else set()
     for b in (0, N - 1, tile - 1, tile, N - tile, N - tile - 1):
         if 0 <= b < N:
             pick.add(b)
