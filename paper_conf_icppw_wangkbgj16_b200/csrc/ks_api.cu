@@ -376,18 +376,19 @@ ks_status eval_fp32(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
 // Row-major [rows][inner] operand, one box = box_rows x 64 bytes (16 FP32 or
 // 32 FP16 elements), SWIZZLE_64B: the K-major smem layout of the MMA operands.
 ks_status encode_2d_sw64(CUtensorMap* map, const void* base, int64_t inner, int64_t rows, int box_rows,
-                         bool f16 = false) {
+                         bool f16 = false, bool rows32 = false) {
   PFN_encodeTiled enc = get_encode();
   if (!enc) return fail(KS_ECUDA, "cuTensorMapEncodeTiled unavailable from the driver");
   const size_t es = f16 ? 2 : 4;
+  const size_t row_bytes = rows32 ? 32 : 64;  // rows32: 32-byte boxes with SWIZZLE_32B
   cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)rows};
   cuuint64_t strides[1] = {(cuuint64_t)inner * es};
-  cuuint32_t box[2] = {(cuuint32_t)(64 / es), (cuuint32_t)box_rows};
+  cuuint32_t box[2] = {(cuuint32_t)(row_bytes / es), (cuuint32_t)box_rows};
   cuuint32_t estr[2] = {1, 1};
   CUresult r = enc(map, f16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
-                   const_cast<void*>(base), dims, strides, box, estr,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                   const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   rows32 ? CU_TENSOR_MAP_SWIZZLE_32B : CU_TENSOR_MAP_SWIZZLE_64B,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return fail(KS_ECUDA, "cuTensorMapEncodeTiled (2D SW64) failed (CUresult %d)", (int)r);
   return KS_OK;
 }
@@ -470,8 +471,12 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
     r1_clamp = mode == 3 ? 0 : mode == 2 ? 2 : 1;
     fold = r1;
   }
-  // k_pad in elements: one 64-byte row chunk per pipeline stage = 16 FP32 or 32 FP16
-  const int k_pad = f16 ? (int)round_up(K + 6 * (fold ? 1 : 0), 2 * ks::kTcKC) : tc_k_pad(K);
+  // k_pad in elements: one 64-byte row chunk per pipeline stage = 16 FP32 or 32 FP16; the R = 1
+  // kernel at K + 6 <= 16 keeps 32-byte rows (16 halves: half the operand bytes; cfg5's prepared
+  // source set, 1,048,576 x 2 x 32 B, then stays in the 126 MB L2)
+  const bool narrow = r1 && K + 6 <= ks::kTcKC;
+  const int k_pad = narrow ? ks::kTcKC
+                    : f16 ? (int)round_up(K + 6 * (fold ? 1 : 0), 2 * ks::kTcKC) : tc_k_pad(K);
   const int aug = f16 ? 0 : tc_aug(K);  // FP16 mode: norms stay in FP32 in the epilogue (or fold)
   const int tile_s = ks::fused_tc_tile_s(vcc);
   const int box_s = r1 ? 128 : tile_s;  // sources per operand tile of the kernel
@@ -513,9 +518,9 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
             "source prep (TC)");
   }
   ctx->launches += 1;
-  ks_status s = encode_2d_sw64(&ctx->tmB_hi, ctx->src_hi.p, k_pad, m_pad, box_s, f16);
+  ks_status s = encode_2d_sw64(&ctx->tmB_hi, ctx->src_hi.p, k_pad, m_pad, box_s, f16, narrow);
   if (s != KS_OK) return s;
-  s = encode_2d_sw64(&ctx->tmB_lo, ctx->src_lo.p, k_pad, m_pad, box_s, f16);
+  s = encode_2d_sw64(&ctx->tmB_lo, ctx->src_lo.p, k_pad, m_pad, box_s, f16, narrow);
   if (s != KS_OK) return s;
   ctx->k_pad = k_pad;
   ctx->m_pad = m_pad;
@@ -546,7 +551,8 @@ ks_status eval_r1(ks_ctx* ctx, const CUtensorMap* maps, int64_t N, float* V) {
   KS_CUDA(ctx->counters.reserve((size_t)sk.n_t, st, true), "allocate tile counters");
   ks::R1Args a;
   a.N = N;
-  a.n_kc = ctx->k_pad / 32;
+  a.narrow = ctx->k_pad == ks::kTcKC ? 1 : 0;
+  a.n_kc = a.narrow ? 1 : ctx->k_pad / 32;
   a.kdims = ctx->tc_kdims;
   a.kcols = ctx->tc_kcols;
   a.logw = ctx->r1 == 2 ? 1 : 0;
@@ -627,9 +633,10 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   }
   ctx->launches += 1;
   CUtensorMap maps[6];
-  ks_status s = encode_2d_sw64(&maps[0], ctx->tgt_hi.p, k_pad, n_pad, ks::kTcTileT, f16);
+  const bool narrow = ctx->r1 && k_pad == ks::kTcKC;  // 32-byte operand rows (R = 1 kernel, K + 6 <= 16)
+  ks_status s = encode_2d_sw64(&maps[0], ctx->tgt_hi.p, k_pad, n_pad, ks::kTcTileT, f16, narrow);
   if (s != KS_OK) return s;
-  s = encode_2d_sw64(&maps[1], ctx->tgt_lo.p, k_pad, n_pad, ks::kTcTileT, f16);
+  s = encode_2d_sw64(&maps[1], ctx->tgt_lo.p, k_pad, n_pad, ks::kTcTileT, f16, narrow);
   if (s != KS_OK) return s;
   maps[2] = ctx->tmB_hi;
   maps[3] = ctx->tmB_lo;

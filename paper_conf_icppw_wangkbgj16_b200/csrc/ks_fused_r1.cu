@@ -69,7 +69,7 @@ constexpr int kR1Groups = 4;                 // epilogue groups = TMEM S buffers
 constexpr int kR1EpiWarps = 4 * kR1Groups;  // one warp per TMEM lane quarter per group
 constexpr int kR1Threads = 128 + 32 * kR1EpiWarps;
 constexpr int kR1TS = 128;                   // sources per unit
-constexpr uint32_t kR1Plane = 128u * 64u;    // 128 rows x one 64-byte chunk (8 KB)
+constexpr uint32_t kR1Plane = 128u * 64u;    // 128 rows x one 64-byte chunk (8 KB); 4 KB with 32-byte rows
 constexpr int kR1WSlots = 8;                 // weight ring (weight mode)
 constexpr int kR1MaxStages = 8;
 constexpr uint32_t kR1Smem = 227u * 1024u;   // dynamic shared memory requested
@@ -209,10 +209,12 @@ __global__ void __launch_bounds__(kR1Threads, 1)
   }
 
   // ---- geometry: planes per tile (chunk 0: hi, lo; chunk 1: hi, + lo when it holds coordinates)
-  const int n_kc = args.n_kc;  // 64-byte chunks of 32 halves: 1 or 2
+  const int n_kc = args.n_kc;  // operand chunks: 1 or 2 of 32 halves (64-byte rows), or 1 of 16 (narrow)
+  const bool narrow = args.narrow != 0;  // K + 6 <= 16: 32-byte rows, SWIZZLE_32B, one K step
   const bool lo1 = n_kc == 2 && args.kdims > 32;
   const int P = 2 + (n_kc == 2 ? (lo1 ? 2 : 1) : 0);
-  const uint32_t tile_bytes = (uint32_t)P * kR1Plane;
+  const uint32_t plane = narrow ? kR1Plane / 2 : kR1Plane;
+  const uint32_t tile_bytes = (uint32_t)P * plane;
   int D = (int)((kR1Region - 2 * tile_bytes) / tile_bytes);
   if (D > kR1MaxStages) D = kR1MaxStages;
   const uint32_t offA = 0, offS = 2 * tile_bytes;
@@ -287,10 +289,10 @@ __global__ void __launch_bounds__(kR1Threads, 1)
           const int y = (int)(cu.tt * 128);
           mbar_arrive_expect_tx(&afull[ab], tile_bytes);
           tma_load_2d(ap, &mA_hi, 0, y, &afull[ab]);
-          tma_load_2d(ap + kR1Plane, &mA_lo, 0, y, &afull[ab]);
+          tma_load_2d(ap + plane, &mA_lo, 0, y, &afull[ab]);
           if (n_kc == 2) {
-            tma_load_2d(ap + 2 * kR1Plane, &mA_hi, 32, y, &afull[ab]);
-            if (lo1) tma_load_2d(ap + 3 * kR1Plane, &mA_lo, 32, y, &afull[ab]);
+            tma_load_2d(ap + 2 * plane, &mA_hi, 32, y, &afull[ab]);
+            if (lo1) tma_load_2d(ap + 3 * plane, &mA_lo, 32, y, &afull[ab]);
           }
         }
         __syncwarp();
@@ -303,10 +305,10 @@ __global__ void __launch_bounds__(kR1Threads, 1)
         const int y = cu.st * kR1TS;
         mbar_arrive_expect_tx(&full[s], tile_bytes);
         tma_load_2d(sp, &mB_hi, 0, y, &full[s]);
-        tma_load_2d(sp + kR1Plane, &mB_lo, 0, y, &full[s]);
+        tma_load_2d(sp + plane, &mB_lo, 0, y, &full[s]);
         if (n_kc == 2) {
-          tma_load_2d(sp + 2 * kR1Plane, &mB_hi, 32, y, &full[s]);
-          if (lo1) tma_load_2d(sp + 3 * kR1Plane, &mB_lo, 32, y, &full[s]);
+          tma_load_2d(sp + 2 * plane, &mB_hi, 32, y, &full[s]);
+          if (lo1) tma_load_2d(sp + 3 * plane, &mB_lo, 32, y, &full[s]);
         }
       }
       __syncwarp();
@@ -326,15 +328,15 @@ __global__ void __launch_bounds__(kR1Threads, 1)
     const uint32_t idS = idesc_f16(128, kR1TS);
     // products per 16-column K step: 3 (coordinates: lo.hi, hi.lo, hi.hi), 1 (norm pieces only), 0
     uint32_t plan = 0;
-    for (int st4 = 0; st4 < 2 * n_kc; ++st4) {
+    for (int st4 = 0; st4 < (narrow ? 1 : 2 * n_kc); ++st4) {
       const int col0 = st4 * 16;
       const uint32_t np = col0 >= args.kcols ? 0u : (col0 >= args.kdims ? 1u : 3u);
       plan |= np << (2 * st4);
     }
     // descriptors: low words (start address >> 4) advance within the same high word
-    const uint32_t dhi = (uint32_t)(sdesc_k_sw64(smem) >> 32);
+    const uint32_t dhi = (uint32_t)((narrow ? sdesc_k_sw32(smem) : sdesc_k_sw64(smem)) >> 32);
     const uint32_t dA0 = (uint32_t)sdesc_k_sw64(smem + offA), dS0 = (uint32_t)sdesc_k_sw64(smem + offS);
-    constexpr uint32_t kP16 = kR1Plane >> 4;
+    const uint32_t kP16 = plane >> 4;
     const uint32_t tile16 = tile_bytes >> 4;
     int s = 0;
     uint32_t ph = 0;
@@ -597,7 +599,7 @@ cudaError_t launch_fused_r1(const CUtensorMap* maps, const R1Args& a, int npoly,
 int fused_r1_stages(int K) {
   const int n_kc = K + 6 <= 32 ? 1 : 2;
   const int P = 2 + (n_kc == 2 ? (K > 32 ? 2 : 1) : 0);
-  const uint32_t tb = (uint32_t)P * kR1Plane;
+  const uint32_t tb = (uint32_t)P * (K + 6 <= 16 ? kR1Plane / 2 : kR1Plane);
   int d = (int)((kR1Region - 2 * tb) / tb);
   return d > kR1MaxStages ? kR1MaxStages : d;
 }

@@ -159,6 +159,7 @@ struct TcArgs {
 struct R1Args {
   int64_t N;              // targets
   int n_kc;               // 64-byte operand chunks (32 halves each): 1 or 2
+  int narrow;             // K + 6 <= 16: one chunk of 16 halves (32-byte rows, SWIZZLE_32B maps)
   int kdims;              // coordinate columns (= K): K steps below need all three split products
   int kcols;              // K + 6: steps at or past it are zero padding
   int logw;               // host allows the log-weight mode (decided on the device from wstat)

@@ -390,6 +390,12 @@ __device__ __forceinline__ uint64_t sdesc_k_sw64(const void* smem_ptr) {
   return a | (1ull << 16) | ((uint64_t)(512 >> 4) << 32) | (1ull << 46) | (4ull << 61);
 }
 
+// The same for 32-byte rows (SWIZZLE_32B atoms: 8 rows of 32 B = 256 B apart, layout 6).
+__device__ __forceinline__ uint64_t sdesc_k_sw32(const void* smem_ptr) {
+  const uint64_t a = (uint64_t)((smem_u32(smem_ptr) >> 4) & 0x3FFF);
+  return a | (1ull << 16) | ((uint64_t)(256 >> 4) << 32) | (1ull << 46) | (6ull << 61);
+}
+
 // Instruction descriptor, kind::tf32: D F32 (bits 4-5 = 1), A TF32 (7-9 = 2),
 // B TF32 (10-12 = 2), both K-major, N >> 3 in [17,23), M >> 4 in [24,29).
 // kind::f16 instruction descriptor: D F32 (bit 4), A/B F16 (format 0), K-major, M, N.
