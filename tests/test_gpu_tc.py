@@ -82,6 +82,17 @@ def test_shapes_k_r(oracle_mod, K, R):
     check(oracle_mod, a, W, b, h)
 
 
+@pytest.mark.parametrize("K,R", [(512, 1), (1024, 3), (4096, 1), (4096, 17), (64, 128), (32, 256), (300, 200)])
+def test_abi_extremes_k_r(oracle_mod, K, R):
+    """The ABI accepts K <= 4096 and R <= 256 (include/ks.h): the largest dimensions (operand
+    rows of 128-256 64-byte chunks streamed per unit) and the widest weight blocks (R split into
+    launches of 32 columns, the last one partial) meet the bar.  h scales with sqrt(K) so kernel
+    values stay non-degenerate."""
+    M, N = (700, 260) if K >= 1024 else (1300, 300)
+    a, W, b, h = workloads.custom(M, N, K, R, 0.3 * np.sqrt(K), seed=K + R, wkind="signed")
+    check(oracle_mod, a, W, b, h)
+
+
 @pytest.mark.parametrize("K", [4, 8, 32])
 def test_tensor_core_path_for_low_k(oracle_mod, K):
     """NEXT-3: the tcgen05 path on request for K <= 32, R = 1."""
