@@ -598,8 +598,9 @@ def run_unfused(args):
            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
            "config": {"workload": workload_desc(c),
                       "design": "cuBLAS SGEMM (FP32, TF32 off) of the centred, 2c-prescaled targets x sources "
-                                "into HBM, norm add + clamp + exp2 as PyTorch elementwise passes, cuBLAS GEMM "
-                                "with W; targets chunked to an 8 GiB intermediate (tools/unfused.py)",
+                                "into HBM, then ONE pass reading each element once: norm add, d^2 >= 0 clamp, "
+                                "exp2, times W, row sum (tools/unfused_expw.cu): 8 HBM bytes per pair; targets "
+                                "chunked to a 24 GiB intermediate (tools/unfused.py)",
                       "l2": "flushed before every step"},
            "hbm_bytes_per_pair": bpp,
            "hbm_bound_ms": {k: v * pairs / (load_peaks().get("hbm_gbs", 6545.9) * 1e9) * 1e3 for k, v in bpp.items()},

@@ -295,3 +295,19 @@ def test_auto_policy():
         with ks.KernelSum(32, 1.0, "auto") as plan:
             plan.set_sources(torch.rand((M, 32), device="cuda"), torch.rand((M, 1), device="cuda"))
             assert plan.info()["path"] == want and plan.info()["precision"] == prec
+
+
+# ---------------------------------------------------------------- the paper's grid corners (NEXT-2)
+@pytest.mark.parametrize("orient,K", [("paper", 32), ("paper", 256), ("flip", 32), ("flip", 256)])
+def test_paper_grid_corners(oracle_mod, orient, K):
+    """The corners of the paper's workload grid at M = 524,288 in both
+    orientations (reading Q21): 1,024 weighted sources x 524,288 targets (Alg.1's own, 4,096
+    target tiles of 8 source tiles) and 524,288 sources x 1,024 targets (8 target tiles swept by
+    stream-K), on sampled targets."""
+    if _PREC["p"] == "fp32" and K > 32:
+        pytest.skip("the FP32 kernel serves K <= 32")
+    M = 524288
+    ns, nt = (1024, M) if orient == "paper" else (M, 1024)
+    a, W, b, h = workloads.custom(ns, nt, K, 1, np.sqrt(K) / 4.0, wkind="pos", seed=K + (1 if orient == "paper" else 2))
+    J = workloads.sample_targets(nt, 40 if orient == "paper" else 24, seed=K)
+    check(oracle_mod, a, W, b, h, J=J)
