@@ -1,31 +1,32 @@
-// ks_fused_tc.cu -- the fused tensor-core (tcgen05 / TMEM) kernel-summation
-// kernel for K > 32 or R > 1 weight columns (scope rows a2-a7, TC variant).
+// ks_fused_tc.cu -- the general fused tensor-core (tcgen05 / TMEM) kernel-summation kernel:
+// every (K, R) the dedicated R = 1 kernel (ks_fused_r1.cu: R = 1, split-FP16, K <= 58) does not
+// serve -- R > 1, K > 58, the TF32 modes, and R = 1 with KS_OPT_R1_KERNEL = 0 (scope rows a2-a7).
+// Also the prep kernels of the tensor-core path (a1 sources, a2 targets, FP16 weight split).
 //
 // What it computes (PAPER.md SS III-C, Alg.2; Eq.3):
-//   S_ji = sum_d bh_jd * a_id           (a = 2c alpha_hat, bh = beta_hat)
-//   t_ji = min(S_ji + na_i + nb_j, 0)   (= -log2(e) d^2/(2h^2), clamped d^2 >= 0)
+//   S_ji = sum_d bh_jd * a_id           (a = 2c alpha_hat, bh = beta_hat; split operands)
+//   t_ji = min(S_ji r_j + na_i + nb_j, 0) (= -log2(e) d^2/(2h^2), clamped d^2 >= 0; with the
+//                                          folded layout the norms ride in S)
 //   P_ji = ex2(t_ji) = exp(-||alpha_i - beta_j||^2 / (2h^2))        (Eq.1)
 //   V_jr = sum_i P_ji W_ir                                          (Eq.2)
-// Both contractions run on the 5th-generation tensor cores in TF32 with a
-// hi/lo split of every operand ("3xTF32": lo.hi + hi.lo + hi.hi, the lo.lo
-// term is below FP32 rounding), so the result matches FP32 arithmetic
-// (SS3 reading Q16, SS4 tolerances); KS_PREC_TF32 keeps hi.hi only.
+// Contraction: kind::f16 with FP16 hi/lo splits of power-of-2 scaled operands ("3xF16", the
+// default: lo.hi + hi.lo + hi.hi, reading Q24), or kind::tf32 with TF32 hi/lo ("3xTF32") or a
+// single TF32 product ("TF32", reported separately).
 //
-// Structure (one persistent 384-thread CTA per SM, stream-K over
-// (128-target tile x 128-source tile) units, like the FP32 kernel):
-//   warp 0   TMA producer: per unit, the W^T tile (hi/lo, 3-D box) and na into
-//            a 2-slot ring; per 16-wide K chunk, A = targets (hi/lo) and
-//            B = sources (hi/lo) tiles (SWIZZLE_64B) into an S-stage ring.
-//   warp 1   MMA issuer (one thread): S(q) = A B^T into TMEM buffer q%2
-//            (M=128, N=128, K=8 per instruction), then V(q-1) += P(q-1) W
-//            with P read from TMEM (A operand in TMEM, M=128, N=r_c, K=8).
-//   warp 2   TMEM allocation (512 columns: S0 | S1 | P_lo | V).
-//   warps 4-11 epilogue: tcgen05.ld S, add norms, clamp, MUFU ex2, split P into
-//            TF32 hi/lo, tcgen05.st P_hi in place of S and P_lo beside it;
-//            every <= 4 units read V (FP32 TMEM accumulator) into FP64
-//            registers; at segment end write V or a partial + deterministic
-//            last-arriver fix-up (no atomics on V).
-// The M x N kernel matrix exists only as 128x128 TMEM tiles.
+// Structure (one persistent 640-thread CTA per SM, full waves of target tiles then a stream-K
+// remainder with a deterministic last-arriver fix-up):
+//   warp 0   TMA producer of the operand stages (targets resident per target tile where they
+//            fit: R = 1 with <= 2 operand chunks, or the FP16 V-MMA kernel at K <= 256);
+//   warp 1   MMA issuer: S(q) = A B^T into TMEM (M = 128; N = 256 sources with the weighted sum
+//            on CUDA cores, 128 otherwise), then with the tensor-core weighted sum V += P W with
+//            P read from TMEM;
+//   warp 2   TMEM allocation (512 columns);
+//   warp 3   producer of the per-tile source norms / weights (own ring);
+//   warps 4-19  16 epilogue warps: tcgen05.ld S, norms, exp2 (MUFU.EX2, part on the FMA pipe
+//            for R = 1), then either the weighted sum on CUDA cores (R <= 16: two ping-pong
+//            groups on alternate tiles) or P split into FP16 (or TF32) hi/lo written back to TMEM
+//            for the V MMA; V folded into FP64 and written (or a stream-K partial slot).
+// The M x N kernel matrix exists only as TMEM tiles.
 #include "ks_internal.h"
 #include <cuda_fp16.h>
 #include "ks_ptx.cuh"
