@@ -84,7 +84,8 @@ typedef struct {
   int64_t fused_launches; /* cumulative launches of the fused kernel         */
   double c_log2;        /* c = log2(e) / (2 h^2), the ex2 prescale           */
   int kernel;           /* 0 none, 1 FP32 kernel, 2 general tcgen05 kernel,
-                           3 R = 1 tcgen05 kernel (ks_fused_r1.cu)            */
+                           3 R = 1 tcgen05 kernel (ks_fused_r1.cu),
+                           4 R > 1 tcgen05 kernel (ks_fused_rv.cu)            */
   int exp_poly;         /* exponential pairs of every 16 on the FMA pipe      */
   int r1_epilogue;      /* R = 1 kernel: KS_OPT_R1_EPILOGUE in effect (0 log-
                            weights, no d^2 clamp; 1 clamp; 2 |d^2|; 3 none)  */
@@ -151,15 +152,17 @@ KS_API ks_status ks_eval_host(ks_ctx *ctx, const float *beta, int64_t N, float *
  * beside an option, when set at ks_create, gives its initial value (read once there;
  * later calls never read the environment). */
 typedef enum {
-  KS_OPT_R1_KERNEL = 1,       /* KS_R1: 1 (default) the dedicated R = 1 kernel where it applies
-                                 (split-FP16, K <= 58), 0 the general tcgen05 kernel [sources] */
+  KS_OPT_R1_KERNEL = 1,       /* KS_R1: 1 (default) the dedicated folded kernels where they apply
+                                 (split-FP16, K <= 58: R = 1 and R > 1), 0 the general tcgen05
+                                 kernel [sources] */
   KS_OPT_R1_EPILOGUE = 2,     /* KS_R1_MODE: 0 (default) log-weights when every W_i >= 0 (no
                                  d^2 >= 0 clamp; any W_i < 0 takes mode 1), 1 weights with the
                                  d^2 >= 0 clamp, 2 weights with d^2 -> |d^2|, 3 weights without
                                  a clamp [sources] */
   KS_OPT_EXP_POLY = 3,        /* KS_R1_POLY: exponential pairs of every 16 computed on the FMA
                                  pipe instead of MUFU (0, 4..8; -1 default) [eval] */
-  KS_OPT_WEIGHTED_SUM = 4,    /* KS_TC_VCC: -1 auto, 0 tensor cores, 1 CUDA cores (R <= 16) [sources] */
+  KS_OPT_WEIGHTED_SUM = 4,    /* KS_TC_VCC: -1 auto, 0 tensor cores, 1 CUDA cores (R <= 16; the
+                                 general kernel) [sources] */
   KS_OPT_LOG_WEIGHTS = 5,     /* KS_TC_LOGW: general kernel, R = 1: 1 (default) / 0 [sources] */
   KS_OPT_FOLD = 6,            /* KS_TC_FOLD: general kernel, R = 1: -1 auto, 0 off, 1 forced [sources] */
   KS_OPT_AUG = 7,             /* KS_TC_AUG: TF32 modes: -1 auto, 0, 1 norms in 2 K columns [sources] */

@@ -142,6 +142,7 @@ struct ks_ctx {
   int tc_kcols = 0, tc_kdims = 0;  // live operand columns / columns needing every split product
   int tc_vcc = 0;  // RV: weighted sum on CUDA cores over RV padded columns (0: tensor-core V path)
   int r1 = 0;      // R = 1 folded kernel (ks_fused_r1.cu): 2 = log-weight mode allowed, 3 = weight mode only
+  int rv = 0;      // R > 1 folded kernel (ks_fused_rv.cu)
   int r1_clamp = 0;
   CUtensorMap tmB_hi, tmB_lo;
   DBuf<float> mu;         // [k_pad]
@@ -412,12 +413,12 @@ ks_status encode_wt(CUtensorMap* map, const float* base, int64_t m_pad, int r_pa
 // wcat [2 r_pad][m_pad] FP16 viewed as {32 sources, 2 r_pad rows, m_pad/32 chunks}: one box =
 // 4 chunks x 2 r_c rows x 64 B = the K-major SWIZZLE_64B B operand ([W_hi | W_lo] rows) of the
 // FP16 V-MMA for one 128-source tile.
-ks_status encode_wcat(CUtensorMap* map, const void* base, int64_t m_pad, int r_pad, int r_c) {
+ks_status encode_wcat(CUtensorMap* map, const void* base, int64_t m_pad, int r_pad, int r_c, int tile_s) {
   PFN_encodeTiled enc = get_encode();
   if (!enc) return fail(KS_ECUDA, "cuTensorMapEncodeTiled unavailable from the driver");
   cuuint64_t dims[3] = {32, (cuuint64_t)(2 * r_pad), (cuuint64_t)(m_pad / 32)};
   cuuint64_t strides[2] = {(cuuint64_t)m_pad * 2, 64};
-  cuuint32_t box[3] = {32, (cuuint32_t)(2 * r_c), (cuuint32_t)(ks::kTcTileS / 32)};
+  cuuint32_t box[3] = {32, (cuuint32_t)(2 * r_c), (cuuint32_t)(tile_s / 32)};
   cuuint32_t estr[3] = {1, 1, 1};
   CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 3, const_cast<void*>(base), dims, strides, box, estr,
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
@@ -464,23 +465,33 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   // reading Q28).  KS_OPT_R1_EPILOGUE: 0 = log-weights when every W_i >= 0 (decided on the
   // device), else the weight mode with the clamp; 1 = weight mode with the d^2 >= 0 clamp for any
   // W; 2 = weight mode with |d^2|; 3 = weight mode without a clamp.
-  int r1 = 0, r1_clamp = 0;
+  int r1 = 0, r1_clamp = 0, rv = 0;
   if (f16 && vcc == 1 && K + 6 <= 2 * 2 * ks::kTcKC && ks::opt(KS_OPT_R1_KERNEL, 1) != 0) {
     const int mode = ks::opt(KS_OPT_R1_EPILOGUE, 0);
     r1 = mode == 0 ? 2 : 3;
     r1_clamp = mode == 3 ? 0 : mode == 2 ? 2 : 1;
     fold = r1;
   }
+  // R > 1, split-FP16, K + 6 <= 64: the multi-column kernel (ks_fused_rv.cu) on the same skeleton,
+  // weighted sum as a second tcgen05 MMA (fold mode 4: norms + the 2^14 P scale in the
+  // contraction; the FP16 weight split of reading Q27).  KS_OPT_R1_KERNEL = 0 selects the general
+  // kernel for both.
+  if (f16 && R > 1 && K + 6 <= 2 * 2 * ks::kTcKC && ks::opt(KS_OPT_R1_KERNEL, 1) != 0 &&
+      ks::opt(KS_OPT_WEIGHTED_SUM, -1) != 1) {
+    rv = 1;
+    vcc = 0;
+    fold = 4;
+  }
   // k_pad in elements: one 64-byte row chunk per pipeline stage = 16 FP32 or 32 FP16; the R = 1
   // kernel at K + 6 <= 16 keeps 32-byte rows (16 halves: half the operand bytes; cfg5's prepared
   // source set, 1,048,576 x 2 x 32 B, then stays in the 126 MB L2)
-  const bool narrow = r1 && K + 6 <= ks::kTcKC;
+  const bool narrow = (r1 || rv) && K + 6 <= ks::kTcKC;
   const int k_pad = narrow ? ks::kTcKC
                     : f16 ? (int)round_up(K + 6 * (fold ? 1 : 0), 2 * ks::kTcKC) : tc_k_pad(K);
   const int aug = f16 ? 0 : tc_aug(K);  // FP16 mode: norms stay in FP32 in the epilogue (or fold)
   const int tile_s = ks::fused_tc_tile_s(vcc);
-  const int box_s = r1 ? 128 : tile_s;  // sources per operand tile of the kernel
-  const int64_t m_pad = round_up(M > 0 ? M : 1, tile_s);
+  const int box_s = r1 ? 128 : rv ? ks::kRvTileS : tile_s;  // sources per operand tile of the kernel
+  const int64_t m_pad = round_up(M > 0 ? M : 1, rv ? ks::kRvTileS : tile_s);
   const int r_pad = (int)round_up(R, 16);
   cudaStream_t st = ctx->stream;
   const size_t nsrc = f16 ? ((size_t)m_pad * k_pad + 1) / 2 : (size_t)m_pad * k_pad, nw = (size_t)r_pad * m_pad;
@@ -529,6 +540,7 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   ctx->tc_fold = fold;  // 1: general kernel (device-side f16_fold_ok); 2, 3: R = 1 kernel (fold shift)
   ctx->r1 = r1;
   ctx->r1_clamp = r1_clamp;
+  ctx->rv = rv;
   ctx->tc_kcols = f16 ? K + 6 * (fold ? 1 : 0) : K + 2 * aug;
   ctx->tc_kdims = f16 ? K : K + 2 * aug;
   ctx->tc_vcc = vcc;
@@ -612,6 +624,90 @@ ks_status eval_r1(ks_ctx* ctx, const CUtensorMap* maps, int64_t N, float* V) {
   return KS_OK;
 }
 
+// R > 1 folded kernel (ks_fused_rv.cu): 96-source units, one launch per block of 16 or 32
+// weight columns.
+ks_status eval_rv(ks_ctx* ctx, CUtensorMap* maps, int64_t N, float* V) {
+  cudaStream_t st = ctx->stream;
+  ks::StreamK sk;
+  sk.n_t = round_up(N, ks::kTcTileT) / ks::kTcTileT;
+  sk.n_s = (int32_t)(ctx->m_pad / ks::kRvTileS);
+  sk.units = sk.n_t * (int64_t)sk.n_s;
+  int64_t g = ctx->num_sms;
+  if (g > sk.units) g = sk.units;
+  sk.grid = (int32_t)g;
+  KS_CUDA(ctx->partial.reserve((size_t)sk.grid * 2 * 128 * 32, st, false), "allocate partials");
+  KS_CUDA(ctx->counters.reserve((size_t)sk.n_t, st, true), "allocate tile counters");
+  ks::RvArgs a;
+  a.N = N;
+  a.narrow = ctx->k_pad == ks::kTcKC ? 1 : 0;
+  a.n_kc = a.narrow ? 1 : ctx->k_pad / 32;
+  a.kdims = ctx->tc_kdims;
+  a.kcols = ctx->tc_kcols;
+  a.R = ctx->R;
+  a.wcol = ctx->wcol.p;
+  a.V = V;
+  a.partial = ctx->partial.p;
+  a.counters = ctx->counters.p;
+  a.sk = sk;
+  a.trace = nullptr;
+  a.cta_times = nullptr;
+  if (ctx->opts.v[KS_OPT_MEASURE_CLOCK]) {  // the first launch (columns 0 .. r_c - 1) is measured
+    KS_CUDA(ctx->clk_buf.reserve((size_t)ctx->num_sms * 4, st, false), "allocate clock buffer");
+    a.cta_times = ctx->clk_buf.p;
+    ctx->clk_ctas = sk.grid;
+  }
+  a.dbg = 0;
+#if KS_DEBUG
+  {
+    const char* e = getenv("KS_RV_DEBUG");  // measurement builds only: drops work, wrong results
+    a.dbg = e ? atoi(e) : 0;
+  }
+#endif
+  const char* dbg = ctx->cta_times_path.empty() ? nullptr : ctx->cta_times_path.c_str();
+  if (dbg) {  // KS_TRACE builds write the unit clocks of CTA 0 (first 16/32-column launch)
+    KS_CUDA(ctx->dbg_times.reserve((size_t)12 * 4096, st, true), "allocate debug timers");
+    KS_CUDA(cudaMemsetAsync(ctx->dbg_times.p, 0, (size_t)12 * 4096 * 8, st), "zero debug timers");
+    a.trace = ctx->dbg_times.p;
+  }
+  for (int r_off = 0; r_off < ctx->r_pad;) {
+    const int r_c = (ctx->r_pad - r_off >= 32) ? 32 : 16;
+    a.r_c = r_c;
+    a.r_off = r_off;
+    a.r_valid = (ctx->R - r_off < r_c) ? (ctx->R - r_off) : r_c;
+    ks_status s = encode_wcat(&maps[4], ctx->wt_hi.p, ctx->m_pad, ctx->r_pad, r_c, ks::kRvTileS);
+    if (s != KS_OK) return s;
+    cudaEvent_t stop;
+    s = timed_begin(ctx, &stop);
+    if (s != KS_OK) return s;
+    KS_CUDA(ks::launch_fused_rv(maps, a, st), "fused R > 1 kernel launch");
+    ctx->launches++;
+    ctx->fused_launches++;
+    ctx->last_grid = sk.grid;
+    s = timed_end(ctx, stop);
+    if (s != KS_OK) return s;
+    r_off += r_c;
+    a.trace = nullptr;
+    a.cta_times = nullptr;
+  }
+  if (dbg) {
+    std::vector<unsigned long long> h((size_t)12 * 4096);
+    KS_CUDA(cudaMemcpyAsync(h.data(), ctx->dbg_times.p, h.size() * 8, cudaMemcpyDeviceToHost, st), "copy trace");
+    KS_CUDA(cudaStreamSynchronize(st), "synchronize");
+    FILE* f = fopen(dbg, "a");
+    if (f) {  // per unit: S issued, epilogue wake, P ready, V issued, S waits done, V waits done,
+              // V vempty done, V pready done, fold start, fold end, -, -
+      for (int q = 0; q < 4096 && h[12 * q] != 0; ++q) {
+        fprintf(f, "trace %d", q);
+        for (int k = 0; k < 12; ++k) fprintf(f, " %llu", h[12 * q + k]);
+        fprintf(f, "\n");
+      }
+      fprintf(f, "--\n");
+      fclose(f);
+    }
+  }
+  return KS_OK;
+}
+
 ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   cudaStream_t st = ctx->stream;
   const int k_pad = ctx->k_pad;
@@ -633,7 +729,7 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   }
   ctx->launches += 1;
   CUtensorMap maps[6];
-  const bool narrow = ctx->r1 && k_pad == ks::kTcKC;  // 32-byte operand rows (R = 1 kernel, K + 6 <= 16)
+  const bool narrow = (ctx->r1 || ctx->rv) && k_pad == ks::kTcKC;  // 32-byte operand rows (K + 6 <= 16)
   ks_status s = encode_2d_sw64(&maps[0], ctx->tgt_hi.p, k_pad, n_pad, ks::kTcTileT, f16, narrow);
   if (s != KS_OK) return s;
   s = encode_2d_sw64(&maps[1], ctx->tgt_lo.p, k_pad, n_pad, ks::kTcTileT, f16, narrow);
@@ -641,6 +737,7 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   maps[2] = ctx->tmB_hi;
   maps[3] = ctx->tmB_lo;
   if (ctx->r1) return eval_r1(ctx, maps, N, V);
+  if (ctx->rv) return eval_rv(ctx, maps, N, V);
 
   ks::StreamK sk;
   sk.n_t = n_pad / ks::kTcTileT;
@@ -705,7 +802,7 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
     a.r_off = r_off;
     a.r_valid = (ctx->R - r_off < r_c) ? (ctx->R - r_off) : r_c;
     if (f16) {  // FP16 V-MMA: one wcat map (hi and lo rows of the r_c columns in one box)
-      s = encode_wcat(&maps[4], ctx->wt_hi.p, ctx->m_pad, ctx->r_pad, r_c);
+      s = encode_wcat(&maps[4], ctx->wt_hi.p, ctx->m_pad, ctx->r_pad, r_c, ks::kTcTileS);
       if (s != KS_OK) return s;
       maps[5] = maps[4];
     } else {
@@ -1069,7 +1166,7 @@ ks_status ks_get_info(const ks_ctx* ctx, ks_info* out) {
   out->k_pad = ctx->k_pad;
   const bool tc = ctx->have_src && ctx->path == KS_PATH_TC;
   out->tile_t = tc ? ks::kTcTileT : ks::kTileT;
-  out->tile_s = tc ? (ctx->r1 ? 128 : ks::fused_tc_tile_s(ctx->tc_vcc)) : ks::kTileS;
+  out->tile_s = tc ? (ctx->r1 ? 128 : ctx->rv ? ks::kRvTileS : ks::fused_tc_tile_s(ctx->tc_vcc)) : ks::kTileS;
   out->num_ctas = ctx->last_grid;
   out->stages = !ctx->k_pad ? 0
                 : tc && ctx->r1 ? ks::fused_r1_stages(ctx->K)
@@ -1083,8 +1180,10 @@ ks_status ks_get_info(const ks_ctx* ctx, ks_info* out) {
   out->launches = ctx->launches;
   out->fused_launches = ctx->fused_launches;
   out->c_log2 = ctx->c;
-  out->kernel = !ctx->have_src ? 0 : ctx->path == KS_PATH_FP32 ? 1 : ctx->r1 ? 3 : 2;
-  out->exp_poly = ctx->r1 ? ks::r1_poly_for(ctx->opts.v[KS_OPT_EXP_POLY]) : ctx->opts.v[KS_OPT_EXP_POLY];
+  out->kernel = !ctx->have_src ? 0 : ctx->path == KS_PATH_FP32 ? 1 : ctx->r1 ? 3 : ctx->rv ? 4 : 2;
+  out->exp_poly = ctx->r1   ? ks::r1_poly_for(ctx->opts.v[KS_OPT_EXP_POLY])
+                  : ctx->rv ? ks::rv_poly_for(ctx->opts.v[KS_OPT_EXP_POLY])
+                            : ctx->opts.v[KS_OPT_EXP_POLY];
   out->r1_epilogue = ctx->r1 ? ctx->opts.v[KS_OPT_R1_EPILOGUE] : -1;
   return KS_OK;
 }

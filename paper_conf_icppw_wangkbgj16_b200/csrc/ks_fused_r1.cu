@@ -217,6 +217,8 @@ __global__ void __launch_bounds__(kR1Threads, 1)
   const uint32_t tile_bytes = (uint32_t)P * plane;
   int D = (int)((kR1Region - 2 * tile_bytes) / tile_bytes);
   if (D > kR1MaxStages) D = kR1MaxStages;
+  D &= ~1;  // even: the S-MMA warp of unit q (q & 1) also issues unit q + D, so it waits on every
+            // phase of a stage's full barrier (a parity wait must never skip a phase)
   const uint32_t offA = 0, offS = 2 * tile_bytes;
   uint8_t* wring = smem + kR1Region;
   double* red = reinterpret_cast<double*>(smem + kR1Region + kR1Ring);  // [4 groups][128 rows]

@@ -1349,8 +1349,10 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
   const float nai = live ? (float)(-c * n) : 0.f;
   const double c2 = 2.0 * c;
   // aug (FP16): 1 folded layout when f16_fold_ok, 2 always folded (fold shift), 3 the same
-  // without log-weights (the R = 1 kernel's weight mode)
-  const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && !(F16 && aug == 3);
+  // without log-weights (the R = 1 kernel's weight mode), 4 the same plus the exponent offset
+  // kPExp (the multi-column kernel's P 2^kPExp, reading Q27: the MMA delivers t + 14)
+  const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && !(F16 && aug >= 3);
+  const double eoff = (F16 && aug == 4) ? 14.0 : 0.0;
   // log2(W_i / Wmax) (R = 1, W >= 0; -inf for W_i = 0 and padding)
   const double wl = !logw ? 0.0 : live ? log2((double)W[i]) - log2((double)__uint_as_float(wstat[0])) : -INFINITY;
   float sA = 1.f;
@@ -1363,7 +1365,7 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
       const int fsh = aug >= 2 ? f16_fold_shift(amax, c, K) : 0;
       one = __float2half(ldexpf(1.f, fsh));
       sA = ldexpf(1.f, f16_fold_exp(c));
-      const double nf = ldexp(-c * n + wl, -fsh);  // finite unless W_i = 0: then the FP16 stand-in for -inf
+      const double nf = ldexp(-c * n + wl + eoff, -fsh);  // finite unless W_i = 0: then the FP16 stand-in for -inf
       if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
       else split3_f16(nf, np);
     } else {

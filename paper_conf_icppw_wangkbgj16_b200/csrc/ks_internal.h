@@ -114,6 +114,7 @@ namespace ks {
 // ---------------------------------------------------------------- tensor-core (tcgen05) path
 constexpr int kTcTileT = 128;  // targets per tile = MMA M = TMEM lanes
 constexpr int kTcTileS = 128;  // sources per tile = N of the S MMA = K of the V MMA
+constexpr int kRvTileS = 96;   // sources per unit of the R > 1 kernel (ks_fused_rv.cu)
 constexpr int kTcKC = 16;      // K floats per pipeline stage (64-byte rows, SWIZZLE_64B)
 constexpr int kTcEpiWarps = 16;  // epilogue warps (4 per TMEM lane group)
 constexpr int kTcThreads = 128 + 32 * kTcEpiWarps;  // warp 0 operand TMA, 1 MMA, 2 TMEM alloc, 3 norms/weights loads, 4.. epilogue
@@ -175,6 +176,25 @@ struct R1Args {
   int dbg;                // KS_DEBUG builds only (KS_R1_DEBUG): 1 no epilogue math, 2 no MMAs, 3 neither, 4 + no source loads
 };
 cudaError_t launch_fused_r1(const CUtensorMap* maps, const R1Args& a, int npoly, cudaStream_t st);
+
+// ---------------------------------------------------------------- R > 1 folded kernel (ks_fused_rv.cu)
+// Split-FP16, K + 6 <= 64, weights as the FP16 V-MMA's wcat (launch_prep_wcat); r_c = 16 or 32
+// weight columns per launch.  maps: A_hi, A_lo, B_hi, B_lo (128-row boxes), wcat (encode_wcat).
+struct RvArgs {
+  int64_t N;
+  int n_kc, narrow, kdims, kcols;
+  int r_c, r_off, r_valid, R;  // columns of this launch, first column, valid ones, V row stride
+  const unsigned* wcol;        // [r_pad] FP32 bits of max_i |W_ir| (column scale exponents)
+  float* V;                    // [N][R]
+  float* partial;              // [grid][2][128][r_c]
+  int* counters;               // [n_t]
+  StreamK sk;
+  unsigned long long* trace;   // KS_TRACE builds: [4096][12] unit clocks of CTA 0, or nullptr
+  int dbg;                     // KS_DEBUG builds: work-dropping bits (ks_fused_rv.cu), else 0
+  unsigned long long* cta_times;  // KS_OPT_MEASURE_CLOCK: [grid][4] globaltimer / clock64 at start, end
+};
+cudaError_t launch_fused_rv(const CUtensorMap* maps, const RvArgs& a, cudaStream_t st);
+int rv_poly_for(int opt_value);
 int fused_r1_stages(int K);
 int r1_poly();
 int r1_poly_for(int opt_value);  // the NPOLY the R = 1 kernel runs for a KS_OPT_EXP_POLY value
