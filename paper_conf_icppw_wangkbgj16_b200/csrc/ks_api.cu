@@ -442,11 +442,13 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   // Weighted sum: on CUDA cores (vcc = padded R, 256-source tiles) or as a second tensor-core
   // MMA (vcc = 0).  Split-FP16 crossover measured at M = N = 65,536 (tools/vsweep.py, DESIGN.md
   // SS7): the tensor-core V costs the same for any R, the CUDA-core V grows with R -- CUDA cores
-  // for R <= 4, and for R <= 8 when K > 48; TF32 modes keep CUDA cores up to R = 16.
+  // for R <= 4, for R <= 8 when K > 48, and for R <= 16 when K >= 256 (measured round 2,
+  // profiles/r02/policy_sweeps.txt: K = 256, R = 16 at 262,144^2 ties within 0.5%, R = 8 is 20%
+  // faster on CUDA cores); TF32 modes keep CUDA cores up to R = 16.
   // KS_OPT_WEIGHTED_SUM = 0 / 1 forces the tensor-core / CUDA-core (R <= 16) variant.
   const int ovs = ks::opt(KS_OPT_WEIGHTED_SUM, -1);
   int vcc = ks::fused_tc_rv(R);
-  if (f16 && (R > 8 || (R > 4 && K <= 48))) vcc = 0;
+  if (f16 && (R > 8 || (R > 4 && K <= 48)) && !(K >= 256 && R <= 16)) vcc = 0;
   if (ovs == 0) vcc = 0;
   if (ovs == 1) vcc = ks::fused_tc_rv(R);
   // R = 1 with W >= 0: log-weights in na (decided on the device, no host sync);
