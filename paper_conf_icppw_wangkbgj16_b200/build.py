@@ -32,26 +32,59 @@ def _headers():
         glob.glob(os.path.join(ROOT, "include", "*.h"))
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    os.makedirs(BUILD, exist_ok=True)
+def build(force: bool = False, verbose: bool = False, extra=None, lib: str = None, build_dir: str = None) -> str:
+    """Compile csrc/*.cu (in parallel) and link the library.  `extra` adds nvcc flags (the
+    measurement library: build_debug()); `lib` / `build_dir` default to libks.so / _build."""
+    from concurrent.futures import ThreadPoolExecutor
+    lib = lib or LIB
+    build_dir = build_dir or BUILD
+    flags = FLAGS + list(extra or [])
+    os.makedirs(build_dir, exist_ok=True)
     srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")))
     hdr_mtime = max([os.path.getmtime(h) for h in _headers()] + [0])
-    objs = []
+    objs, cmds = [], []
     for s in srcs:
-        o = os.path.join(BUILD, os.path.basename(s)[:-3] + ".o")
+        o = os.path.join(build_dir, os.path.basename(s)[:-3] + ".o")
         objs.append(o)
         if force or not os.path.exists(o) or os.path.getmtime(o) < max(os.path.getmtime(s), hdr_mtime):
-            cmd = [NVCC, *ARCH, *FLAGS, "-c", s, "-o", o]
+            cmd = [NVCC, *ARCH, *flags, "-c", s, "-o", o]
             if verbose:
                 cmd.insert(1, "-Xptxas=-v")
                 print(" ".join(cmd), flush=True)
-            subprocess.check_call(cmd)
-    if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < max(os.path.getmtime(o) for o in objs):
-        tmp = LIB + f".tmp{os.getpid()}"
+            cmds.append(cmd)
+    if cmds:
+        with ThreadPoolExecutor(max_workers=min(len(cmds), os.cpu_count() or 1)) as ex:
+            for f in [ex.submit(subprocess.check_call, c) for c in cmds]:
+                f.result()
+    if force or not os.path.exists(lib) or os.path.getmtime(lib) < max(os.path.getmtime(o) for o in objs):
+        tmp = lib + f".tmp{os.getpid()}"
         subprocess.check_call([NVCC, *ARCH, "-shared", "-cudart", "static", *objs, "-o", tmp])
-        os.replace(tmp, LIB)
-    return LIB
+        os.replace(tmp, lib)
+    return lib
+
+
+DBG_LIB = os.path.join(PKG, "libks_dbg.so")
+
+
+def build_debug(debug: int = 1, prof: int = 0, trace: int = 0, force: bool = False) -> str:
+    """The measurement library libks_dbg.so (never the shipped libks.so; selected with
+    KS_LIB=libks_dbg.so): KS_DEBUG work-dropping knobs and bounded waits, KS_PROF phase clocks,
+    KS_TRACE unit timeline.  Objects are rebuilt when the flags change."""
+    flags = [f"-DKS_DEBUG={debug}", f"-DKS_PROF={prof}", f"-DKS_TRACE={trace}"]
+    bdir = BUILD + "_dbg"
+    stamp = os.path.join(bdir, "flags")
+    os.makedirs(bdir, exist_ok=True)
+    old = open(stamp).read() if os.path.exists(stamp) else ""
+    if old != " ".join(flags):
+        force = True
+    lib = build(force=force, extra=flags, lib=DBG_LIB, build_dir=bdir)
+    with open(stamp, "w") as f:
+        f.write(" ".join(flags))
+    return lib
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    if "--debug" in sys.argv:
+        print(build_debug(force="--force" in sys.argv))
+    else:
+        print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))

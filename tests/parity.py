@@ -25,6 +25,8 @@ def e_norm(V_gpu, V_ref, W):
     d = np.abs(V_gpu - V_ref)                       # [n, R]
     if d.size == 0:
         return 0.0
+    if not np.all(np.isfinite(V_gpu)):             # NaN / inf never pass (max() would skip a NaN)
+        return float("inf")
     out = 0.0
     for r in range(V_ref.shape[1]):
         if sw[r] == 0.0:

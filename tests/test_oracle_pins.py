@@ -260,7 +260,8 @@ def test_alg1_crosscheck(oracle_mod, cfg):
 # ---------------------------------------------------------------- harness self-test
 def test_metric_catches_injected_bugs(oracle_mod):
     """The parity metric must FAIL for the bugs a kernel could plausibly have
-    (SS4): dropping the last 128-source tile, h off by 1%, 2h^2 -> h^2.
+    (SS4): dropping the last 128-source tile, h off by 1%, 2h^2 -> h^2, a NaN or inf
+    output (found by the GPU-side self-test, tests/test_gpu_harness.py: max() skipped NaNs).
     W >= 0 on the cfg3 distribution (the signed-W metric is lenient)."""
     a, W, b, h = workloads.make(3, M=4096, N=128, wkind="pos")
     h = float(h)
@@ -270,6 +271,12 @@ def test_metric_catches_injected_bugs(oracle_mod):
         "h_x1.01": ev(oracle_mod, a, W, b, h * 1.01),
         "2h2_to_h2": ev(oracle_mod, a, W, b, h / math.sqrt(2.0)),
     }
+    Vn = V.copy()
+    Vn[7, 0] = np.nan  # one non-finite output (a kernel reading garbage) -- max() alone skips a NaN
+    bugs["one_nan"] = Vn
+    Vi = V.copy()
+    Vi[0, 0] = np.inf
+    bugs["one_inf"] = Vi
     for name, Vb in bugs.items():
         assert e_norm(Vb, V, W) > 1e-5, name
     assert e_norm(V.astype(np.float32), V, W) < 1e-7
