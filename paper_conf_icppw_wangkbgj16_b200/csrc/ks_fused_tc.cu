@@ -1333,8 +1333,16 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
                                        void* __restrict__ src_lo, float* __restrict__ na,
                                        float* __restrict__ wt_hi, float* __restrict__ wt_lo,
                                        float* __restrict__ wv, int rv, const unsigned* __restrict__ wstat) {
-  pdl_trigger();  // let the next kernel launch early
-  pdl_wait();     // the source statistics are complete
+  pdl_wait();  // the source statistics are complete (the trigger for the next grid is at the end)
+  // uniform values, once per block (FP64 log2 per thread made the kernel issue-bound)
+  __shared__ int s_fsh, s_fexp;
+  __shared__ double s_lwmax;
+  if (threadIdx.x == 0) {
+    s_fsh = (F16 && aug >= 2) ? f16_fold_shift(amax, c, K) : 0;
+    s_fexp = F16 ? f16_fold_exp(c) : 0;
+    s_lwmax = (wstat != nullptr && wstat[0] != 0u) ? log2((double)__uint_as_float(wstat[0])) : 0.0;
+  }
+  __syncthreads();
   const int lane = threadIdx.x & 31, gl = lane & (G - 1);
   const int64_t i = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
   if (i >= m_pad) return;
@@ -1353,25 +1361,33 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
   // kPExp (the multi-column kernel's P 2^kPExp, reading Q27: the MMA delivers t + 14)
   const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && !(F16 && aug >= 3);
   const double eoff = (F16 && aug == 4) ? 14.0 : 0.0;
-  // log2(W_i / Wmax) (R = 1, W >= 0; -inf for W_i = 0 and padding)
-  const double wl = !logw ? 0.0 : live ? log2((double)W[i]) - log2((double)__uint_as_float(wstat[0])) : -INFINITY;
+  // log2(W_i / Wmax) (R = 1, W >= 0; -inf for W_i = 0 and padding); FP64 log2, so only the
+  // lanes that store it evaluate it
+  auto wl_of = [&]() -> double { return !logw ? 0.0 : live ? log2((double)W[i]) - s_lwmax : -INFINITY; };
   float sA = 1.f;
   bool fa = false;  // folded layout active
+  int fsh = 0;
   __half np[3] = {__float2half(0.f), __float2half(0.f), __float2half(0.f)};
+  bool np_ready = false;
   __half one = __float2half(1.f);  // unit columns (times the target's norm pieces): 2^s
   if constexpr (F16) {
     fa = aug >= 2 || (aug == 1 && f16_fold_ok(amax, c, K));
     if (fa) {
-      const int fsh = aug >= 2 ? f16_fold_shift(amax, c, K) : 0;
+      fsh = s_fsh;
       one = __float2half(ldexpf(1.f, fsh));
-      sA = ldexpf(1.f, f16_fold_exp(c));
-      const double nf = ldexp(-c * n + wl + eoff, -fsh);  // finite unless W_i = 0: then the FP16 stand-in for -inf
-      if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
-      else split3_f16(nf, np);
+      sA = ldexpf(1.f, s_fexp);
     } else {
       sA = ldexpf(1.f, f16_scale_exp((float)(c2 * (double)__uint_as_float(*amax))));
     }
   }
+  // the folded norm pieces, for the lanes that store columns K .. K + 2
+  auto need_np = [&]() {
+    if (np_ready) return;
+    np_ready = true;
+    const double nf = ldexp(-c * n + wl_of() + eoff, -fsh);  // finite unless W_i = 0: then the FP16 stand-in for -inf
+    if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
+    else split3_f16(nf, np);
+  };
   auto coord = [&](int d) -> float {
     if (d < K) {
       const float x = live ? alpha[i * K + d] - mu[d] : 0.f;
@@ -1387,6 +1403,7 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
       __half h0, l0, h1, l1;
       split_f16(a0 * sA, h0, l0);  // exact power-of-2 scaling
       split_f16(a1 * sA, h1, l1);
+      if (fa && d + 1 >= K && d < K + 3) need_np();
       if (fa && d >= K && d < K + 6) {  // folded norm columns: hi planes only
         h0 = d < K + 3 ? np[d - K] : one;
         l0 = __float2half(0.f);
@@ -1403,6 +1420,7 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
       static_cast<float2*>(src_lo)[(i * k_pad + d) >> 1] = make_float2(to_tf32(a0 - ah0), to_tf32(a1 - ah1));
     }
   }
+  const double wl = (gl == 0 && logw && !fa) || (gl == 0 && logw && rv > 0) ? wl_of() : 0.0;
   if (gl == 0) {
     if (fa) {
       na[i] = 0.f;  // folded: the norm and log-weight ride in the contraction
@@ -1425,6 +1443,9 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
     wt_hi[(int64_t)r * m_pad + i] = wh;
     wt_lo[(int64_t)r * m_pad + i] = to_tf32(w - wh);
   }
+  // PDL trigger last: a dependent fused kernel's CTA (640 threads, nearly all of an SM's registers)
+  // launched early would hold its SM while waiting and starve this grid's remaining blocks
+  pdl_trigger();
 }
 
 template <bool F16, int G>
@@ -1433,8 +1454,13 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
                                        const unsigned* __restrict__ amax, void* __restrict__ tgt_hi,
                                        void* __restrict__ tgt_lo, float* __restrict__ nb,
                                        float* __restrict__ tsc) {
-  pdl_trigger();  // let the fused kernel's CTAs start their prologue
-  pdl_wait();     // the source statistics (mu, amax) are complete
+  pdl_wait();  // the source statistics (mu, amax) are complete (trigger at the end)
+  __shared__ int s_fsh, s_fexp;  // uniform, once per block (FP64 log2)
+  if (threadIdx.x == 0) {
+    s_fsh = (F16 && aug >= 2) ? f16_fold_shift(amax, c, K) : 0;
+    s_fexp = F16 ? f16_fold_exp(c) : 0;
+  }
+  __syncthreads();
   const int lane = threadIdx.x & 31, gl = lane & (G - 1);
   const int64_t j = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
   if (j >= n_pad) return;
@@ -1456,12 +1482,15 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
   if constexpr (F16) {
     fa = aug >= 2 || (aug == 1 && f16_fold_ok(amax, c, K));
     if (fa) {
-      const int fsh = aug >= 2 ? f16_fold_shift(amax, c, K) : 0;
+      const int fsh = s_fsh;
       one = __float2half(ldexpf(1.f, fsh));
-      sB = ldexpf(1.f, -f16_fold_exp(c));
+      sB = ldexpf(1.f, -s_fexp);
       far = c * n > ldexp(kFoldFar, fsh);
+      // the folded norm pieces, for the lanes that store columns K + 3 .. K + 5
+      bool mine = false;
+      for (int d = 2 * gl; d < k_pad; d += 2 * G) mine |= (d + 1 >= K + 3 && d < K + 6);
       if (far) mp[0] = __float2half(kFoldNegInf);
-      else split3_f16(ldexp(-c * n, -fsh), mp);
+      else if (mine) split3_f16(ldexp(-c * n, -fsh), mp);
     } else {
       bmax = group_max<G>(bmax);
       const int eA = f16_scale_exp((float)(2.0 * c * (double)__uint_as_float(*amax)));
@@ -1503,6 +1532,9 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
     nb[j] = (fa || (!F16 && aug)) ? 0.f : nbj;
     tsc[j] = rj;
   }
+  // PDL trigger last: a dependent fused kernel's CTA (640 threads, nearly all of an SM's registers)
+  // launched early would hold its SM while waiting and starve this grid's remaining blocks
+  pdl_trigger();
 }
 
 // FP16 V-MMA weights (reading Q27): per-column max |W_ir| (block partials, fixed-order
@@ -1567,13 +1599,172 @@ cudaError_t launch_prep_wcat(const float* W, int64_t M, int64_t m_pad, int R, in
   return cudaGetLastError();
 }
 
+// Folded-layout prep (fold modes 2-4: the R = 1 and multi-column kernels, K + 6 <= k_pad <= 64),
+// one row per 8 lanes, lane g owning the CPL = k_pad / 8 consecutive columns [g CPL, g CPL + CPL):
+// every coordinate is loaded once (coalesced: a warp covers 4 consecutive rows), the hi / lo
+// halves leave as one 4-16-byte store per plane, and the uniform values (fold shift, scale
+// exponent, log2 max W) are evaluated once per block.  Same values as prep_tc_*_kernel<true, G>
+// up to the FP64 summation order of the norms.  (The generic kernels spent ~200 warp
+// instructions per row on per-pair bounds checks, int64 index arithmetic and repeated FP64
+// log2: issue-bound at 20 us for cfg3's 65,536 sources.)
+template <int CPL>
+__device__ __forceinline__ void store_halves(void* base, int64_t off_halves, const __half (&h)[CPL]) {
+  uint32_t w[CPL / 2];
+#pragma unroll
+  for (int k = 0; k < CPL / 2; ++k) {
+    const __half2 v = __halves2half2(h[2 * k], h[2 * k + 1]);
+    w[k] = *reinterpret_cast<const uint32_t*>(&v);
+  }
+  uint32_t* dst = reinterpret_cast<uint32_t*>(static_cast<__half*>(base) + off_halves);
+  if constexpr (CPL == 8) {
+    *reinterpret_cast<uint4*>(dst) = make_uint4(w[0], w[1], w[2], w[3]);
+  } else if constexpr (CPL == 4) {
+    *reinterpret_cast<uint2*>(dst) = make_uint2(w[0], w[1]);
+  } else {
+    dst[0] = w[0];
+  }
+}
+
+template <int CPL>
+__global__ void __launch_bounds__(256) prep_fold_sources_kernel(
+    const float* __restrict__ alpha, const float* __restrict__ W, int64_t M, int64_t m_pad, int K, int R,
+    const float* __restrict__ mu, double c, int aug, const unsigned* __restrict__ amax, void* __restrict__ src_hi,
+    void* __restrict__ src_lo, float* __restrict__ na, float* __restrict__ wv, int rv,
+    const unsigned* __restrict__ wstat) {
+  constexpr int G = 8, KP = 8 * CPL;
+  pdl_wait();  // the source statistics are complete (trigger at the end)
+  __shared__ int s_fsh, s_fexp;
+  __shared__ double s_lwmax;
+  if (threadIdx.x == 0) {
+    s_fsh = f16_fold_shift(amax, c, K);
+    s_fexp = f16_fold_exp(c);
+    s_lwmax = (wstat != nullptr && wstat[0] != 0u) ? log2((double)__uint_as_float(wstat[0])) : 0.0;
+  }
+  __syncthreads();
+  const int lane = threadIdx.x & 31, g = lane & (G - 1);
+  const int64_t i = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
+  if (i >= m_pad) return;
+  const bool live = i < M;
+  const int d0 = g * CPL;
+  float x[CPL];
+  double n = 0.0;
+#pragma unroll
+  for (int k = 0; k < CPL; ++k) {
+    const int d = d0 + k;
+    x[k] = (live && d < K) ? alpha[i * K + d] - mu[d] : 0.f;  // FP32 centring, as the target side
+    n += (double)x[k] * (double)x[k];
+  }
+  n = group_sum<G>(n);
+  const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && aug < 3;
+  const int fsh = s_fsh;
+  const float sA = ldexpf(1.f, s_fexp);
+  const double c2 = 2.0 * c;
+  const __half one = __float2half(ldexpf(1.f, fsh)), zero = __float2half(0.f);
+  __half np[3] = {zero, zero, zero};
+  double wl = 0.0;
+  const bool has_np = d0 + CPL > K && d0 < K + 3;  // this lane stores a folded norm piece
+  if (has_np || (g == 0 && logw && rv > 0)) wl = !logw ? 0.0 : live ? log2((double)W[i]) - s_lwmax : -INFINITY;
+  if (has_np) {
+    const double nf = ldexp(-c * n + wl + (aug == 4 ? 14.0 : 0.0), -fsh);  // W_i = 0: the FP16 stand-in for -inf
+    if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
+    else split3_f16(nf, np);
+  }
+  __half hi[CPL], lo[CPL];
+#pragma unroll
+  for (int k = 0; k < CPL; ++k) {
+    const int d = d0 + k;
+    if (d < K) {
+      split_f16((float)(c2 * (double)x[k]) * sA, hi[k], lo[k]);  // exact power-of-2 scaling
+    } else {
+      hi[k] = d < K + 3 ? np[d - K] : d < K + 6 ? one : zero;  // folded norm columns: hi planes only
+      lo[k] = zero;
+    }
+  }
+  store_halves<CPL>(src_hi, i * KP + d0, hi);
+  store_halves<CPL>(src_lo, i * KP + d0, lo);
+  if (g == 0) na[i] = 0.f;  // folded: the norm and log-weight ride in the contraction
+  for (int r = g; r < rv; r += G) wv[i * rv + r] = logw ? (float)wl : (live && r < R) ? W[i * R + r] : 0.f;
+  // PDL trigger last: a dependent fused kernel's CTA (640 threads, nearly all of an SM's registers)
+  // launched early would hold its SM while waiting and starve this grid's remaining blocks
+  pdl_trigger();
+}
+
+template <int CPL>
+__global__ void __launch_bounds__(256) prep_fold_targets_kernel(const float* __restrict__ beta, int64_t N,
+                                                                int64_t n_pad, int K, const float* __restrict__ mu,
+                                                                double c, const unsigned* __restrict__ amax,
+                                                                void* __restrict__ tgt_hi, void* __restrict__ tgt_lo,
+                                                                float* __restrict__ nb, float* __restrict__ tsc) {
+  constexpr int G = 8, KP = 8 * CPL;
+  pdl_wait();  // the source statistics (mu, amax) are complete (trigger at the end)
+  __shared__ int s_fsh, s_fexp;
+  if (threadIdx.x == 0) {
+    s_fsh = f16_fold_shift(amax, c, K);
+    s_fexp = f16_fold_exp(c);
+  }
+  __syncthreads();
+  const int lane = threadIdx.x & 31, g = lane & (G - 1);
+  const int64_t j = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
+  if (j >= n_pad) return;
+  const bool live = j < N;
+  const int d0 = g * CPL;
+  float x[CPL];
+  double n = 0.0;
+#pragma unroll
+  for (int k = 0; k < CPL; ++k) {
+    const int d = d0 + k;
+    x[k] = (live && d < K) ? beta[j * K + d] - mu[d] : 0.f;
+    n += (double)x[k] * (double)x[k];
+  }
+  n = group_sum<G>(n);
+  const int fsh = s_fsh;
+  const float sB = ldexpf(1.f, -s_fexp);
+  const __half one = __float2half(ldexpf(1.f, fsh)), zero = __float2half(0.f);
+  const bool far = c * n > ldexp(kFoldFar, fsh);  // row beyond every source: kernel row 0
+  __half mp[3] = {zero, zero, zero};
+  if (far) mp[0] = __float2half(kFoldNegInf);
+  else if (d0 + CPL > K + 3 && d0 < K + 6) split3_f16(ldexp(-c * n, -fsh), mp);
+  __half hi[CPL], lo[CPL];
+#pragma unroll
+  for (int k = 0; k < CPL; ++k) {
+    const int d = d0 + k;
+    if (d < K) {
+      split_f16((far ? 0.f : x[k]) * sB, hi[k], lo[k]);
+    } else {
+      hi[k] = d < K + 3 ? one : d < K + 6 ? mp[d - K - 3] : zero;
+      lo[k] = zero;
+    }
+  }
+  store_halves<CPL>(tgt_hi, j * KP + d0, hi);
+  store_halves<CPL>(tgt_lo, j * KP + d0, lo);
+  if (g == 0) {
+    nb[j] = 0.f;
+    tsc[j] = 1.f;
+  }
+  // PDL trigger last: a dependent fused kernel's CTA (640 threads, nearly all of an SM's registers)
+  // launched early would hold its SM while waiting and starve this grid's remaining blocks
+  pdl_trigger();
+}
+
 template <bool F16>
 static cudaError_t launch_prep_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K,
                                        int k_pad, int R, int r_pad, const float* mu, double c, int aug,
                                        const unsigned* amax, void* src_hi, void* src_lo, float* na, float* wt_hi,
                                        float* wt_lo, float* wv, int rv, const unsigned* wstat, cudaStream_t st) {
   if (m_pad == 0) return cudaSuccess;
-  const int bs = 256, G = prep_group(K);
+  const int bs = 256;
+  if (F16 && aug >= 2 && K + 6 <= k_pad && (k_pad == 16 || k_pad == 32 || k_pad == 64) && r_pad == 0 &&
+      opt(KS_OPT_PREP_LANES, 0) == 0) {
+    const unsigned grid = (unsigned)((m_pad * 8 + bs - 1) / bs);
+#define KS_PREP_F(cpl)                                                                                          \
+  return launch_pdl(prep_fold_sources_kernel<cpl>, grid, bs, 0, st, alpha, W, M, m_pad, K, R, mu, c, aug, amax, \
+                    src_hi, src_lo, na, wv, rv, wstat)
+    if (k_pad == 16) KS_PREP_F(2);
+    if (k_pad == 32) KS_PREP_F(4);
+    KS_PREP_F(8);
+#undef KS_PREP_F
+  }
+  const int G = prep_group(K);
   const unsigned grid = (unsigned)((m_pad * G + bs - 1) / bs);
 #define KS_PREP_S(g)                                                                                        \
   return launch_pdl(prep_tc_sources_kernel<F16, g>, grid, bs, 0, st, alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, \
@@ -1593,7 +1784,19 @@ static cudaError_t launch_prep_targets(const float* beta, int64_t N, int64_t n_p
                                        const float* mu, double c, int aug, const unsigned* amax, void* tgt_hi,
                                        void* tgt_lo, float* nb, float* tsc, cudaStream_t st) {
   if (n_pad == 0) return cudaSuccess;
-  const int bs = 256, G = prep_group(K);
+  const int bs = 256;
+  if (F16 && aug >= 2 && K + 6 <= k_pad && (k_pad == 16 || k_pad == 32 || k_pad == 64) &&
+      opt(KS_OPT_PREP_LANES, 0) == 0) {
+    const unsigned grid = (unsigned)((n_pad * 8 + bs - 1) / bs);
+#define KS_PREP_F(cpl)                                                                                             \
+  return launch_pdl(prep_fold_targets_kernel<cpl>, grid, bs, 0, st, beta, N, n_pad, K, mu, c, amax, tgt_hi, tgt_lo, nb, \
+                    tsc)
+    if (k_pad == 16) KS_PREP_F(2);
+    if (k_pad == 32) KS_PREP_F(4);
+    KS_PREP_F(8);
+#undef KS_PREP_F
+  }
+  const int G = prep_group(K);
   const unsigned grid = (unsigned)((n_pad * G + bs - 1) / bs);
 #define KS_PREP_T(g)                                                                                           \
   return launch_pdl(prep_tc_targets_kernel<F16, g>, grid, bs, 0, st, beta, N, n_pad, K, k_pad, mu, c, aug, amax, \
