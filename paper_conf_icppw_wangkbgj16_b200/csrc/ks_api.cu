@@ -22,6 +22,7 @@
 
 #include "../../include/ks.h"
 #include "ks_internal.h"
+#include <nvtx3/nvToolsExt.h>
 
 #ifndef KS_DEBUG
 #define KS_DEBUG 0
@@ -991,7 +992,15 @@ ks_status ks_set_stream(ks_ctx* ctx, void* cuda_stream) {
   return KS_OK;
 }
 
+// NVTX range per ABI call (header-only NVTX 3: a no-op unless a profiler is attached), so an
+// nsys / ncu capture shows ks_set_sources / ks_eval (and the host variants) around their launches
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+
 ks_status ks_set_sources(ks_ctx* ctx, const float* alpha, const float* W, int64_t M, int R) {
+  NvtxRange nvtx("ks_set_sources");
   if (check_ctx(ctx)) return KS_EINVAL;
   OptScope opt_scope(ctx);
   if (M < 0) return fail(KS_EINVAL, "M=%lld < 0", (long long)M);
@@ -1029,6 +1038,7 @@ ks_status ks_set_sources(ks_ctx* ctx, const float* alpha, const float* W, int64_
 }
 
 ks_status ks_eval(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
+  NvtxRange nvtx("ks_eval");
   if (check_ctx(ctx)) return KS_EINVAL;
   OptScope opt_scope(ctx);
   if (N < 0) return fail(KS_EINVAL, "N=%lld < 0", (long long)N);
@@ -1074,6 +1084,7 @@ ks_status host_api_init(ks_ctx* ctx) {
 }  // namespace
 
 ks_status ks_set_sources_host(ks_ctx* ctx, const float* alpha, const float* W, int64_t M, int R) {
+  NvtxRange nvtx("ks_set_sources_host");
   if (check_ctx(ctx)) return KS_EINVAL;
   OptScope opt_scope(ctx);
   if (M < 0) return fail(KS_EINVAL, "M=%lld < 0", (long long)M);
@@ -1100,6 +1111,7 @@ ks_status ks_set_sources_host(ks_ctx* ctx, const float* alpha, const float* W, i
 }
 
 ks_status ks_eval_host(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
+  NvtxRange nvtx("ks_eval_host");
   if (check_ctx(ctx)) return KS_EINVAL;
   OptScope opt_scope(ctx);
   if (N < 0) return fail(KS_EINVAL, "N=%lld < 0", (long long)N);
