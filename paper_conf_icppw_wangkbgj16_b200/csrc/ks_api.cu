@@ -273,13 +273,13 @@ cudaError_t source_stats(ks_ctx* ctx, const float* alpha, const float* W, bool w
                          bool want_amax) {
   cudaStream_t st = ctx->stream;
   const int K = ctx->K;
-  // ~8 K coordinates per block (256 rows at K = 32, 32 rows at K = 256): a few unrolled loads
-  // per thread; at most 1024 blocks when the last block reduces them (K <= 32), 4096 when
-  // K + 1 blocks do (launch_source_stats)
-  const int64_t rows = K >= 8192 ? 1 : 8192 / K;
+  // ~2K coordinates per block (64 rows at K = 32, 8 rows at K = 256): one round of unrolled loads
+  // per thread (the kernel is load-latency bound); beyond 256 blocks the partials are reduced by
+  // K + 1 blocks (launch_source_stats), not the last block alone
+  const int64_t rows = K >= 2048 ? 1 : 2048 / K;
   int64_t np64 = (M + rows - 1) / rows;
   if (np64 < 1) np64 = 1;
-  if (np64 > (K > 32 ? 4096 : 1024)) np64 = K > 32 ? 4096 : 1024;
+  if (np64 > 4096) np64 = 4096;
   const int nparts = (int)np64;
   cudaError_t e;
   if ((e = ctx->mean_part.reserve((size_t)nparts * K, st, false)) != cudaSuccess) return e;
@@ -289,7 +289,7 @@ cudaError_t source_stats(ks_ctx* ctx, const float* alpha, const float* W, bool w
   if ((e = ctx->mu.reserve(k_pad, st, false)) != cudaSuccess) return e;
   if (want_amax && (e = ctx->amax.reserve(1, st, false)) != cudaSuccess) return e;
   if (want_w && (e = ctx->wstat.reserve(2, st, false)) != cudaSuccess) return e;
-  ctx->launches += K > 32 ? 2 : 1;
+  ctx->launches += (K > 32 || nparts > 256) ? 2 : 1;  // launch_source_stats' split
   return ks::launch_source_stats(alpha, W, M, K, k_pad, nparts, ctx->mean_part.p, ctx->mean_pmm.p, ctx->mean_pw.p,
                                  ctx->stats_counter.p, ctx->mu.p, want_amax ? ctx->amax.p : nullptr,
                                  want_w ? ctx->wstat.p : nullptr, st);

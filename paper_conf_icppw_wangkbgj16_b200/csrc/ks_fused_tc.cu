@@ -1600,28 +1600,58 @@ cudaError_t launch_prep_wcat(const float* W, int64_t M, int64_t m_pad, int R, in
 }
 
 // Folded-layout prep (fold modes 2-4: the R = 1 and multi-column kernels, K + 6 <= k_pad <= 64),
-// one row per 8 lanes, lane g owning the CPL = k_pad / 8 consecutive columns [g CPL, g CPL + CPL):
-// every coordinate is loaded once (coalesced: a warp covers 4 consecutive rows), the hi / lo
-// halves leave as one 4-16-byte store per plane, and the uniform values (fold shift, scale
+// one row per 8 lanes.  Lane g owns NCH chunks of V = min(4, k_pad / 8) consecutive columns,
+// chunk c at column V g + 8 V c, so the 8 lanes of a row read one contiguous 8V-float span per
+// chunk (a float4 / float2 each when K is a multiple of V) and write one contiguous span of
+// halves per plane; every coordinate is loaded once; the uniform values (fold shift, scale
 // exponent, log2 max W) are evaluated once per block.  Same values as prep_tc_*_kernel<true, G>
 // up to the FP64 summation order of the norms.  (The generic kernels spent ~200 warp
 // instructions per row on per-pair bounds checks, int64 index arithmetic and repeated FP64
 // log2: issue-bound at 20 us for cfg3's 65,536 sources.)
 template <int CPL>
-__device__ __forceinline__ void store_halves(void* base, int64_t off_halves, const __half (&h)[CPL]) {
-  uint32_t w[CPL / 2];
+struct FoldLanes {
+  static constexpr int V = CPL >= 4 ? 4 : CPL, NCH = CPL / V;
+  __device__ static int col(int g, int c, int k) { return V * g + 8 * V * c + k; }
+};
+
+template <int CPL>
+__device__ __forceinline__ void fold_load_row(const float* __restrict__ row, const float* __restrict__ mu, int K,
+                                              bool live, int g, float (&x)[CPL]) {
+  using L = FoldLanes<CPL>;
 #pragma unroll
-  for (int k = 0; k < CPL / 2; ++k) {
-    const __half2 v = __halves2half2(h[2 * k], h[2 * k + 1]);
-    w[k] = *reinterpret_cast<const uint32_t*>(&v);
+  for (int c = 0; c < L::NCH; ++c) {
+    const int d = L::col(g, c, 0);
+    if (live && d + L::V <= K && (K % L::V) == 0) {
+      if constexpr (L::V == 4) {
+        const float4 v = *reinterpret_cast<const float4*>(row + d);
+        x[4 * c] = v.x, x[4 * c + 1] = v.y, x[4 * c + 2] = v.z, x[4 * c + 3] = v.w;
+      } else {
+        const float2 v = *reinterpret_cast<const float2*>(row + d);
+        x[2 * c] = v.x, x[2 * c + 1] = v.y;
+      }
+#pragma unroll
+      for (int k = 0; k < L::V; ++k) x[L::V * c + k] -= mu[d + k];  // FP32 centring, both sides alike
+    } else {
+#pragma unroll
+      for (int k = 0; k < L::V; ++k) x[L::V * c + k] = (live && d + k < K) ? row[d + k] - mu[d + k] : 0.f;
+    }
   }
-  uint32_t* dst = reinterpret_cast<uint32_t*>(static_cast<__half*>(base) + off_halves);
-  if constexpr (CPL == 8) {
-    *reinterpret_cast<uint4*>(dst) = make_uint4(w[0], w[1], w[2], w[3]);
-  } else if constexpr (CPL == 4) {
-    *reinterpret_cast<uint2*>(dst) = make_uint2(w[0], w[1]);
-  } else {
-    dst[0] = w[0];
+}
+
+template <int CPL>
+__device__ __forceinline__ void fold_store_row(void* base, int64_t row_halves, int g, const __half (&h)[CPL]) {
+  using L = FoldLanes<CPL>;
+#pragma unroll
+  for (int c = 0; c < L::NCH; ++c) {
+    __half* dst = static_cast<__half*>(base) + row_halves + L::col(g, c, 0);
+    const __half2 v0 = __halves2half2(h[L::V * c], h[L::V * c + 1]);
+    if constexpr (L::V == 4) {
+      const __half2 v1 = __halves2half2(h[L::V * c + 2], h[L::V * c + 3]);
+      *reinterpret_cast<uint2*>(dst) =
+          make_uint2(*reinterpret_cast<const uint32_t*>(&v0), *reinterpret_cast<const uint32_t*>(&v1));
+    } else {
+      *reinterpret_cast<uint32_t*>(dst) = *reinterpret_cast<const uint32_t*>(&v0);
+    }
   }
 }
 
@@ -1631,6 +1661,7 @@ __global__ void __launch_bounds__(256) prep_fold_sources_kernel(
     const float* __restrict__ mu, double c, int aug, const unsigned* __restrict__ amax, void* __restrict__ src_hi,
     void* __restrict__ src_lo, float* __restrict__ na, float* __restrict__ wv, int rv,
     const unsigned* __restrict__ wstat) {
+  using L = FoldLanes<CPL>;
   constexpr int G = 8, KP = 8 * CPL;
   pdl_wait();  // the source statistics are complete (trigger at the end)
   __shared__ int s_fsh, s_fexp;
@@ -1645,15 +1676,11 @@ __global__ void __launch_bounds__(256) prep_fold_sources_kernel(
   const int64_t i = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
   if (i >= m_pad) return;
   const bool live = i < M;
-  const int d0 = g * CPL;
   float x[CPL];
+  fold_load_row<CPL>(alpha + i * K, mu, K, live, g, x);
   double n = 0.0;
 #pragma unroll
-  for (int k = 0; k < CPL; ++k) {
-    const int d = d0 + k;
-    x[k] = (live && d < K) ? alpha[i * K + d] - mu[d] : 0.f;  // FP32 centring, as the target side
-    n += (double)x[k] * (double)x[k];
-  }
+  for (int k = 0; k < CPL; ++k) n += (double)x[k] * (double)x[k];
   n = group_sum<G>(n);
   const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && aug < 3;
   const int fsh = s_fsh;
@@ -1661,8 +1688,13 @@ __global__ void __launch_bounds__(256) prep_fold_sources_kernel(
   const double c2 = 2.0 * c;
   const __half one = __float2half(ldexpf(1.f, fsh)), zero = __float2half(0.f);
   __half np[3] = {zero, zero, zero};
+  bool has_np = false;  // this lane stores a folded norm piece (columns K .. K + 2)
+#pragma unroll
+  for (int q = 0; q < CPL; ++q) {
+    const int d = L::col(g, q / L::V, q % L::V);
+    has_np |= d >= K && d < K + 3;
+  }
   double wl = 0.0;
-  const bool has_np = d0 + CPL > K && d0 < K + 3;  // this lane stores a folded norm piece
   if (has_np || (g == 0 && logw && rv > 0)) wl = !logw ? 0.0 : live ? log2((double)W[i]) - s_lwmax : -INFINITY;
   if (has_np) {
     const double nf = ldexp(-c * n + wl + (aug == 4 ? 14.0 : 0.0), -fsh);  // W_i = 0: the FP16 stand-in for -inf
@@ -1671,17 +1703,17 @@ __global__ void __launch_bounds__(256) prep_fold_sources_kernel(
   }
   __half hi[CPL], lo[CPL];
 #pragma unroll
-  for (int k = 0; k < CPL; ++k) {
-    const int d = d0 + k;
+  for (int q = 0; q < CPL; ++q) {
+    const int d = L::col(g, q / L::V, q % L::V);
     if (d < K) {
-      split_f16((float)(c2 * (double)x[k]) * sA, hi[k], lo[k]);  // exact power-of-2 scaling
+      split_f16((float)(c2 * (double)x[q]) * sA, hi[q], lo[q]);  // exact power-of-2 scaling
     } else {
-      hi[k] = d < K + 3 ? np[d - K] : d < K + 6 ? one : zero;  // folded norm columns: hi planes only
-      lo[k] = zero;
+      hi[q] = d < K + 3 ? np[d - K] : d < K + 6 ? one : zero;  // folded norm columns: hi planes only
+      lo[q] = zero;
     }
   }
-  store_halves<CPL>(src_hi, i * KP + d0, hi);
-  store_halves<CPL>(src_lo, i * KP + d0, lo);
+  fold_store_row<CPL>(src_hi, i * KP, g, hi);
+  fold_store_row<CPL>(src_lo, i * KP, g, lo);
   if (g == 0) na[i] = 0.f;  // folded: the norm and log-weight ride in the contraction
   for (int r = g; r < rv; r += G) wv[i * rv + r] = logw ? (float)wl : (live && r < R) ? W[i * R + r] : 0.f;
   // PDL trigger last: a dependent fused kernel's CTA (640 threads, nearly all of an SM's registers)
@@ -1695,6 +1727,7 @@ __global__ void __launch_bounds__(256) prep_fold_targets_kernel(const float* __r
                                                                 double c, const unsigned* __restrict__ amax,
                                                                 void* __restrict__ tgt_hi, void* __restrict__ tgt_lo,
                                                                 float* __restrict__ nb, float* __restrict__ tsc) {
+  using L = FoldLanes<CPL>;
   constexpr int G = 8, KP = 8 * CPL;
   pdl_wait();  // the source statistics (mu, amax) are complete (trigger at the end)
   __shared__ int s_fsh, s_fexp;
@@ -1707,36 +1740,38 @@ __global__ void __launch_bounds__(256) prep_fold_targets_kernel(const float* __r
   const int64_t j = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
   if (j >= n_pad) return;
   const bool live = j < N;
-  const int d0 = g * CPL;
   float x[CPL];
+  fold_load_row<CPL>(beta + j * K, mu, K, live, g, x);
   double n = 0.0;
 #pragma unroll
-  for (int k = 0; k < CPL; ++k) {
-    const int d = d0 + k;
-    x[k] = (live && d < K) ? beta[j * K + d] - mu[d] : 0.f;
-    n += (double)x[k] * (double)x[k];
-  }
+  for (int k = 0; k < CPL; ++k) n += (double)x[k] * (double)x[k];
   n = group_sum<G>(n);
   const int fsh = s_fsh;
   const float sB = ldexpf(1.f, -s_fexp);
   const __half one = __float2half(ldexpf(1.f, fsh)), zero = __float2half(0.f);
   const bool far = c * n > ldexp(kFoldFar, fsh);  // row beyond every source: kernel row 0
+  bool mine = false;  // this lane stores a folded norm piece (columns K + 3 .. K + 5)
+#pragma unroll
+  for (int q = 0; q < CPL; ++q) {
+    const int d = L::col(g, q / L::V, q % L::V);
+    mine |= d >= K + 3 && d < K + 6;
+  }
   __half mp[3] = {zero, zero, zero};
   if (far) mp[0] = __float2half(kFoldNegInf);
-  else if (d0 + CPL > K + 3 && d0 < K + 6) split3_f16(ldexp(-c * n, -fsh), mp);
+  else if (mine) split3_f16(ldexp(-c * n, -fsh), mp);
   __half hi[CPL], lo[CPL];
 #pragma unroll
-  for (int k = 0; k < CPL; ++k) {
-    const int d = d0 + k;
+  for (int q = 0; q < CPL; ++q) {
+    const int d = L::col(g, q / L::V, q % L::V);
     if (d < K) {
-      split_f16((far ? 0.f : x[k]) * sB, hi[k], lo[k]);
+      split_f16((far ? 0.f : x[q]) * sB, hi[q], lo[q]);
     } else {
-      hi[k] = d < K + 3 ? one : d < K + 6 ? mp[d - K - 3] : zero;
-      lo[k] = zero;
+      hi[q] = d < K + 3 ? one : d < K + 6 ? mp[d - K - 3] : zero;
+      lo[q] = zero;
     }
   }
-  store_halves<CPL>(tgt_hi, j * KP + d0, hi);
-  store_halves<CPL>(tgt_lo, j * KP + d0, lo);
+  fold_store_row<CPL>(tgt_hi, j * KP, g, hi);
+  fold_store_row<CPL>(tgt_lo, j * KP, g, lo);
   if (g == 0) {
     nb[j] = 0.f;
     tsc[j] = 1.f;

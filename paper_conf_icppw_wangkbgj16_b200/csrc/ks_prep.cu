@@ -267,7 +267,7 @@ __global__ void __launch_bounds__(256) stats_final_kernel(int64_t M, int K, int 
 cudaError_t launch_source_stats(const float* alpha, const float* W, int64_t M, int K, int k_pad, int nparts,
                                 double* part, float* pmm, unsigned* pw, unsigned* counter, float* mu,
                                 unsigned* amax, unsigned* wstat, cudaStream_t st) {
-  const bool split = K > 32;  // wide points: reduce the partials with K + 1 blocks
+  const bool split = K > 32 || nparts > 256;  // reduce the partials with K + 1 blocks (a parallel tree per dim)
   source_stats_kernel<<<nparts, 256, 0, st>>>(alpha, W, M, K, k_pad, nparts, part, pmm, pw, split ? nullptr : counter,
                                               mu, amax, wstat);
   if (split) stats_final_kernel<<<K + 1, 256, 0, st>>>(M, K, k_pad, nparts, part, pmm, pw, mu, amax, wstat);
