@@ -19,12 +19,15 @@
 //   warp 2    TMEM allocation; the V-MMA issuer (unit order: one issuer, so the TMEM
 //             accumulation order is fixed -> bitwise deterministic);
 //   warp 20   TMA producer of each unit's weight tile ([W_hi | W_lo] rows, 96 sources);
-//   warps 4..19  2 epilogue groups of 8 warps (group q % 2 computes unit q's P and writes it back
-//             in place, then releases it to the V issuer; with 4 S buffers a group alternates
-//             between two, so its next unit's S is computed while it works); every epilogue warp
-//             also folds RC / 4 columns of each V block (<= kRvBlock units of a target tile) from
-//             TMEM into compensated FP32 shared-memory row sums and, at a target tile's end,
-//             writes them to V or a stream-K partial.
+//   warps 4..19  4 epilogue groups of 4 warps, one per TMEM lane quarter (group q % 4 computes
+//             unit q's P in S buffer q % 4 and writes it back in place, then releases it to the
+//             V issuer; the V issuer releases the buffer to the next S MMA as soon as it has
+//             *issued* the unit's V MMAs -- tcgen05.mma ops execute in issue order); every
+//             epilogue warp also folds RC / 4 columns of each V block (<= kRvBlock units of a
+//             target tile) from TMEM into compensated FP32 shared-memory row sums and, at a
+//             target tile's end, writes them to V or a stream-K partial.  (Two groups of 8
+//             warps, each alternating between two buffers, measured 2% slower: a group's next S
+//             waited on the other buffer's V.)
 // Units are 128 targets x 96 sources.  TMEM: 4 S buffers x 96 columns | 2 V blocks x 2 RC columns
 // (RC = 16: [V_hh+lh | V_hl]; RC = 32: the two 16-column groups side by side).
 #include "ks_internal.h"
@@ -74,7 +77,9 @@ constexpr int kRvSBufs = 4;          // S buffers (TMEM columns 0..383)
 constexpr int kRvTS = kRvTileS;            // sources per unit (4 x 96 S columns + 2 V blocks fit 512)
 constexpr uint32_t kRvPlane = 128u * 64u;   // target plane (128 rows x 64 B); source planes 96 rows
 constexpr int kRvMaxStages = 8;
-constexpr int kRvBlock = 4;          // units per V block (FP32 TMEM accumulation <= 32 K steps)
+constexpr int kRvBlock = 8;          // units per V block (FP32 TMEM accumulation over <= 768 sources;
+                                     // 4 measured 2% slower: the V issuer waits for all 16 warps'
+                                     // fold of the block two back)
 constexpr uint32_t kRvSmem = 227u * 1024u;
 constexpr uint32_t kRvBars = 1024u;
 constexpr uint32_t kRvColV = kRvSBufs * kRvTS;  // 384
@@ -248,7 +253,7 @@ __global__ void __launch_bounds__(kRvThreads, 1)
     for (int i = 0; i < kRvSBufs; ++i) {
       mbar_init(&sfull[i], 1);
       mbar_init(&sempty[i], 1);
-      mbar_init(&pready[i], 8);  // the unit's group (8 warps)
+      mbar_init(&pready[i], 4);  // the unit's group (4 warps)
     }
     for (int i = 0; i < kRvWSlots; ++i) {
       mbar_init(&wfull[i], 1);
@@ -437,7 +442,13 @@ __global__ void __launch_bounds__(kRvThreads, 1)
           for (int g = 0; g < RC / 16; ++g)
             mma_f16_ts_lo(dV + 32u * g, aHi + 8u, bd + (uint32_t)((g * 32 * 64) >> 4), whi, idV1, 1u, lead);
         }
-        tc_commit_if(&sempty[bq], lead);
+        // the S buffer may take unit q + 4's S MMAs as soon as this unit's V MMAs are *issued*:
+        // tcgen05.mma ops execute in issue order, so the V MMAs read P before the next S MMA
+        // overwrites it (a commit here would add the V execution and the commit round trip to
+        // every group's wait for its next unit)
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&sempty[bq]);
         tc_commit_if(&wempty[slot], lead);
         if (lane == 0) RV_TRACE(q, 3);
         if (last) {
@@ -452,13 +463,13 @@ __global__ void __launch_bounds__(kRvThreads, 1)
       q0 += len;
     }
   } else if (warp >= 4 && warp < 20) {
-    // ================= epilogue: group gr (8 warps) computes P of units q % 2 == gr, warp (g, hc)
-    // lane quarter g, columns 48 hc .. 48 hc + 47; every warp also folds RC / 4 weight columns of V
-    // (the fold's work and latency split over both groups, so neither stalls its P pipeline long)
+    // ================= epilogue: group gr (4 warps, one per TMEM lane quarter g) computes P of the
+    // units q % 4 == gr in S buffer gr; every warp also folds RC / 4 weight columns of V (the
+    // fold's work and latency split over all 16 warps)
     const int ew = warp - 4;
-    const int g = ew & 3, hc = (ew >> 2) & 1, gr = ew >> 3;
+    const int g = ew & 3, gr = ew >> 2;      // TMEM lane quarter, group (= S buffer, units q % 4 == gr)
     constexpr int kNC = RC / 4;              // weight columns this warp folds
-    const int rlo = (2 * gr + hc) * kNC;     // first of them
+    const int rlo = gr * kNC;                // first of them
     const int rhi = rlo + kNC;
     const int row = 32 * g + lane;
     const uint32_t lane_off = (uint32_t)(32 * g) << 16;
@@ -517,28 +528,34 @@ __global__ void __launch_bounds__(kRvThreads, 1)
       sc.segment(q0, tt, st0, len);
       const int seg_blocks = (len + kRvBlock - 1) / kRvBlock;
       for (int j = 0; j < len; ++j, ++q) {
-        if ((q & 1) == gr) {
+        if ((q & 3) == gr) {
           RV_WAIT(&sfull[bq], (uint32_t)(u3 & 1), "sfull", q);
-          if (lane == 0 && ew == 8 * gr) RV_TRACE(q, 1);
+          if (lane == 0 && ew == 4 * gr) RV_TRACE(q, 1);
           tc_fence_after();
-          // this warp's 48 columns: 3 K steps of 16 sources, as a 32-column and a 16-column batch
-          const uint32_t ta = tbase + lane_off + (uint32_t)(bq * kRvTS + 48 * hc);
-          uint32_t sa[32], sb[16];
+          // all 96 columns of the unit for this lane quarter: 6 K steps of 16 sources in three
+          // 32-column batches, the next batch's load in flight while one is computed
+          const uint32_t ta = tbase + lane_off + (uint32_t)(bq * kRvTS);
+          uint32_t sa[32], sb[32];
           if (!(KS_DEBUG && (args.dbg & 4))) {
           tmem_ld32(ta, sa);
           tmem_wait_ld();
-          tmem_ld16(ta + 32, sb);
+          tmem_ld32(ta + 32, sb);
           rv_batch<NPOLY, 32>(sa);
-          if (!(KS_DEBUG && (args.dbg & (8 | 64)))) tmem_st32(ta, sa);
+          if (!(KS_DEBUG && (args.dbg & 8))) tmem_st32(ta, sa);
           tmem_wait_ld();
-          rv_batch<NPOLY, 16>(sb);
-          if (!(KS_DEBUG && (args.dbg & (8 | 32)))) tmem_st16(ta + 32, sb);
+          tmem_wait_st();  // sa is reloaded next
+          tmem_ld32(ta + 64, sa);
+          rv_batch<NPOLY, 32>(sb);
+          if (!(KS_DEBUG && (args.dbg & 8))) tmem_st32(ta + 32, sb);
+          tmem_wait_ld();
+          rv_batch<NPOLY, 32>(sa);
+          if (!(KS_DEBUG && (args.dbg & (8 | 32)))) tmem_st32(ta + 64, sa);  // 32: a third of P never stored
           if (!(KS_DEBUG && (args.dbg & 16))) tmem_wait_st();
           }
           tc_fence_before();
           __syncwarp();
           if (lane == 0) mbar_arrive(&pready[bq]);
-          if (lane == 0 && ew == 8 * gr) RV_TRACE(q, 2);
+          if (lane == 0 && ew == 4 * gr) RV_TRACE(q, 2);
           // fold the completed V blocks of this tile (the V issuer reuses a block's columns two
           // blocks later); one not yet complete is tried again after the next unit rather than
           // stalling the P pipeline
@@ -547,9 +564,9 @@ __global__ void __launch_bounds__(kRvThreads, 1)
               const int jl = (blk_next - blk_total) * kRvBlock;  // first unit of the block
               if (jl > j) break;
               if (!__all_sync(0xffffffffu, mbar_test(&vfull[blk_next & 1], (uint32_t)((blk_next >> 1) & 1)))) break;
-              if (lane == 0 && ew == 8 * gr) RV_TRACE(q, 8);
+              if (lane == 0 && ew == 4 * gr) RV_TRACE(q, 8);
               fold(blk_next++);
-              if (lane == 0 && ew == 8 * gr) RV_TRACE(q, 9);
+              if (lane == 0 && ew == 4 * gr) RV_TRACE(q, 9);
             }
           }
         }
@@ -576,7 +593,7 @@ __global__ void __launch_bounds__(kRvThreads, 1)
           named_bar_sync(2, 32 * kRvEpiWarps);
           const int64_t b_first = rv_sk_owner(tr * n_s, sc.Urem, sc.Gr);
           const int64_t b_last = rv_sk_owner(tr * n_s + n_s - 1, sc.Urem, sc.Gr);
-          if (row == 0 && hc == 0 && gr == 0) {
+          if (row == 0 && gr == 0) {
             const int old = atomicAdd(&args.counters[tt], 1);
             const int lastc = (old == (int)(b_last - b_first));
             if (lastc) args.counters[tt] = 0;
