@@ -525,7 +525,7 @@ def run_ours(args):
                       "k_pad": info1["k_pad"], "ctas": info1["num_ctas"],
                       "stages": info1["stages"],
                       "kernel": {1: "ks_fused_fp32_kernel", 2: "ks_fused_tc_kernel",
-                                 3: "ks_fused_r1_kernel"}.get(info1["kernel"], "?"),
+                                 3: "ks_fused_r1_kernel", 4: "ks_fused_rv_kernel"}.get(info1["kernel"], "?"),
                       # north_star's d^2 >= 0 clamp: the FP32 kernel and the R > 1 / weight-mode
                       # epilogues clamp; the default R = 1 log-weight epilogue does not (DESIGN.md
                       # Q8: overshoot bounded by the Eq.3 rounding, tests/test_gpu_r1.py)
