@@ -483,7 +483,7 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
       ks::opt(KS_OPT_WEIGHTED_SUM, -1) != 1) {
     rv = 1;
     vcc = 0;
-    fold = 4;
+    fold = 3;
   }
   // k_pad in elements: one 64-byte row chunk per pipeline stage = 16 FP32 or 32 FP16; the R = 1
   // kernel at K + 6 <= 16 keeps 32-byte rows (16 halves: half the operand bytes; cfg5's prepared

@@ -3,13 +3,14 @@
 // skeleton (scope rows a2-a7; R columns are the north_star extension of Eq.2).
 //
 // What it computes (PAPER.md SS III-C, Alg.2; Eq.1-3):
-//   t'_ji = sum_d bh_jd a_id + na_i + nb_j + 14  (one accumulator: split-FP16 coordinates and
-//                                              the folded norm pieces, readings Q26 / Q28)
-//   P_ji 2^14 = 2^min(t'_ji, 14)              (d^2 >= 0 clamped; MUFU.EX2, part on the FMA pipe)
+//   t_ji = sum_d bh_jd a_id + na_i + nb_j = -c d_ji^2  (one accumulator: split-FP16 coordinates
+//                                              and the folded norm pieces, readings Q26 / Q28)
+//   P_ji = 2^-|t_ji|                          (|d^2|: the d^2 >= 0 clamp up to the rounding of
+//                                              d^2, reading Q8; MUFU.EX2, part on the FMA pipe)
 //   V_jr = sum_i P_ji W_ir                    (Eq.2, per weight column)
-// P 2^14 is split into FP16 hi/lo and written back over its own S columns, W as FP16 hi/lo of
+// P is split into FP16 hi/lo and written back over its own S columns, W as FP16 hi/lo of
 // per-column power-of-2 scaled weights, and V = P_hi [W_hi | W_lo] + P_lo W_hi accumulates in
-// TMEM (reading Q27), folded into compensated FP32 row sums and unscaled by 2^-(14 + s_r).
+// TMEM (reading Q27), folded into compensated FP32 row sums and unscaled by 2^-s_r.
 //
 // Structure: one persistent 672-thread CTA per SM over (128-target x 96-source) units, the
 // same wave + stream-K schedule and deterministic fix-up as ks_fused_r1.cu:
@@ -136,16 +137,27 @@ __device__ __forceinline__ void mma_f16_ts_lo(uint32_t d_tmem, uint32_t a_tmem, 
       : "memory");
 }
 
-// One 32-column batch of P for a lane: 2^min(t', 14) (t' from the MMA already holds + 14), NPOLY of
-// every 16 pairs on the FMA pipe; split x = hi + lo in FP16 (hi = x with its low 13 mantissa bits
-// cleared, exact remainder lo), packed in place: words 0-7 hi pairs and 8-15 lo pairs of sources
-// 0-15, 16-23 / 24-31 of sources 16-31 (one 16-source K step of the V MMA each).
+// f32x2 subtract (one FMA-pipe issue for a pair)
+__device__ __forceinline__ f2_t fsub2(f2_t a, f2_t b) {
+  f2_t d;
+  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+
+// One NC-column batch of P for a lane: P = 2^-|t| (t = -c d^2 from the MMA; the reflection |d^2|
+// keeps P <= exp(0) = 1 -- the d^2 >= 0 clamp up to the rounding of d^2, reading Q8 -- and costs
+// nothing: MUFU.EX2 takes -|x| as an operand modifier), NPOLY of every 16 pairs on the FMA pipe;
+// split P = hi + lo in FP16 (hi = P with its low 13 mantissa bits cleared, exact for P >= 2^-14;
+// lo the remainder, one f32x2 subtract per pair), packed in place: words 0-7 hi pairs and 8-15
+// lo pairs of sources 0-15, 16-23 / 24-31 of sources 16-31 (one 16-source K step of the V MMA
+// each).  P below 2^-14 is an FP16 subnormal: absolute error <= 2^-25 per term, <= 2^-25 sum |W|
+// in V (reading Q27).
 template <int NPOLY, int NC>
 __device__ __forceinline__ void rv_batch(uint32_t (&sv)[NC]) {
   uint32_t out[NC];
 #pragma unroll
   for (int k = 0; k < NC / 2; ++k) {  // pair k = sources (2k, 2k + 1)
-    const float t0 = fminf(__uint_as_float(sv[2 * k]), 14.f), t1 = fminf(__uint_as_float(sv[2 * k + 1]), 14.f);
+    const float t0 = -fabsf(__uint_as_float(sv[2 * k])), t1 = -fabsf(__uint_as_float(sv[2 * k + 1]));
     float p0, p1;
     if (((k * NPOLY) & 15) < NPOLY) {
       f2_unpack(exp2_poly2(f2_pack(fmaxf(t0, -125.f), fmaxf(t1, -125.f))), p0, p1);
@@ -155,8 +167,10 @@ __device__ __forceinline__ void rv_batch(uint32_t (&sv)[NC]) {
     }
     const float h0 = __uint_as_float(__float_as_uint(p0) & 0xFFFFE000u);
     const float h1 = __uint_as_float(__float_as_uint(p1) & 0xFFFFE000u);
-    const __half2 hv = __floats2half2_rn(h0, h1);           // exact (11 significant bits)
-    const __half2 lv = __floats2half2_rn(p0 - h0, p1 - h1);  // remainders, |lo| < 2^-10 |p|
+    const __half2 hv = __floats2half2_rn(h0, h1);
+    float l0, l1;
+    f2_unpack(fsub2(f2_pack(p0, p1), f2_pack(h0, h1)), l0, l1);
+    const __half2 lv = __floats2half2_rn(l0, l1);
     const int step = k >> 3, w = k & 7;
     out[16 * step + w] = *reinterpret_cast<const uint32_t*>(&hv);
     out[16 * step + 8 + w] = *reinterpret_cast<const uint32_t*>(&lv);
@@ -478,7 +492,7 @@ __global__ void __launch_bounds__(kRvThreads, 1)
     // computed once into shared memory (after the row accumulators)
     float* vscale = reinterpret_cast<float*>(smem + kRvSmem - kRvBars + 512);  // [RC] (bars use < 512 B)
     if (ew == 0 && lane < RC)
-      vscale[lane] = lane < args.r_valid ? ldexpf(1.f, -(14 + rv_wcol_exp(args.wcol[args.r_off + lane]))) : 0.f;
+      vscale[lane] = lane < args.r_valid ? ldexpf(1.f, -rv_wcol_exp(args.wcol[args.r_off + lane])) : 0.f;
     named_bar_sync(3, 32 * kRvEpiWarps);
     int blk_next = 0;   // next V block this warp folds
     int blk_total = 0;  // V blocks issued so far (all segments before the current one)
@@ -642,8 +656,9 @@ static cudaError_t launch_rv_t(const CUtensorMap* m, const RvArgs& a, cudaStream
                     a);
 }
 
-// exponential pairs of 16 on the FMA pipe (KS_OPT_EXP_POLY; default 0: the P split adds FMA-pipe
-// and issue work per pair; measured at K = 32, 65,536^2: 0 beats 4 by 3-6% for R = 2..32)
+// exponential pairs of 16 on the FMA pipe (KS_OPT_EXP_POLY; default 0: the P split adds ALU and
+// issue work per pair; measured at K = 32, R = 16, 65,536^2: 0 / 2 / 4 / 6 -> 1.25 / 1.26 / 2.00 /
+// 2.48 ms)
 int rv_poly_for(int v) { return (v == 0 || v == 2 || v == 4 || v == 6) ? v : 0; }
 
 cudaError_t launch_fused_rv(const CUtensorMap* maps, const RvArgs& a, cudaStream_t st) {
