@@ -162,8 +162,14 @@ def energy_per_step(step, dev_index: int, seconds: float, sync):
         dt = time.perf_counter() - t0
         e1 = pynvml.nvmlDeviceGetTotalEnergyConsumption(hdl)
         j = (e1 - e0) / 1e3
-        return {"j_per_step": j / n, "avg_power_w": j / dt, "steps": n, "seconds": dt,
-                "source": "nvmlDeviceGetTotalEnergyConsumption (board, mJ), whole steps incl. L2 flush-free loop"}
+        out = {"j_per_step": j / n, "avg_power_w": j / dt, "steps": n, "seconds": dt,
+               "source": "nvmlDeviceGetTotalEnergyConsumption (board, mJ), whole steps incl. L2 flush-free loop"}
+        try:  # the board cap the steps ran against (SS6: the headline is power-bound)
+            out["power_limit_w"] = pynvml.nvmlDeviceGetEnforcedPowerLimit(hdl) / 1e3
+            out["power_frac_of_limit"] = out["avg_power_w"] / out["power_limit_w"]
+        except Exception:
+            pass
+        return out
     except Exception as e:  # pragma: no cover - no NVML
         return {"unavailable": str(e)}
 
