@@ -476,9 +476,9 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
     fold = r1;
   }
   // R > 1, split-FP16, K + 6 <= 64: the multi-column kernel (ks_fused_rv.cu) on the same skeleton,
-  // weighted sum as a second tcgen05 MMA (fold mode 4: norms + the 2^14 P scale in the
-  // contraction; the FP16 weight split of reading Q27).  KS_OPT_R1_KERNEL = 0 selects the general
-  // kernel for both.
+  // weighted sum as a second tcgen05 MMA (fold mode 3: the norms in the contraction with the fold
+  // shift, no log-weights; the FP16 weight split of reading Q27).  KS_OPT_R1_KERNEL = 0 selects
+  // the general kernel for both.
   if (f16 && R > 1 && K + 6 <= 2 * 2 * ks::kTcKC && ks::opt(KS_OPT_R1_KERNEL, 1) != 0 &&
       ks::opt(KS_OPT_WEIGHTED_SUM, -1) != 1) {
     rv = 1;

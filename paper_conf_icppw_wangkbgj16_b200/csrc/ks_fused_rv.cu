@@ -488,7 +488,7 @@ __global__ void __launch_bounds__(kRvThreads, 1)
     const int row = 32 * g + lane;
     const uint32_t lane_off = (uint32_t)(32 * g) << 16;
     for (int r = rlo; r < rhi; ++r) vacc[r * 128 + row] = vcmp[r * 128 + row] = 0.f;
-    // per-column unscale 2^-(14 + s_r) (exact), s_r from the column's max |W| (reading Q27);
+    // per-column unscale 2^-s_r (exact), s_r from the column's max |W| (reading Q27);
     // computed once into shared memory (after the row accumulators)
     float* vscale = reinterpret_cast<float*>(smem + kRvSmem - kRvBars + 512);  // [RC] (bars use < 512 B)
     if (ew == 0 && lane < RC)

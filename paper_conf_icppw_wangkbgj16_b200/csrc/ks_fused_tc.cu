@@ -1357,10 +1357,8 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
   const float nai = live ? (float)(-c * n) : 0.f;
   const double c2 = 2.0 * c;
   // aug (FP16): 1 folded layout when f16_fold_ok, 2 always folded (fold shift), 3 the same
-  // without log-weights (the R = 1 kernel's weight mode), 4 the same plus the exponent offset
-  // kPExp (the multi-column kernel's P 2^kPExp, reading Q27: the MMA delivers t + 14)
+  // without log-weights (the R = 1 kernel's weight mode and the multi-column kernel)
   const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && !(F16 && aug >= 3);
-  const double eoff = (F16 && aug == 4) ? 14.0 : 0.0;
   // log2(W_i / Wmax) (R = 1, W >= 0; -inf for W_i = 0 and padding); FP64 log2, so only the
   // lanes that store it evaluate it
   auto wl_of = [&]() -> double { return !logw ? 0.0 : live ? log2((double)W[i]) - s_lwmax : -INFINITY; };
@@ -1384,7 +1382,7 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
   auto need_np = [&]() {
     if (np_ready) return;
     np_ready = true;
-    const double nf = ldexp(-c * n + wl_of() + eoff, -fsh);  // finite unless W_i = 0: then the FP16 stand-in for -inf
+    const double nf = ldexp(-c * n + wl_of(), -fsh);  // finite unless W_i = 0: then the FP16 stand-in for -inf
     if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
     else split3_f16(nf, np);
   };
@@ -1599,7 +1597,7 @@ cudaError_t launch_prep_wcat(const float* W, int64_t M, int64_t m_pad, int R, in
   return cudaGetLastError();
 }
 
-// Folded-layout prep (fold modes 2-4: the R = 1 and multi-column kernels, K + 6 <= k_pad <= 64),
+// Folded-layout prep (fold modes 2, 3: the R = 1 and multi-column kernels, K + 6 <= k_pad <= 64),
 // one row per 8 lanes.  Lane g owns NCH chunks of V = min(4, k_pad / 8) consecutive columns,
 // chunk c at column V g + 8 V c, so the 8 lanes of a row read one contiguous 8V-float span per
 // chunk (a float4 / float2 each when K is a multiple of V) and write one contiguous span of
@@ -1697,7 +1695,7 @@ __global__ void __launch_bounds__(256) prep_fold_sources_kernel(
   double wl = 0.0;
   if (has_np || (g == 0 && logw && rv > 0)) wl = !logw ? 0.0 : live ? log2((double)W[i]) - s_lwmax : -INFINITY;
   if (has_np) {
-    const double nf = ldexp(-c * n + wl + (aug == 4 ? 14.0 : 0.0), -fsh);  // W_i = 0: the FP16 stand-in for -inf
+    const double nf = ldexp(-c * n + wl, -fsh);  // W_i = 0: the FP16 stand-in for -inf
     if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
     else split3_f16(nf, np);
   }
