@@ -178,7 +178,10 @@ typedef enum {
   KS_OPT_FP32_SPLIT = 15,     /* KS_FP32_SPLIT: FP32 kernel tile body: -1 auto, 0, 1 [eval] */
   KS_OPT_MEASURE_CLOCK = 16,  /* 1: the R = 1 kernel records globaltimer and clock64 at every CTA's
                                  start and end, for ks_clock_read (measurement, 0 default) [eval] */
-  KS_OPT_COUNT_ = 17
+  KS_OPT_EVAL_CHUNK0 = 17,    /* KS_EVAL_CHUNK0: ks_eval_host first chunk in 128-target tiles: 0
+                                 auto (one wave of tiles when N >= 2 waves), -1 equal chunks,
+                                 t > 0 that many tiles [eval] */
+  KS_OPT_COUNT_ = 18
 } ks_option;
 
 /* Set / read a tuning option.  KS_EINVAL for an unknown option or a value out of its range. */

@@ -215,6 +215,7 @@ const OptSpec kOpt[KS_OPT_COUNT_] = {
     {"KS_EVAL_CHUNKS", 0, 0, 4},
     {"KS_FP32_SPLIT", -1, -1, 1},
     {"KS_MEASURE_CLOCK", 0, 0, 1},
+    {"KS_EVAL_CHUNK0", 0, -1, 1 << 20},
 };
 
 void init_opts(ks_ctx* ctx) {
@@ -1127,21 +1128,39 @@ ks_status ks_eval_host(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   KS_CUDA(ctx->h_V.reserve(nv, ctx->stream, false), "allocate V staging");
   // The uploads run on the copy stream (overlapping a source prep still in flight on `stream`;
   // the staging buffer's previous readers finished before the previous ks_eval_host returned).
-  // Large N: up to 4 chunks of >= half a wave of 128-target tiles each; chunk c is evaluated
-  // while chunk c + 1 uploads and its V downloads while chunk c + 1 evaluates (KS_OPT_EVAL_CHUNKS
-  // = n forces n; measured at cfg3, same box: 1 / 2 / 3 / 4 chunks 1.455 / 1.383 / 1.386 / 1.363 ms
-  // per host-API step).
-  const int och = ctx->opts.v[KS_OPT_EVAL_CHUNKS];
-  const int64_t half_wave = (int64_t)ctx->num_sms * 64;
-  int nch = (int)(N / half_wave);
-  if (och >= 1 && och <= 4) nch = och;
+  // Chunks: chunk c is evaluated while chunk c + 1 uploads and its V downloads while chunk c + 1
+  // evaluates.  Default (KS_OPT_EVAL_CHUNK0 = 0) for N >= 2 waves of 128-target tiles: the
+  // first chunk is exactly one wave (every CTA one whole target tile, no stream-K split) so the
+  // first launch starts as soon as 148 tiles have arrived, and the rest is one launch (its upload
+  // hides under the first one; measured at cfg3, SS7).  Smaller N, or
+  // KS_OPT_EVAL_CHUNK0 = -1: up to 4 equal chunks of >= half a wave each.  KS_OPT_EVAL_CHUNK0 = t
+  // > 0 makes the first chunk t tiles; KS_OPT_EVAL_CHUNKS = n forces n chunks in total.
+  const int och = ctx->opts.v[KS_OPT_EVAL_CHUNKS], oc0 = ctx->opts.v[KS_OPT_EVAL_CHUNK0];
+  const int64_t wave = (int64_t)ctx->num_sms * 128, half_wave = wave / 2;
+  int64_t first = 0;  // targets in chunk 0 when it differs from the others
+  if (oc0 > 0) first = (int64_t)oc0 * 128;
+  else if (oc0 == 0 && N >= 2 * wave) first = wave;
+  if (first >= N) first = 0;
+  int nch;
+  if (first > 0) nch = (och >= 2 && och <= 4) ? och : 2;
+  else {
+    nch = (int)(N / half_wave);
+    if (och >= 1 && och <= 4) nch = och;
+  }
   if (nch > 4) nch = 4;
   if (nch < 1) nch = 1;
   int64_t off[4] = {0, 0, 0, 0}, cnt[4] = {0, 0, 0, 0};
   {
-    const int64_t per = round_up((N + nch - 1) / nch, 128);
     int64_t o = 0;
-    for (int c = 0; c < nch; ++c) {
+    int c0 = 0;
+    if (first > 0) {
+      cnt[0] = first;
+      o = first;
+      c0 = 1;
+    }
+    const int rest = nch - c0;
+    const int64_t per = round_up((N - o + rest - 1) / rest, 128);
+    for (int c = c0; c < nch; ++c) {
       off[c] = o;
       cnt[c] = (N - o < per) ? N - o : per;
       o += cnt[c];

@@ -33,13 +33,15 @@ def precision(request):
     yield request.param
 
 
-def gpu_eval(alpha, W, beta, h, precision=None, host=False):
+def gpu_eval(alpha, W, beta, h, precision=None, host=False, options=None):
     precision = precision or _PREC["p"]
     K = alpha.shape[1]
     W = np.asarray(W, np.float32)
     if W.ndim == 1:
         W = W[:, None]
     with ks.KernelSum(K, float(h), precision) as plan:
+        for k, v in (options or {}).items():
+            plan.set_option(k, v)
         if host:
             plan.set_sources_host(alpha, W)
             return plan.eval_host(beta).astype(np.float64)
@@ -207,6 +209,22 @@ def test_host_api_chunked_eval(oracle_mod, N):
     Vh = gpu_eval(a, W, b, h, host=True)
     assert np.max(np.abs(Vh - Vd)) <= 1e-6 * np.abs(W).sum()
     J = workloads.sample_targets(N, 300, seed=5)
+    check(oracle_mod, a, W, b, h, J=J, V=Vh)
+
+
+@pytest.mark.parametrize("chunks,chunk0", [(1, 0), (0, -1), (3, 5), (4, 0), (2, 300), (0, 1000)])
+def test_host_api_chunk_schedules(oracle_mod, chunks, chunk0):
+    """Every ks_eval_host chunk schedule (one launch; equal chunks; a first chunk of t tiles,
+    default one wave of tiles, and the rest in n - 1 chunks; a first chunk past N) gives the
+    one-piece device result to rounding and meets the bar.  N = 40,077: > 2 waves of tiles
+    on 148 SMs, a ragged last tile."""
+    if _PREC["p"] != "3xf16":
+        pytest.skip("chunking is independent of the precision")
+    a, W, b, h = workloads.make(3, M=2000, N=40077, wkind="pos")
+    Vd = gpu_eval(a, W, b, h)
+    Vh = gpu_eval(a, W, b, h, host=True, options={"eval_chunks": chunks, "eval_chunk0": chunk0})
+    assert np.max(np.abs(Vh - Vd)) <= 1e-6 * np.abs(W).sum()
+    J = workloads.sample_targets(40077, 200, seed=6)
     check(oracle_mod, a, W, b, h, J=J, V=Vh)
 
 
