@@ -181,7 +181,10 @@ typedef enum {
   KS_OPT_EVAL_CHUNK0 = 17,    /* KS_EVAL_CHUNK0: ks_eval_host first chunk in 128-target tiles: 0
                                  auto (one wave of tiles when N >= 2 waves), -1 equal chunks,
                                  t > 0 that many tiles [eval] */
-  KS_OPT_COUNT_ = 18
+  KS_OPT_COOP_PREP = 18,      /* KS_COOP_PREP: folded layouts (R = 1 and multi-column kernels):
+                                 1 (default) source statistics and prep in one cooperative
+                                 launch, 0 the separate kernels [sources] */
+  KS_OPT_COUNT_ = 19
 } ks_option;
 
 /* Set / read a tuning option.  KS_EINVAL for an unknown option or a value out of its range. */

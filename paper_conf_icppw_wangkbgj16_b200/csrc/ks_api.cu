@@ -151,6 +151,7 @@ struct ks_ctx {
   DBuf<float> mean_pmm;   // [nparts][K][2] column min/max
   DBuf<unsigned> mean_pw; // [nparts][2] weight statistics
   DBuf<unsigned> stats_counter;  // arrival counter of the statistics kernels (left zero)
+  DBuf<unsigned> coop_bar;       // grid barrier of the cooperative source prep {arrivals, departures}
   DBuf<unsigned> wcol, wcol_part; // FP16 V-MMA: per-column max |W| bits [r_pad], block partials
   CUtensorMap tmap_src;
 
@@ -216,6 +217,7 @@ const OptSpec kOpt[KS_OPT_COUNT_] = {
     {"KS_FP32_SPLIT", -1, -1, 1},
     {"KS_MEASURE_CLOCK", 0, 0, 1},
     {"KS_EVAL_CHUNK0", 0, -1, 1 << 20},
+    {"KS_COOP_PREP", 1, 0, 1},
 };
 
 void init_opts(ks_ctx* ctx) {
@@ -508,13 +510,35 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   KS_CUDA(ctx->mu.reserve(k_pad, st, false), "allocate mean buffer");
   // mean, max |alpha - mu| (FP16 scaling) and the R = 1 weight statistics in one launch
   const bool want_wstat = use_wstat || r1;  // the R = 1 kernel decides its epilogue from wstat
-  KS_CUDA(source_stats(ctx, alpha, W, want_wstat, M, k_pad, f16), "source statistics");
+  // folded layouts (the R = 1 and multi-column kernels): statistics and source prep in one
+  // cooperative launch (KS_OPT_COOP_PREP = 0: the separate statistics and prep kernels)
+  const bool coop = f16 && fold >= 2 && K + 6 <= k_pad && (k_pad == 16 || k_pad == 32 || k_pad == 64) &&
+                    ks::opt(KS_OPT_PREP_LANES, 0) == 0 && ks::opt(KS_OPT_COOP_PREP, 1) != 0;
+  if (coop) {
+    const int grid = ks::coop_prep_grid(k_pad, m_pad, ctx->num_sms);
+    KS_CUDA(ctx->mean_part.reserve((size_t)grid * K, st, false), "allocate statistics partials");
+    KS_CUDA(ctx->mean_pmm.reserve((size_t)grid * K * 2, st, false), "allocate statistics partials");
+    KS_CUDA(ctx->mean_pw.reserve((size_t)grid * 2, st, false), "allocate statistics partials");
+    KS_CUDA(ctx->coop_bar.reserve(2, st, true), "allocate grid barrier");
+    KS_CUDA(ctx->stats_counter.reserve(1, st, true), "allocate statistics counter");  // the W column prep
+    KS_CUDA(ctx->amax.reserve(1, st, false), "allocate amax");
+    if (want_wstat) KS_CUDA(ctx->wstat.reserve(2, st, false), "allocate weight statistics");
+    KS_CUDA(ks::launch_prep_fold_sources_coop(alpha, W, M, m_pad, K, k_pad, R, ctx->c, fold, grid,
+                                              ctx->mean_part.p, ctx->mean_pmm.p, ctx->mean_pw.p, ctx->coop_bar.p,
+                                              ctx->mu.p, ctx->amax.p, want_wstat ? ctx->wstat.p : nullptr,
+                                              ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wv.p, vcc, st),
+            "statistics + source prep (cooperative, folded)");
+  } else {
+    KS_CUDA(source_stats(ctx, alpha, W, want_wstat, M, k_pad, f16), "source statistics");
+  }
   const unsigned* wst = want_wstat ? ctx->wstat.p : nullptr;
   if (f16) {
-    KS_CUDA(ks::launch_prep_f16_sources(alpha, W, M, m_pad, K, k_pad, R, 0, ctx->mu.p, ctx->c,
-                                        ctx->amax.p, fold, ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p,
-                                        ctx->wt_lo.p, ctx->wv.p, vcc, wst, st),
-            "source prep (TC, FP16)");
+    if (!coop) {
+      KS_CUDA(ks::launch_prep_f16_sources(alpha, W, M, m_pad, K, k_pad, R, 0, ctx->mu.p, ctx->c,
+                                          ctx->amax.p, fold, ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wt_hi.p,
+                                          ctx->wt_lo.p, ctx->wv.p, vcc, wst, st),
+              "source prep (TC, FP16)");
+    }
     if (vcc == 0) {  // weighted sum on the tensor cores in FP16 (reading Q27): wcat in the W hi buffer
       int np = (int)((M + 1023) / 1024);
       if (np < 1) np = 1;
@@ -927,6 +951,7 @@ ks_status ks_destroy(ks_ctx* ctx) {
   ctx->wcol.release();
   ctx->wcol_part.release();
   ctx->stats_counter.release();
+  ctx->coop_bar.release();
   ctx->partial.release();
   ctx->counters.release();
   ctx->dbg_times.release();

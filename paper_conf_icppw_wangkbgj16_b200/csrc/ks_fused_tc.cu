@@ -27,6 +27,9 @@
 //            groups on alternate tiles) or P split into FP16 (or TF32) hi/lo written back to TMEM
 //            for the V MMA; V folded into FP64 and written (or a stream-K partial slot).
 // The M x N kernel matrix exists only as TMEM tiles.
+#ifndef KS_DEBUG
+#define KS_DEBUG 0  // measurement builds (libks_dbg.so): work-dropping knobs
+#endif
 #include "ks_internal.h"
 #include <cuda_fp16.h>
 #include "ks_ptx.cuh"
@@ -131,12 +134,15 @@ __device__ __forceinline__ bool f16_fold_ok(const unsigned* amax, double c, int 
 // c K amax^2 = 2^12 the norm pieces are stored as n 2^-s and the opposite operand's unit
 // columns hold 2^s (exact), s = ceil(log2(c K amax^2 / 2^12)) <= 15, so the folded layout is
 // valid for every input and needs no device-side fallback.
-__device__ __forceinline__ int f16_fold_shift(const unsigned* amax, double c, int K) {
-  const double a = (double)__uint_as_float(*amax);
+__device__ __forceinline__ int f16_fold_shift_v(float amax, double c, int K) {
+  const double a = (double)amax;
   const double v = c * (double)K * a * a / 4096.0;
   if (!(v > 1.0)) return 0;  // (NaN: 0)
   const int s = (int)ceil(log2(v));
   return s > 15 ? 15 : s;
+}
+__device__ __forceinline__ int f16_fold_shift(const unsigned* amax, double c, int K) {
+  return f16_fold_shift_v(__uint_as_float(*amax), c, K);
 }
 // balanced scaling: |2c x 2^eF| ~ |x 2^-eF| for coordinates of equal spread
 __device__ __forceinline__ int f16_fold_exp(double c) {
@@ -1653,36 +1659,25 @@ __device__ __forceinline__ void fold_store_row(void* base, int64_t row_halves, i
   }
 }
 
+// One source row i of the folded layout (8 lanes per row, lane g; the warp's rows all in range
+// or all out: full-mask shuffles).  mu may be global or shared memory; the uniform values (fold
+// shift fsh, scale exponent fexp, log2 max W) are evaluated once per block by the caller.
 template <int CPL>
-__global__ void __launch_bounds__(256) prep_fold_sources_kernel(
-    const float* __restrict__ alpha, const float* __restrict__ W, int64_t M, int64_t m_pad, int K, int R,
-    const float* __restrict__ mu, double c, int aug, const unsigned* __restrict__ amax, void* __restrict__ src_hi,
-    void* __restrict__ src_lo, float* __restrict__ na, float* __restrict__ wv, int rv,
-    const unsigned* __restrict__ wstat) {
+__device__ __forceinline__ void fold_source_row(const float* row, const float* wrow,
+                                                int64_t M, int K, int R, const float* mu, double c, bool logw,
+                                                int fsh, int fexp, double lwmax, int64_t i, int g,
+                                                void* __restrict__ src_hi, void* __restrict__ src_lo,
+                                                float* __restrict__ na, float* __restrict__ wv, int rv) {
   using L = FoldLanes<CPL>;
   constexpr int G = 8, KP = 8 * CPL;
-  pdl_wait();  // the source statistics are complete (trigger at the end)
-  __shared__ int s_fsh, s_fexp;
-  __shared__ double s_lwmax;
-  if (threadIdx.x == 0) {
-    s_fsh = f16_fold_shift(amax, c, K);
-    s_fexp = f16_fold_exp(c);
-    s_lwmax = (wstat != nullptr && wstat[0] != 0u) ? log2((double)__uint_as_float(wstat[0])) : 0.0;
-  }
-  __syncthreads();
-  const int lane = threadIdx.x & 31, g = lane & (G - 1);
-  const int64_t i = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
-  if (i >= m_pad) return;
   const bool live = i < M;
   float x[CPL];
-  fold_load_row<CPL>(alpha + i * K, mu, K, live, g, x);
+  fold_load_row<CPL>(row, mu, K, live, g, x);
   double n = 0.0;
 #pragma unroll
   for (int k = 0; k < CPL; ++k) n += (double)x[k] * (double)x[k];
   n = group_sum<G>(n);
-  const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && aug < 3;
-  const int fsh = s_fsh;
-  const float sA = ldexpf(1.f, s_fexp);
+  const float sA = ldexpf(1.f, fexp);
   const double c2 = 2.0 * c;
   const __half one = __float2half(ldexpf(1.f, fsh)), zero = __float2half(0.f);
   __half np[3] = {zero, zero, zero};
@@ -1693,7 +1688,7 @@ __global__ void __launch_bounds__(256) prep_fold_sources_kernel(
     has_np |= d >= K && d < K + 3;
   }
   double wl = 0.0;
-  if (has_np || (g == 0 && logw && rv > 0)) wl = !logw ? 0.0 : live ? log2((double)W[i]) - s_lwmax : -INFINITY;
+  if (has_np || (g == 0 && logw && rv > 0)) wl = !logw ? 0.0 : live ? log2((double)wrow[0]) - lwmax : -INFINITY;
   if (has_np) {
     const double nf = ldexp(-c * n + wl, -fsh);  // W_i = 0: the FP16 stand-in for -inf
     if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
@@ -1713,10 +1708,268 @@ __global__ void __launch_bounds__(256) prep_fold_sources_kernel(
   fold_store_row<CPL>(src_hi, i * KP, g, hi);
   fold_store_row<CPL>(src_lo, i * KP, g, lo);
   if (g == 0) na[i] = 0.f;  // folded: the norm and log-weight ride in the contraction
-  for (int r = g; r < rv; r += G) wv[i * rv + r] = logw ? (float)wl : (live && r < R) ? W[i * R + r] : 0.f;
+  for (int r = g; r < rv; r += G) wv[i * rv + r] = logw ? (float)wl : (live && r < R) ? wrow[r] : 0.f;
+}
+
+template <int CPL>
+__global__ void __launch_bounds__(256) prep_fold_sources_kernel(
+    const float* __restrict__ alpha, const float* __restrict__ W, int64_t M, int64_t m_pad, int K, int R,
+    const float* __restrict__ mu, double c, int aug, const unsigned* __restrict__ amax, void* __restrict__ src_hi,
+    void* __restrict__ src_lo, float* __restrict__ na, float* __restrict__ wv, int rv,
+    const unsigned* __restrict__ wstat) {
+  constexpr int G = 8;
+  pdl_wait();  // the source statistics are complete (trigger at the end)
+  __shared__ int s_fsh, s_fexp;
+  __shared__ double s_lwmax;
+  if (threadIdx.x == 0) {
+    s_fsh = f16_fold_shift(amax, c, K);
+    s_fexp = f16_fold_exp(c);
+    s_lwmax = (wstat != nullptr && wstat[0] != 0u) ? log2((double)__uint_as_float(wstat[0])) : 0.0;
+  }
+  __syncthreads();
+  const int lane = threadIdx.x & 31, g = lane & (G - 1);
+  const int64_t i = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
+  if (i < m_pad) {
+    const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && aug < 3;
+    fold_source_row<CPL>(alpha + i * K, W + i * R, M, K, R, mu, c, logw, s_fsh, s_fexp, s_lwmax, i, g, src_hi, src_lo, na, wv,
+                         rv);
+  }
   // PDL trigger last: a dependent fused kernel's CTA (640 threads, nearly all of an SM's registers)
   // launched early would hold its SM while waiting and starve this grid's remaining blocks
   pdl_trigger();
+}
+
+// Grid-wide barrier of a cooperative launch (every block resident), self-resetting so that any
+// launch order, CUDA-graph replay included, finds it at zero: arrivals bar[0] (each block's
+// thread 0 adds 1, then polls until all nblocks have arrived), departures bar[1]
+// (coop_grid_depart at the end of the kernel: the last block to depart -- every block has passed
+// the barrier by then -- zeroes both).  Thread 0 releases the block's writes (bar.sync, then a
+// fence) and acquires the others'.
+__device__ __forceinline__ void coop_grid_sync(unsigned* bar, unsigned nblocks) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    atomicAdd(bar, 1u);
+    unsigned v;
+    do {
+      asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
+    } while (v < nblocks);
+  }
+  __syncthreads();
+}
+__device__ __forceinline__ void coop_grid_depart(unsigned* bar, unsigned nblocks) {
+  if (threadIdx.x == 0 && atomicAdd(bar + 1, 1u) == nblocks - 1u) {
+    bar[0] = 0u;
+    bar[1] = 0u;
+  }
+}
+
+// Source statistics and the folded source prep in ONE cooperative launch (scope row a1; the
+// separate path is source_stats_kernel (+ stats_final_kernel) + prep_fold_sources_kernel, whose
+// launch latencies chained to ~28 us at cfg3, SS6).  One 1024-thread block per SM,
+// block b owns rows [b chunk, (b + 1) chunk) of the padded layout (chunk a multiple of 64):
+//   phase 1  the block's rows, contiguous in memory, staged into shared memory with 16-byte
+//            loads (sub-chunks of `rows_cap` rows when they do not fit), then reduced in a fixed
+//            order: FP64 column sums, FP32 column min/max, weight max / "any W_i < 0 or NaN"
+//            -> partials [b]
+//   barrier  (coop_grid_sync)
+//   phase 2  EVERY block reduces the G partials in the same fixed order (identical arithmetic,
+//            so identical mu / amax / wstat in every block; block 0 publishes them for the
+//            target prep and the fused kernel) -- no second barrier
+//   phase 3  the block's rows through fold_source_row, from shared memory when the whole chunk
+//            was staged (else re-read from L2).
+// mu, amax and wstat are the same quantities as launch_source_stats' (the FP64 column sums
+// may round differently: a different fixed order).
+constexpr int kCoopThreads = 1024;
+template <int CPL>
+__global__ void __launch_bounds__(kCoopThreads, 1) prep_fold_sources_coop_kernel(
+    const float* __restrict__ alpha, const float* __restrict__ W, int64_t M, int64_t m_pad, int K, int k_pad, int R,
+    double c, int aug, int64_t chunk, int rows_cap, double* __restrict__ part, float* __restrict__ pmm,
+    unsigned* __restrict__ pw, unsigned* __restrict__ bar, float* __restrict__ mu, unsigned* __restrict__ amax,
+    unsigned* __restrict__ wstat, void* __restrict__ src_hi, void* __restrict__ src_lo, float* __restrict__ na,
+    float* __restrict__ wv, int rv, int dbg_stop) {
+  constexpr int NT = kCoopThreads;
+  extern __shared__ __align__(16) float s_a[];  // [rows_cap][K], then (R = 1) [rows_cap] weights
+  float* s_wr = s_a + (size_t)rows_cap * K;
+  __shared__ double red[NT];
+  __shared__ float rmn[NT], rmx[NT];
+  __shared__ float s_mu[64];
+  __shared__ unsigned s_w[2], s_amax;
+  __shared__ int s_fsh, s_fexp;
+  __shared__ bool s_logw;
+  __shared__ double s_lwmax;
+  const unsigned nb = gridDim.x;
+  const int b = blockIdx.x, t = threadIdx.x;
+  const bool want_w = wstat != nullptr;
+  if (t == 0) {
+    s_w[0] = s_w[1] = 0u;
+    s_amax = 0u;
+  }
+  const int64_t r0 = (int64_t)b * chunk < m_pad ? (int64_t)b * chunk : m_pad;
+  const int64_t r1 = r0 + chunk < m_pad ? r0 + chunk : m_pad;  // padded rows of this block
+  const int64_t r1m = r1 < M ? r1 : M;                          // live rows
+  const bool staged = r1m - r0 <= rows_cap;                      // phase 3 reads shared memory
+  // ---- phase 1: partials of this block's rows (rpp row lanes x K dims)
+  const int rpp = NT / K, ro = t / K, d = t % K;
+  {
+    double s = 0.0;
+    float mn = INFINITY, mx = -INFINITY;
+    for (int64_t q0 = r0; q0 < r1m; q0 += rows_cap) {
+      const int nr = (int)(r1m - q0 < rows_cap ? r1m - q0 : rows_cap);
+      const int n = nr * K;
+      const float* src = alpha + q0 * K;  // 16-byte aligned: q0 is a multiple of 64
+      __syncthreads();                    // the previous sub-chunk is consumed
+      const int n4 = n >> 2;
+#pragma unroll 4
+      for (int e = t; e < n4; e += NT)
+        reinterpret_cast<float4*>(s_a)[e] = __ldg(reinterpret_cast<const float4*>(src) + e);
+      for (int e = 4 * n4 + t; e < n; e += NT) s_a[e] = src[e];
+      __syncthreads();
+      if (ro < rpp)
+#pragma unroll 4
+        for (int r = ro; r < nr; r += rpp) {
+          const float x = s_a[r * K + d];
+          s += (double)x;
+          mn = fminf(mn, x);
+          mx = fmaxf(mx, x);
+        }
+    }
+    float wm = 0.f;
+    unsigned neg = 0u;
+    if (want_w) {
+#pragma unroll 4
+      for (int64_t r = r0 + t; r < r1m; r += NT) {
+        const float w = W[r];
+        if (staged) s_wr[r - r0] = w;  // phase 3 reads it from here
+        wm = fmaxf(wm, fabsf(w));
+        neg |= (w < 0.f || w != w) ? 1u : 0u;  // NaN weights take the general path
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        wm = fmaxf(wm, __shfl_xor_sync(0xffffffffu, wm, o));
+        neg |= __shfl_xor_sync(0xffffffffu, neg, o);
+      }
+    }
+    red[t] = s;
+    rmn[t] = mn;
+    rmx[t] = mx;
+    __syncthreads();  // red / rmn / rmx written, s_w initialised
+    if (want_w && (t & 31) == 0) {
+      atomicMax(&s_w[0], __float_as_uint(wm));  // max and or: order-independent, exact
+      atomicOr(&s_w[1], neg);
+    }
+    if (t < K) {
+      double acc = 0.0;
+      for (int q = 0; q < rpp; ++q) {
+        acc += red[q * K + t];
+        mn = fminf(mn, rmn[q * K + t]);
+        mx = fmaxf(mx, rmx[q * K + t]);
+      }
+      part[(int64_t)b * K + t] = acc;
+      pmm[((int64_t)b * K + t) * 2] = mn;
+      pmm[((int64_t)b * K + t) * 2 + 1] = mx;
+    }
+    __syncthreads();
+    if (want_w && t == 0) {
+      pw[2 * b] = s_w[0];
+      pw[2 * b + 1] = s_w[1];
+    }
+  }
+  if (KS_DEBUG && dbg_stop == 1) return;  // measurement builds: phase 1 only (wrong results)
+  coop_grid_sync(bar, nb);  // (orders every thread's partials: bar.sync, then thread 0's fence)
+  if (KS_DEBUG && dbg_stop == 2) {  // + the barrier
+    coop_grid_depart(bar, nb);
+    return;
+  }
+  // ---- phase 2: the nb partials, the same fixed order in every block
+  {
+    double s = 0.0;
+    float mn = INFINITY, mx = -INFINITY;
+    if (ro < rpp)
+#pragma unroll 4
+      for (int q = ro; q < (int)nb; q += rpp) {
+        s += __ldcg(&part[(int64_t)q * K + d]);
+        const float2 m2 = __ldcg(reinterpret_cast<const float2*>(&pmm[((int64_t)q * K + d) * 2]));
+        mn = fminf(mn, m2.x);
+        mx = fmaxf(mx, m2.y);
+      }
+    red[t] = s;
+    rmn[t] = mn;
+    rmx[t] = mx;
+    if (t == 0) s_w[0] = s_w[1] = 0u;
+    __syncthreads();
+    if (t < K) {
+      double acc = 0.0;
+      for (int q = 0; q < rpp; ++q) {
+        acc += red[q * K + t];
+        mn = fminf(mn, rmn[q * K + t]);
+        mx = fmaxf(mx, rmx[q * K + t]);
+      }
+      const float m = M > 0 ? (float)(acc / (double)M) : 0.f;
+      s_mu[t] = m;
+      // NaN coordinates give a NaN mean; fmaxf(NaN, 0) = 0 then ignores them
+      if (M > 0) atomicMax(&s_amax, __float_as_uint(fmaxf(fmaxf(mx - m, m - mn), 0.f)));
+    } else if (t < k_pad) {
+      s_mu[t] = 0.f;
+    }
+    if (want_w && t >= NT - 32) {  // the last warp: weight statistics
+      const int l = t & 31;
+      unsigned wm = 0u, neg = 0u;
+      for (int q = l; q < (int)nb; q += 32) {
+        wm = max(wm, __ldcg(&pw[2 * q]));
+        neg |= __ldcg(&pw[2 * q + 1]);
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        wm = max(wm, __shfl_xor_sync(0xffffffffu, wm, o));
+        neg |= __shfl_xor_sync(0xffffffffu, neg, o);
+      }
+      if (l == 0) {
+        s_w[0] = wm;  // non-negative FP32 values order as their bit patterns
+        s_w[1] = neg;
+      }
+    }
+    __syncthreads();
+    if (t == 0) {  // the block-uniform values of phase 3, once (FP64 log2: ~100 FP64 instructions each)
+      s_fsh = f16_fold_shift_v(__uint_as_float(s_amax), c, K);
+      s_fexp = f16_fold_exp(c);
+      s_logw = want_w && s_w[1] == 0u && s_w[0] != 0u && aug < 3;
+      s_lwmax = (want_w && s_w[0] != 0u) ? log2((double)__uint_as_float(s_w[0])) : 0.0;
+    }
+    if (b == 0) {
+      if (t < k_pad) mu[t] = s_mu[t];
+      if (t == 0) {
+        *amax = s_amax;
+        if (want_w) {
+          wstat[0] = s_w[0];
+          wstat[1] = s_w[1];
+        }
+      }
+    }
+  }
+  if (KS_DEBUG && dbg_stop == 3) {  // + the final statistics
+    coop_grid_depart(bar, nb);
+    return;
+  }
+  // ---- phase 3: this block's rows of the padded layout (multiples of 64 rows: whole warps)
+  __syncthreads();
+  {
+    const int fsh = s_fsh, fexp = s_fexp;
+    const bool logw = s_logw;
+    const double lwmax = s_lwmax;
+    const int g = t & 7;
+    // warp-uniform row base (the warp index through a shuffle: the compiler then knows the warp
+    // is converged at group_sum's shuffles and emits plain SHFL, not WARPSYNC.COLLECTIVE loops)
+    const int64_t wb = r0 + 4 * __shfl_sync(0xffffffffu, t >> 5, 0);
+    for (int64_t base = wb; base < r1; base += NT / 8) {
+      const int64_t i = base + ((t & 31) >> 3);
+      const float* row = staged ? s_a + (i - r0) * K : alpha + i * K;
+      const float* wrow = (staged && R == 1) ? s_wr + (i - r0) : W + i * R;
+      fold_source_row<CPL>(row, wrow, M, K, R, s_mu, c, logw, fsh, fexp, lwmax, i, g, src_hi, src_lo, na, wv, rv);
+    }
+  }
+  coop_grid_depart(bar, nb);
+  pdl_trigger();  // the target prep / fused kernel may launch (they wait for this grid to complete)
 }
 
 template <int CPL>
@@ -1850,6 +2103,66 @@ cudaError_t launch_prep_tc_sources(const float* alpha, const float* W, int64_t M
                                    const unsigned* wstat, cudaStream_t st) {
   return launch_prep_sources<false>(alpha, W, M, m_pad, K, k_pad, R, r_pad, mu, c, aug, nullptr, src_hi, src_lo, na,
                                     wt_hi, wt_lo, wv, rv, wstat, st);
+}
+
+// Cooperative statistics + folded source prep: one block per SM (every block resident).
+constexpr int kCoopSmem = 160 * 1024;  // staged source rows per block
+
+int coop_prep_grid(int k_pad, int64_t m_pad, int num_sms) {
+  (void)k_pad;
+  int64_t g = num_sms;
+  const int64_t need = (m_pad + 63) / 64;
+  if (g > need) g = need;
+  return g < 1 ? 1 : (int)g;
+}
+
+template <int CPL>
+static cudaError_t coop_launch(const cudaLaunchConfig_t& cfg, const float* alpha, const float* W, int64_t M,
+                               int64_t m_pad, int K, int k_pad, int R, double c, int fold, int64_t chunk, int rows_cap,
+                               double* part, float* pmm, unsigned* pw, unsigned* bar, float* mu, unsigned* amax,
+                               unsigned* wstat, void* src_hi, void* src_lo, float* na, float* wv, int rv) {
+  static std::atomic<uint64_t> attr_done{0};
+  cudaError_t e = smem_optin_once(attr_done, reinterpret_cast<const void*>(prep_fold_sources_coop_kernel<CPL>),
+                                  kCoopSmem);
+  if (e != cudaSuccess) return e;
+  int dbg_stop = 0;
+#if KS_DEBUG
+  {
+    const char* ev = getenv("KS_COOP_STOP");  // measurement builds only: stop after phase n
+    dbg_stop = ev ? atoi(ev) : 0;
+  }
+#endif
+  return cudaLaunchKernelEx(&cfg, prep_fold_sources_coop_kernel<CPL>, alpha, W, M, m_pad, K, k_pad, R, c, fold, chunk,
+                            rows_cap, part, pmm, pw, bar, mu, amax, wstat, src_hi, src_lo, na, wv, rv, dbg_stop);
+}
+
+cudaError_t launch_prep_fold_sources_coop(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K,
+                                          int k_pad, int R, double c, int fold, int grid, double* part, float* pmm,
+                                          unsigned* pw, unsigned* bar, float* mu, unsigned* amax, unsigned* wstat,
+                                          void* src_hi, void* src_lo, float* na, float* wv, int rv, cudaStream_t st) {
+  const int64_t per = (m_pad + grid - 1) / grid;
+  const int64_t chunk = (per + 63) / 64 * 64;
+  int rows_cap = (kCoopSmem / (4 * (K + 1))) / 64 * 64;  // >= 64 rows for K <= 58
+  if (rows_cap > chunk) rows_cap = (int)chunk;
+  const size_t smem = (size_t)4 * (K + 1) * rows_cap;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(kCoopThreads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;  // all blocks co-resident (grid barrier); no PDL
+  attr[0].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  if (k_pad == 16)
+    return coop_launch<2>(cfg, alpha, W, M, m_pad, K, k_pad, R, c, fold, chunk, rows_cap, part, pmm, pw, bar, mu, amax,
+                          wstat, src_hi, src_lo, na, wv, rv);
+  if (k_pad == 32)
+    return coop_launch<4>(cfg, alpha, W, M, m_pad, K, k_pad, R, c, fold, chunk, rows_cap, part, pmm, pw, bar, mu, amax,
+                          wstat, src_hi, src_lo, na, wv, rv);
+  return coop_launch<8>(cfg, alpha, W, M, m_pad, K, k_pad, R, c, fold, chunk, rows_cap, part, pmm, pw, bar, mu, amax,
+                        wstat, src_hi, src_lo, na, wv, rv);
 }
 
 cudaError_t launch_prep_f16_sources(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K, int k_pad,

@@ -228,6 +228,15 @@ cudaError_t launch_prep_f16_sources(const float* alpha, const float* W, int64_t 
                                     int R, int r_pad, const float* mu, double c, const unsigned* amax, int fold,
                                     void* src_hi, void* src_lo, float* na, float* wt_hi, float* wt_lo, float* wv,
                                     int rv, const unsigned* wstat, cudaStream_t st);
+// Folded layouts (fold 2, 3; k_pad in {16, 32, 64}, K + 6 <= k_pad): the source statistics (mu,
+// amax, and wstat when non-null) and the folded source prep in one cooperative launch of `grid`
+// blocks (coop_prep_grid; scratch part [grid][K], pmm [grid][K][2], pw [grid][2]; bar [2] zero
+// when allocated, left zero by every launch).  Same outputs as launch_source_stats + launch_prep_f16_sources.
+int coop_prep_grid(int k_pad, int64_t m_pad, int num_sms);
+cudaError_t launch_prep_fold_sources_coop(const float* alpha, const float* W, int64_t M, int64_t m_pad, int K,
+                                          int k_pad, int R, double c, int fold, int grid, double* part, float* pmm,
+                                          unsigned* pw, unsigned* bar, float* mu, unsigned* amax, unsigned* wstat,
+                                          void* src_hi, void* src_lo, float* na, float* wv, int rv, cudaStream_t st);
 cudaError_t launch_prep_f16_targets(const float* beta, int64_t N, int64_t n_pad, int K, int k_pad, const float* mu,
                                     double c, const unsigned* amax, int fold, void* tgt_hi, void* tgt_lo, float* nb,
                                     float* tsc, cudaStream_t st);

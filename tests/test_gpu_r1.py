@@ -222,3 +222,67 @@ def test_large_magnitudes_stay_finite(oracle_mod, K, opts):
     Vr = oracle_mod.oracle_eval(a, W, a, float(h))
     cka2 = np.log2(np.e) / (2 * 0.25) * K * float(np.abs(a - a.mean(0)).max()) ** 2
     assert e_norm(V, Vr, W) <= 2.0**-18 * cka2 / 600 + 1e-7
+
+
+def _run_any(alpha, W, beta, h, **opts):
+    with ks.KernelSum(alpha.shape[1], float(h), "auto", options=opts) as plan:
+        plan.set_sources(torch.from_numpy(np.ascontiguousarray(alpha)).cuda(),
+                         torch.from_numpy(np.ascontiguousarray(W)).cuda())
+        V = plan.eval(torch.from_numpy(np.ascontiguousarray(beta)).cuda())
+        torch.cuda.synchronize()
+        return V.cpu().numpy().astype(np.float64), plan.info()
+
+
+@pytest.mark.parametrize("K", [1, 4, 10, 16, 26, 32, 58])
+@pytest.mark.parametrize("M,R,wkind", [(1, 1, "pos"), (777, 1, "signed"), (70001, 1, "pos"), (5000, 3, "signed"),
+                                       (3000, 1, "zero")])
+def test_cooperative_source_prep(oracle_mod, K, M, R, wkind):
+    """Source statistics + folded source prep in one cooperative launch (option coop_prep, the
+    default for the R = 1 and multi-column kernels; a grid barrier between the partial and the
+    final statistics) against the separate statistics and prep kernels: the same layout and
+    scales, so V agrees to the rounding of mu's FP64 column sums (a different fixed order); the
+    result meets the bar and is bitwise reproducible.  Covers one source, ragged counts, more
+    rows than one block's share (70,001), R > 1 (multi-column kernel, no weight statistics),
+    negative weights (the weight mode) and all-zero weights."""
+    if wkind == "zero":
+        a, W, b, h = workloads.custom(M, 300, K, R, 1.0, dist="gm", sigma=0.1, wkind="pos", seed=K + M)
+        W = np.zeros_like(W)
+    else:
+        a, W, b, h = workloads.custom(M, 300, K, R, 1.0, dist="gm", sigma=0.1, wkind=wkind, seed=K + M)
+    Vc, info = _run_any(a, W, b, h)
+    assert info["launches"] >= 1
+    Vs, _ = _run_any(a, W, b, h, coop_prep=0)
+    Vc2, _ = _run_any(a, W, b, h)
+    assert np.array_equal(Vc, Vc2)
+    den = max(np.abs(W).sum(), 1e-30)
+    assert np.max(np.abs(Vc - Vs)) / den <= 1e-6
+    Vr = oracle_mod.oracle_eval(a, W, b, float(h))
+    if wkind == "zero":
+        assert np.all(Vc == 0.0)
+    else:
+        assert e_norm(Vc, Vr, W) <= TOL_3XTF32
+
+
+def test_cooperative_prep_graph_replay():
+    """The cooperative source prep's grid barrier resets itself, so ks_set_sources can be
+    captured in a CUDA graph and replayed any number of times, interleaved with live calls."""
+    a, W, b, h = workloads.make(3, M=9000, N=1000, wkind="pos")
+    a2 = a[::-1].copy()
+    ta, ta2, tw, tb = (torch.from_numpy(x).cuda() for x in (a, a2, W, b))
+    with ks.KernelSum(a.shape[1], float(h), "auto") as plan:
+        s = torch.cuda.Stream()
+        with torch.cuda.stream(s):
+            plan.set_sources(ta, tw)
+            ref = plan.eval(tb).clone()
+            plan.set_sources(ta2, tw)
+            s.synchronize()
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=s):
+                plan.set_sources(ta, tw)
+            for _ in range(3):
+                plan.set_sources(ta2, tw)
+                g.replay()
+                g.replay()
+                V = plan.eval(tb)
+                s.synchronize()
+                assert torch.equal(V, ref)
