@@ -68,6 +68,9 @@ def parse():
     p.add_argument("--cpu-seconds", type=float, default=16.0,
                    help="target CPU time of the oracle sample (cfg3 on 16 cores: every target)")
     p.add_argument("--no-flush", action="store_true")
+    p.add_argument("--no-traffic", action="store_true",
+                   help="skip the live ncu DRAM-byte probe of the fused kernel (roofline.traffic)")
+    p.add_argument("--traffic-probe", action="store_true", help=argparse.SUPPRESS)  # child under ncu
     p.add_argument("--precision", default="auto", choices=["auto", "fp32", "3xtf32", "3xf16", "tf32"],
                    help="ks_set_precision (auto: FP32 path for K<=32 and R=1, else 3xTF32 tensor cores)")
     return p.parse_args()
@@ -249,6 +252,56 @@ def load_peaks():
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
     except Exception:
         return {}
+
+
+def traffic_probe_child(args):
+    """Under ncu (measure_traffic): the timed step's set_sources + eval on the same workload, a
+    few times, nothing printed -- ncu records the DRAM counters of the fused kernel."""
+    import torch
+    import paper_conf_icppw_wangkbgj16_b200 as ks
+    c = workloads.CONFIGS[args.cfg]
+    a, W, b, h = workloads.make(c)
+    ta, tw, tb = (torch.from_numpy(x).cuda() for x in (a, W, b))
+    plan = ks.KernelSum(c.K, float(h), args.precision)
+    V = torch.empty((c.N, c.R), device="cuda")
+    flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device="cuda")
+    for _ in range(3):
+        l2_flush(flush)
+        plan.set_sources(ta, tw)
+        plan.eval(tb, out=V)
+    torch.cuda.synchronize()
+    plan.close()
+
+
+def measure_traffic(args, timeout=240):
+    """roofline.traffic measured in this run: ncu (dram__bytes_read.sum + dram__bytes_write.sum,
+    --clock-control none) over the third fused-kernel launch of a child process that runs this
+    workload's step after an L2 flush, like the timed steps.  None when ncu is missing or fails
+    (the caller then falls back to the committed capture)."""
+    import shutil
+    import subprocess
+    ncu = shutil.which("ncu") or "/usr/local/cuda/bin/ncu"
+    if not os.path.exists(ncu):
+        return None
+    cmd = [ncu, "--metrics", "dram__bytes_read.sum,dram__bytes_write.sum", "--clock-control", "none",
+           "--kernel-name", "regex:ks_fused_", "--launch-skip", "2", "--launch-count", "1", "--csv",
+           sys.executable, os.path.abspath(__file__), "--traffic-probe", "--cfg", str(args.cfg),
+           "--precision", args.precision]
+    try:
+        r = subprocess.run(cmd, capture_output=True, text=True, timeout=timeout)
+        rows = [ln for ln in r.stdout.splitlines() if ln.startswith('"') and "dram__bytes" in ln]
+        import csv
+        tot, kern = 0.0, None
+        unit_scale = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "MB": 1e6, "GB": 1e9}
+        for row in csv.reader(rows):
+            # "ID","Process ID","Process Name","Host Name","Kernel Name",...,"Metric Name","Metric Unit","Metric Value"
+            tot += float(row[-1].replace(",", "")) * unit_scale.get(row[-2], 1.0)
+            kern = row[4]
+        if kern is None:
+            return None
+        return {"bytes": tot, "kernel": kern.split("(")[0]}
+    except Exception:
+        return None
 
 
 def load_traffic(cfg, precision="auto"):
@@ -543,6 +596,19 @@ def run_ours(args):
     if energy is not None:
         out["energy"] = energy
 
+    # ---- roofline.traffic: ncu DRAM bytes of one fused launch of this workload, measured now (N=1,
+    # after the timed region; a child process under ncu), else the committed capture
+    if rank == 0 and world == 1 and not args.no_traffic:
+        tr = measure_traffic(args)
+        if tr is not None:
+            roof["traffic"] = tr["bytes"]
+            roof["traffic_source"] = ("measured in this run: ncu dram__bytes_read.sum + dram__bytes_write.sum, "
+                                      "--clock-control none, one launch of %s after an L2 flush" % tr["kernel"])
+        elif roof.get("traffic") is not None:
+            roof["traffic_source"] = "committed ncu capture (profiles/ncu_summary.json); the live probe failed"
+    # algorithmic bytes per launch: alpha, W, beta in FP32, V out
+    roof["algorithmic_bytes"] = 4 * (M * K + M * R + (hi - lo) * K + (hi - lo) * R)
+
     # ---- CPU baseline (oracle) on rank 0 at N=1 only; also a parity spot-check of the timed V
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cb, J, Vr = cpu_baseline(a, W, b, h, args.cpu_seconds)
@@ -626,7 +692,9 @@ def run_unfused(args):
 
 def main():
     args = parse()
-    if args.impl == "reference":
+    if args.traffic_probe:
+        traffic_probe_child(args)
+    elif args.impl == "reference":
         run_reference(args)
     elif args.impl == "unfused":
         run_unfused(args)
