@@ -369,8 +369,6 @@ def run_ours(args):
     ev0 = [torch.cuda.Event(enable_timing=True) for _ in range(n_ev)]
     ev1 = [torch.cuda.Event(enable_timing=True) for _ in range(n_ev)]
     info0 = plan.info()
-    ks.ks_timing_read(plan.ctx, reset=True)
-    ks.ks_timing_enable(plan.ctx, True)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -384,9 +382,21 @@ def run_ours(args):
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
+    info1 = plan.info()
+    # ---- kernel pass: the same K steps again with CUDA events on the launching stream around every
+    # fused launch (ks_timing).  Not inside the timed region above: an event recorded between two
+    # programmatic-dependent launches stops the fused kernel's prologue from overlapping the target
+    # prep, measured +8-12 us per step (SS7).
+    ks.ks_timing_read(plan.ctx, reset=True)
+    ks.ks_timing_enable(plan.ctx, True)
+    torch.cuda.synchronize()
+    for i in range(n_ev):
+        if flush is not None:
+            l2_flush(flush)
+        step()
+    torch.cuda.synchronize()
     ks.ks_timing_enable(plan.ctx, False)
     kern_ms, kern_n = ks.ks_timing_read(plan.ctx, reset=True)
-    info1 = plan.info()
     try:  # effective SM clock of the last timed fused launch (clock64 / globaltimer per CTA)
         kern_ghz = ks.ks_clock_read(plan.ctx)[0]
     except ks.KsError:
@@ -488,7 +498,9 @@ def run_ours(args):
                                    f"16/clk/SM is not binding at K={K}"}
         if clk_sum["sm_mhz"]:
             roof["frac_at_measured_clock"] = achieved / (128 * sms * clk_sum["sm_mhz"] * 1e6 / 1e12)
-    roof.update({"kernel_ms": kms, "kernel_launches_per_step": kern_n / args.steps,
+    roof.update({"kernel_ms": kms, "kernel_timing": "CUDA events around every fused launch on its stream, in a "
+                 "second pass of the same K steps (events inside the timed steps would break the "
+                 "programmatic-dependent-launch overlap)", "kernel_launches_per_step": kern_n / args.steps,
                  "kernel_share_of_step": kms / ms_per_step if ms_per_step else None,
                  "pairs_per_step": pairs_launch})
 

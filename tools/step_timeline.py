@@ -37,11 +37,12 @@ for e in ev:
     if "elementwise" in name or "fill" in name.lower():  # the L2 flush starts a step
         if step:
             print(f"  step span {step[-1][1] + step[-1][2]:.1f} us")
-        step, t0, prev_end = [], None, None
-        print("-- step")
+        step, t0, prev_end = [], None, e.time_range.end
+        print(f"-- step (L2 flush {e.time_range.end - e.time_range.start:.1f} us)")
         continue
     s, d = e.time_range.start, e.time_range.end - e.time_range.start
     if t0 is None:
+        print(f"  first kernel starts {s - prev_end:.1f} us after the flush ends")
         t0 = s
     gap = 0.0 if prev_end is None else s - prev_end
     prev_end = e.time_range.end
