@@ -39,7 +39,8 @@ EXPORTED = ("ks_create", "ks_destroy", "ks_set_precision", "ks_set_stream", "ks_
 OPTIONS = {"r1_kernel": 1, "r1_epilogue": 2, "exp_poly": 3, "weighted_sum": 4, "log_weights": 5, "fold": 6,
            "aug": 7, "clamp": 8, "target_resident": 9, "stages": 10, "ar_stages": 11, "wslots": 12,
            "prep_lanes": 13, "eval_chunks": 14, "fp32_split": 15, "measure_clock": 16,
-           "eval_chunk0": 17, "coop_prep": 18}
+           "eval_chunk0": 17, "coop_prep": 18,
+           "dyn_tail": 19, "dyn_chunk": 20}
 
 
 class KsInfo(ctypes.Structure):
