@@ -184,12 +184,10 @@ typedef enum {
   KS_OPT_COOP_PREP = 18,      /* KS_COOP_PREP: folded layouts (R = 1 and multi-column kernels):
                                  1 (default) source statistics and prep in one cooperative
                                  launch, 0 the separate kernels [sources] */
-  KS_OPT_DYN_TAIL = 19,       /* KS_DYN_TAIL: R = 1 kernel with >= 2 waves of target tiles: 1
-                                 the last wave and the remainder claimed in chunks by the CTAs
-                                 (balances SMs at different clocks; measured not faster under
-                                 the power cap), 0 (default) static stream-K split [eval] */
-  KS_OPT_DYN_CHUNK = 20,      /* KS_DYN_CHUNK: dynamic tail's minimum chunk in units (0: 16) [eval] */
-  KS_OPT_COUNT_ = 21
+  KS_OPT_FOLD_NARROW = 19,    /* KS_FOLD_NARROW: R = 1 kernel, 27 <= K <= 32: 1 (default) the
+                                 folded norm pieces load as one 16-column plane of 32-byte rows,
+                                 0 as a second 64-byte chunk [eval] */
+  KS_OPT_COUNT_ = 20
 } ks_option;
 
 /* Set / read a tuning option.  KS_EINVAL for an unknown option or a value out of its range. */

@@ -146,6 +146,7 @@ struct ks_ctx {
   int rv = 0;      // R > 1 folded kernel (ks_fused_rv.cu)
   int r1_clamp = 0;
   CUtensorMap tmB_hi, tmB_lo;
+  CUtensorMap tmB_f;  // R = 1 fold_narrow: columns 32..47 of the source hi plane, 32-byte boxes
   DBuf<float> mu;         // [k_pad]
   DBuf<double> mean_part; // [nparts][K]
   DBuf<float> mean_pmm;   // [nparts][K][2] column min/max
@@ -162,8 +163,6 @@ struct ks_ctx {
   // eval scratch
   DBuf<float> partial;
   DBuf<int> counters;
-  DBuf<unsigned long long> dyn_claim;  // R = 1 dynamic tail: {chunks claimed, CTAs departed}
-  DBuf<float> dyn_slots;               // ... chunk partials
   DBuf<unsigned long long> dbg_times;
   int last_grid = 0;
 
@@ -220,8 +219,7 @@ const OptSpec kOpt[KS_OPT_COUNT_] = {
     {"KS_MEASURE_CLOCK", 0, 0, 1},
     {"KS_EVAL_CHUNK0", 0, -1, 1 << 20},
     {"KS_COOP_PREP", 1, 0, 1},
-    {"KS_DYN_TAIL", 0, 0, 1},
-    {"KS_DYN_CHUNK", 0, 0, 4096},
+    {"KS_FOLD_NARROW", 1, 0, 1},
 };
 
 void init_opts(ks_ctx* ctx) {
@@ -565,6 +563,10 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   if (s != KS_OK) return s;
   s = encode_2d_sw64(&ctx->tmB_lo, ctx->src_lo.p, k_pad, m_pad, box_s, f16, narrow);
   if (s != KS_OK) return s;
+  if (r1 && k_pad == 64) {  // the fold chunk as one 16-column plane (fold_narrow, eval_r1)
+    s = encode_2d_sw64(&ctx->tmB_f, ctx->src_hi.p, k_pad, m_pad, box_s, true, true);
+    if (s != KS_OK) return s;
+  }
   ctx->k_pad = k_pad;
   ctx->m_pad = m_pad;
   ctx->r_pad = r_pad;
@@ -581,43 +583,6 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   return KS_OK;
 }
 
-// R = 1 kernel's dynamic tail (KS_OPT_DYN_TAIL, off by default): with at least two whole waves of
-// target tiles, the last whole wave and the remainder are claimed in chunks of C units (C a
-// multiple of 4 dividing n_s, C >= 16 (KS_OPT_DYN_CHUNK) and >= n_s / 64, so <= 64 chunk slots per
-// tile).  SMs run at different clocks (per-CTA clock64 / globaltimer at cfg3: 1.658 vs 1.700 GHz,
-// equal cycle counts), so a static split ends at the slowest SM; claimed chunks let the faster
-// ones take more.  Measured at cfg3 (bench A/B, same box): the CTA ends tighten from a 37 to a
-// 9 us spread, but the chunk segments add ~2.7% cycles and the finish launch ~4 us, and under the
-// board power cap the balanced run is not faster (0.909-0.915 vs 0.899 ms per step): kept off.
-struct DynPlan {
-  int on = 0, c = 0, nc = 0;
-  int64_t t0 = 0;
-};
-DynPlan r1_dyn_plan(const ks_ctx* ctx, int64_t n_t, int64_t grid) {
-  DynPlan p;
-  const int64_t n_s = ctx->m_pad / 128;
-  if (ctx->opts.v[KS_OPT_DYN_TAIL] == 0 || grid <= 0 || n_t / grid < 2) return p;
-  const int oc = ctx->opts.v[KS_OPT_DYN_CHUNK];
-  const int64_t cmin = std::max<int64_t>(oc > 0 ? oc : 16, (n_s + 63) / 64);
-  for (int64_t c = (cmin + 3) / 4 * 4; c <= n_s; c += 4) {
-    if (n_s % c == 0) {
-      p.on = 1;
-      p.c = (int)c;
-      p.nc = (int)(n_s / c);
-      p.t0 = (n_t / grid - 1) * grid;
-      break;
-    }
-  }
-  return p;
-}
-
-ks_status reserve_dyn(ks_ctx* ctx, const DynPlan& p, int64_t n_t) {
-  if (!p.on) return KS_OK;
-  KS_CUDA(ctx->dyn_claim.reserve(2, ctx->stream, true), "allocate chunk claim counter");
-  KS_CUDA(ctx->dyn_slots.reserve((size_t)(n_t - p.t0) * p.nc * 4 * 128, ctx->stream, false), "allocate chunk slots");
-  return KS_OK;
-}
-
 // R = 1 folded kernel (ks_fused_r1.cu): 128-source units, one launch.
 ks_status eval_r1(ks_ctx* ctx, const CUtensorMap* maps, int64_t N, float* V) {
   cudaStream_t st = ctx->stream;
@@ -630,16 +595,10 @@ ks_status eval_r1(ks_ctx* ctx, const CUtensorMap* maps, int64_t N, float* V) {
   sk.grid = (int32_t)g;
   KS_CUDA(ctx->partial.reserve((size_t)sk.grid * 2 * 128, st, false), "allocate partials");
   KS_CUDA(ctx->counters.reserve((size_t)sk.n_t, st, true), "allocate tile counters");
-  const DynPlan dp = r1_dyn_plan(ctx, sk.n_t, sk.grid);
-  ks_status ds = reserve_dyn(ctx, dp, sk.n_t);
-  if (ds != KS_OK) return ds;
   ks::R1Args a;
-  a.dyn = dp.on;
-  a.dyn_c = dp.c;
-  a.dyn_nc = dp.nc;
-  a.dyn_t0 = dp.on ? dp.t0 : sk.n_t;
-  a.claim = ctx->dyn_claim.p;
-  a.cslots = ctx->dyn_slots.p;
+  // the second operand chunk holds only the folded norm pieces: load it as one 16-column plane
+  a.fold_narrow = (ctx->k_pad == 64 && ctx->tc_kdims <= 32 && ctx->tc_kcols <= 48 &&
+                   ctx->opts.v[KS_OPT_FOLD_NARROW] != 0) ? 1 : 0;
   a.N = N;
   a.narrow = ctx->k_pad == ks::kTcKC ? 1 : 0;
   a.n_kc = a.narrow ? 1 : ctx->k_pad / 32;
@@ -676,10 +635,6 @@ ks_status eval_r1(ks_ctx* ctx, const CUtensorMap* maps, int64_t N, float* V) {
   if (s != KS_OK) return s;
   KS_CUDA(ks::launch_fused_r1(maps, a, ks::r1_poly(), st), "fused R = 1 kernel launch");
   ctx->launches++;
-  if (a.dyn) {  // the dynamic tail's slot sums (inside the timed region: part of the evaluation)
-    KS_CUDA(ks::launch_r1_dyn_finish(a, st), "dynamic tail finish launch");
-    ctx->launches++;
-  }
   ctx->fused_launches++;
   ctx->last_grid = sk.grid;
   s = timed_end(ctx, stop);
@@ -818,6 +773,15 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
   if (s != KS_OK) return s;
   maps[2] = ctx->tmB_hi;
   maps[3] = ctx->tmB_lo;
+  if (ctx->r1) {  // the fold chunk of the R = 1 kernel's operands as 16-column, 32-byte-row planes
+    maps[4] = maps[0];
+    maps[5] = maps[2];
+    if (k_pad == 64) {
+      s = encode_2d_sw64(&maps[4], ctx->tgt_hi.p, k_pad, n_pad, ks::kTcTileT, true, true);
+      if (s != KS_OK) return s;
+      maps[5] = ctx->tmB_f;
+    }
+  }
   if (ctx->r1) return eval_r1(ctx, maps, N, V);
   if (ctx->rv) return eval_rv(ctx, maps, N, V);
 
@@ -934,11 +898,6 @@ ks_status reserve_targets(ks_ctx* ctx) {
   KS_CUDA(ctx->tgt_lo.reserve(ntg, st, false), "allocate target lo");
   KS_CUDA(ctx->nb.reserve((size_t)n_pad, st, false), "allocate target norms");
   KS_CUDA(ctx->tsc.reserve((size_t)n_pad, st, false), "allocate target scales");
-  if (ctx->r1) {
-    const int64_t n_t = n_pad / ks::kTcTileT;
-    const int64_t grid = std::min<int64_t>(ctx->num_sms, n_t * (ctx->m_pad / 128));
-    return reserve_dyn(ctx, r1_dyn_plan(ctx, n_t, grid), n_t);
-  }
   return KS_OK;
 }
 
@@ -1011,8 +970,6 @@ ks_status ks_destroy(ks_ctx* ctx) {
   ctx->wcol_part.release();
   ctx->stats_counter.release();
   ctx->coop_bar.release();
-  ctx->dyn_claim.release();
-  ctx->dyn_slots.release();
   ctx->partial.release();
   ctx->counters.release();
   ctx->dbg_times.release();
@@ -1288,7 +1245,8 @@ ks_status ks_get_info(const ks_ctx* ctx, ks_info* out) {
   out->tile_s = tc ? (ctx->r1 ? 128 : ctx->rv ? ks::kRvTileS : ks::fused_tc_tile_s(ctx->tc_vcc)) : ks::kTileS;
   out->num_ctas = ctx->last_grid;
   out->stages = !ctx->k_pad ? 0
-                : tc && ctx->r1 ? ks::fused_r1_stages(ctx->K)
+                : tc && ctx->r1 ? ks::fused_r1_stages(ctx->K, ctx->k_pad == 64 && ctx->K <= 32 &&
+                                                                 ctx->opts.v[KS_OPT_FOLD_NARROW] != 0)
                 : (tc ? ks::fused_tc_stages(ctx->tc_vcc, ctx->tc_f16 != 0, ctx->tc_f16 ? ctx->k_pad / 2 : ctx->k_pad,
                                             ctx->r_pad >= 32 ? 32 : 16)
                       : ks::fused_fp32_stages(ctx->k_pad));

@@ -71,8 +71,6 @@ constexpr int kR1Threads = 128 + 32 * kR1EpiWarps;
 constexpr int kR1TS = 128;                   // sources per unit
 constexpr uint32_t kR1Plane = 128u * 64u;    // 128 rows x one 64-byte chunk (8 KB); 4 KB with 32-byte rows
 constexpr int kR1WSlots = 8;                 // weight ring (weight mode)
-constexpr int kR1CRing = 4;                  // dynamic tail: ring of claimed chunk ids
-constexpr int kR1RingReaders = 3 + kR1EpiWarps;  // MMA warps 1, 3, warp 2, the epilogue warps
 constexpr int kR1MaxStages = 8;
 constexpr uint32_t kR1Smem = 227u * 1024u;   // dynamic shared memory requested
 constexpr uint32_t kR1Bars = 1024u;          // barriers + scratch flag at the top
@@ -186,6 +184,7 @@ template <int NPOLY, int CLAMP>
 __global__ void __launch_bounds__(kR1Threads, 1)
     ks_fused_r1_kernel(const __grid_constant__ CUtensorMap mA_hi, const __grid_constant__ CUtensorMap mA_lo,
                        const __grid_constant__ CUtensorMap mB_hi, const __grid_constant__ CUtensorMap mB_lo,
+                       const __grid_constant__ CUtensorMap mA_f, const __grid_constant__ CUtensorMap mB_f,
                        const R1Args args) {
   extern __shared__ __align__(1024) uint8_t smem[];
   if ((smem_u32(smem) & 1023u) != 0u) __trap();  // SWIZZLE_64B atoms and descriptors assume 1 KB alignment
@@ -216,7 +215,10 @@ __global__ void __launch_bounds__(kR1Threads, 1)
   const bool lo1 = n_kc == 2 && args.kdims > 32;
   const int P = 2 + (n_kc == 2 ? (lo1 ? 2 : 1) : 0);
   const uint32_t plane = narrow ? kR1Plane / 2 : kR1Plane;
-  const uint32_t tile_bytes = (uint32_t)P * plane;
+  // fold_narrow: the fold chunk is one 16-column plane of 32-byte rows (4 KB) after the two 8 KB
+  // planes of chunk 0
+  const bool fnar = args.fold_narrow != 0;
+  const uint32_t tile_bytes = fnar ? 2 * plane + kR1Plane / 2 : (uint32_t)P * plane;
   int D = (int)((kR1Region - 2 * tile_bytes) / tile_bytes);
   if (D > kR1MaxStages) D = kR1MaxStages;
   D &= ~1;  // even: the S-MMA warp of unit q (q & 1) also issues unit q + D, so it waits on every
@@ -233,19 +235,11 @@ __global__ void __launch_bounds__(kR1Threads, 1)
   uint64_t* sempty = sfull + kR1Groups;     // [4]
   uint64_t* wfull = sempty + kR1Groups;     // [8]
   uint64_t* wempty = wfull + kR1WSlots;     // [8]
-  uint64_t* cfull = wempty + kR1WSlots;     // [4] dynamic tail: chunk id published
-  uint64_t* cempty = cfull + kR1CRing;       // [4] ... read by every ring reader
-  volatile long long* ring = reinterpret_cast<volatile long long*>(cempty + kR1CRing);  // [4] chunk ids (-1: done)
-  uint32_t* tmem_base_smem = reinterpret_cast<uint32_t*>(const_cast<long long*>(ring) + kR1CRing);
+  uint32_t* tmem_base_smem = reinterpret_cast<uint32_t*>(wempty + kR1WSlots);
   int* flag = reinterpret_cast<int*>(tmem_base_smem + 1);
 
   R1Sched sc;
-  const bool dyn = args.dyn != 0;
-  // dynamic tail: the static schedule covers the whole-tile waves before dyn_t0 only
-  sc.init(dyn ? args.dyn_t0 : args.sk.n_t, args.sk.n_s, args.sk.grid, b);
-  const int64_t n_dyn = args.sk.n_t - args.dyn_t0;  // dynamically scheduled tiles
-  const int64_t n_chunks = dyn ? n_dyn * args.dyn_nc : 0;
-  const int dyn_c = args.dyn_c;
+  sc.init(args.sk.n_t, args.sk.n_s, args.sk.grid, b);
   const int count = sc.count;
   const int n_s = sc.n_s;
 
@@ -265,10 +259,6 @@ __global__ void __launch_bounds__(kR1Threads, 1)
     for (int i = 0; i < kR1WSlots; ++i) {
       mbar_init(&wfull[i], 1);
       mbar_init(&wempty[i], 4);
-    }
-    for (int i = 0; i < kR1CRing; ++i) {
-      mbar_init(&cfull[i], 1);
-      mbar_init(&cempty[i], kR1RingReaders);
     }
     fence_mbar_init();
   }
@@ -293,34 +283,40 @@ __global__ void __launch_bounds__(kR1Threads, 1)
     uint32_t ph = 0;
     int seg = -1;
     int64_t cur_tt = -1;
-    auto load_a = [&](int64_t tt) {  // new segment: target tile tt's planes into buffer seg & 1
-      ++seg;
-      const int ab = seg & 1;
-      mbar_wait_uniform(&aempty[ab], (uint32_t)(((seg >> 1) & 1) ^ 1));
-      if (leader) {
-        uint8_t* ap = smem + offA + ab * tile_bytes;
-        const int y = (int)(tt * 128);
-        mbar_arrive_expect_tx(&afull[ab], tile_bytes);
-        tma_load_2d(ap, &mA_hi, 0, y, &afull[ab]);
-        tma_load_2d(ap + plane, &mA_lo, 0, y, &afull[ab]);
-        if (n_kc == 2) {
-          tma_load_2d(ap + 2 * plane, &mA_hi, 32, y, &afull[ab]);
-          if (lo1) tma_load_2d(ap + 3 * plane, &mA_lo, 32, y, &afull[ab]);
+    R1It cu = r1_begin(sc);
+    for (int q = 0; q < count; ++q, r1_next(sc, cu)) {
+      if (cu.tt != cur_tt) {  // new target tile: its planes into buffer seg & 1
+        ++seg;
+        cur_tt = cu.tt;
+        const int ab = seg & 1;
+        mbar_wait_uniform(&aempty[ab], (uint32_t)(((seg >> 1) & 1) ^ 1));
+        if (leader) {
+          uint8_t* ap = smem + offA + ab * tile_bytes;
+          const int y = (int)(cu.tt * 128);
+          mbar_arrive_expect_tx(&afull[ab], tile_bytes);
+          tma_load_2d(ap, &mA_hi, 0, y, &afull[ab]);
+          tma_load_2d(ap + plane, &mA_lo, 0, y, &afull[ab]);
+          if (fnar) {
+            tma_load_2d(ap + 2 * plane, &mA_f, 32, y, &afull[ab]);
+          } else if (n_kc == 2) {
+            tma_load_2d(ap + 2 * plane, &mA_hi, 32, y, &afull[ab]);
+            if (lo1) tma_load_2d(ap + 3 * plane, &mA_lo, 32, y, &afull[ab]);
+          }
         }
+        __syncwarp();
       }
-      __syncwarp();
-    };
-    auto load_b = [&](int st) {  // source tile st into stage s
       mbar_wait_uniform(&empty[s], ph ^ 1u);
       if (leader && dbg_noload) {
         mbar_arrive(&full[s]);
       } else if (leader) {
         uint8_t* sp = smem + offS + s * tile_bytes;
-        const int y = st * kR1TS;
+        const int y = cu.st * kR1TS;
         mbar_arrive_expect_tx(&full[s], tile_bytes);
         tma_load_2d(sp, &mB_hi, 0, y, &full[s]);
         tma_load_2d(sp + plane, &mB_lo, 0, y, &full[s]);
-        if (n_kc == 2) {
+        if (fnar) {
+          tma_load_2d(sp + 2 * plane, &mB_f, 32, y, &full[s]);
+        } else if (n_kc == 2) {
           tma_load_2d(sp + 2 * plane, &mB_hi, 32, y, &full[s]);
           if (lo1) tma_load_2d(sp + 3 * plane, &mB_lo, 32, y, &full[s]);
         }
@@ -329,45 +325,6 @@ __global__ void __launch_bounds__(kR1Threads, 1)
       if (++s == D) {
         s = 0;
         ph ^= 1u;
-      }
-    };
-    R1It cu = r1_begin(sc);
-    for (int q = 0; q < count; ++q, r1_next(sc, cu)) {
-      if (cu.tt != cur_tt) {
-        cur_tt = cu.tt;
-        load_a(cu.tt);
-      }
-      load_b(cu.st);
-    }
-    if (dyn) {
-      // dynamic tail: claim chunk ids (one claim ahead: its latency overlaps the loads), publish
-      // each in the ring for the other roles, then load its target tile and its dyn_c source tiles;
-      // id -> tile dyn_t0 + id % n_dyn, chunk id / n_dyn (chunk-major: CTAs sweep the same sources)
-      int r = 0;
-      uint32_t rph = 0;
-      unsigned long long nxt = 0;
-      const int llane = __ffs(__ballot_sync(0xffffffffu, leader)) - 1;
-      if (leader) nxt = atomicAdd(args.claim, 1ull);
-      int64_t id = (int64_t)__shfl_sync(0xffffffffu, nxt, llane);
-      for (;;) {
-        const bool done = id >= n_chunks;
-        mbar_wait_uniform(&cempty[r], rph ^ 1u);
-        if (leader) {
-          ring[r] = done ? -1ll : (long long)id;
-          mbar_arrive(&cfull[r]);  // release: the id is visible to the readers' wait
-        }
-        __syncwarp();
-        if (++r == kR1CRing) {
-          r = 0;
-          rph ^= 1u;
-        }
-        if (done) break;
-        if (leader) nxt = atomicAdd(args.claim, 1ull);
-        const int64_t tt = args.dyn_t0 + id % n_dyn;
-        const int st0 = (int)(id / n_dyn) * dyn_c;
-        load_a(tt);
-        for (int u = 0; u < dyn_c; ++u) load_b(st0 + u);
-        id = (int64_t)__shfl_sync(0xffffffffu, nxt, llane);
       }
     }
   } else if (warp == 1 || warp == 3) {
@@ -388,6 +345,7 @@ __global__ void __launch_bounds__(kR1Threads, 1)
     }
     // descriptors: low words (start address >> 4) advance within the same high word
     const uint32_t dhi = (uint32_t)((narrow ? sdesc_k_sw32(smem) : sdesc_k_sw64(smem)) >> 32);
+    const uint32_t dhi1 = fnar ? (uint32_t)(sdesc_k_sw32(smem) >> 32) : dhi;  // chunk 1's layout
     const uint32_t dA0 = (uint32_t)sdesc_k_sw64(smem + offA), dS0 = (uint32_t)sdesc_k_sw64(smem + offS);
     const uint32_t kP16 = plane >> 4;
     const uint32_t tile16 = tile_bytes >> 4;
@@ -395,20 +353,21 @@ __global__ void __launch_bounds__(kR1Threads, 1)
     uint32_t ph = 0;
     int seg = -1;
     int64_t cur_tt = -1;
-    auto new_seg = [&]() {  // new target tile: release the previous buffer, wait for this one
-      if (seg >= 0) tc_commit_if(&aempty[seg & 1], lead);
-      ++seg;
-      mbar_wait_uniform(&afull[seg & 1], (uint32_t)((seg >> 1) & 1));
-    };
-    // one unit q (this warp's when q & 1 == mine; the other warp's only advance the stage counter)
-    auto unit = [&](int q) {
+    R1It cu = r1_begin(sc);
+    for (int q = 0; q < count; ++q, r1_next(sc, cu)) {
       const int bq = q & (kR1Groups - 1);
-      if ((q & 1) != mine) {
+      if (cu.tt != cur_tt) {  // new target tile: release the previous buffer, wait for this one
+        if (seg >= 0) tc_commit_if(&aempty[seg & 1], lead);
+        ++seg;
+        cur_tt = cu.tt;
+        mbar_wait_uniform(&afull[seg & 1], (uint32_t)((seg >> 1) & 1));
+      }
+      if ((q & 1) != mine) {  // the other warp's unit: only the stage counter advances
         if (++s == D) {
           s = 0;
           ph ^= 1u;
         }
-        return;
+        continue;
       }
       R1_PROF_BEGIN(w0);
       if (q >= kR1Groups) mbar_wait_uniform(&sempty[bq], (uint32_t)(((q >> 2) - 1) & 1));  // group bq read unit q - 4
@@ -437,7 +396,7 @@ __global__ void __launch_bounds__(kR1Threads, 1)
             mma_f16_lo(dS, aH + o, bL + o, dhi, idS, 1u, lead);
             mma_f16_lo(dS, aH + o, bH + o, dhi, idS, 1u, lead);
           } else if (np == 1u) {
-            mma_f16_lo(dS, aH + o, bH + o, dhi, idS, acc0, lead);
+            mma_f16_lo(dS, aH + o, bH + o, kc == 0 ? dhi : dhi1, idS, acc0, lead);
           }
         }
       }
@@ -449,67 +408,20 @@ __global__ void __launch_bounds__(kR1Threads, 1)
         s = 0;
         ph ^= 1u;
       }
-    };
-    int q = 0;
-    R1It cu = r1_begin(sc);
-    for (; q < count; ++q, r1_next(sc, cu)) {
-      if (cu.tt != cur_tt) {
-        cur_tt = cu.tt;
-        new_seg();
-      }
-      unit(q);
-    }
-    if (dyn) {  // dynamic tail: every chunk is a new segment of dyn_c units
-      int r = 0;
-      uint32_t rph = 0;
-      for (;;) {
-        mbar_wait_uniform(&cfull[r], rph);
-        const long long id = ring[r];
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&cempty[r]);
-        if (++r == kR1CRing) {
-          r = 0;
-          rph ^= 1u;
-        }
-        if (id < 0) break;
-        new_seg();
-        for (int u = 0; u < dyn_c; ++u, ++q) unit(q);
-      }
     }
   } else if (warp == 2) {
     // ================= weight-mode producer: the unit's 128 weights (512 B) into the ring
-    const bool leader = elect_one();
-    auto wload = [&](int q, int st) {
-      const int slot = q % kR1WSlots;
-      mbar_wait(&wempty[slot], (uint32_t)(((q / kR1WSlots) & 1) ^ 1));
-      if (leader) {
-        mbar_arrive_expect_tx(&wfull[slot], 512u);
-        bulk_load(wring + slot * 512, args.wv + (int64_t)st * kR1TS, 512u, &wfull[slot]);
-      }
-      __syncwarp();
-    };
-    int q = 0;
     if (!logw) {
+      const bool leader = elect_one();
       R1It cu = r1_begin(sc);
-      for (; q < count; ++q, r1_next(sc, cu)) wload(q, cu.st);
-    }
-    if (dyn) {  // dynamic tail: read every published chunk id (a ring reader in both modes)
-      int r = 0;
-      uint32_t rph = 0;
-      for (;;) {
-        mbar_wait(&cfull[r], rph);
-        const long long id = ring[r];
+      for (int q = 0; q < count; ++q, r1_next(sc, cu)) {
+        const int slot = q % kR1WSlots;
+        mbar_wait(&wempty[slot], (uint32_t)(((q / kR1WSlots) & 1) ^ 1));
+        if (leader) {
+          mbar_arrive_expect_tx(&wfull[slot], 512u);
+          bulk_load(wring + slot * 512, args.wv + (int64_t)cu.st * kR1TS, 512u, &wfull[slot]);
+        }
         __syncwarp();
-        if (lane == 0) mbar_arrive(&cempty[r]);
-        if (++r == kR1CRing) {
-          r = 0;
-          rph ^= 1u;
-        }
-        if (id < 0) break;
-        if (!logw) {
-          const int st0 = (int)(id / n_dyn) * dyn_c;
-          for (int u = 0; u < dyn_c; ++u, ++q) wload(q, st0 + u);
-        }
       }
     }
   } else if (warp >= 4) {
@@ -532,8 +444,22 @@ __global__ void __launch_bounds__(kR1Threads, 1)
       vlo += (vhi - (sum - bb)) + (blk - bb);
       vhi = sum;
     };
-    // this group's units of [q, q_end) (q % 4 == gr), each S buffer read then released
-    auto run_units = [&](int q, int q_end) {
+    // segments (runs of units of one target tile) computed once each, so the unit loop keeps
+    // only q and the segment end live
+    for (int q = 0; q < count;) {
+      int64_t tt;
+      int st0, len;
+      if (q < sc.qw) {
+        tt = b + (int64_t)(q / n_s) * sc.G;
+        st0 = 0;
+        len = n_s;
+      } else {
+        const int64_t v = sc.v0 + (q - sc.qw);
+        tt = sc.rem_t0 + v / n_s;
+        st0 = (int)(v % n_s);
+        len = n_s - st0 < count - q ? n_s - st0 : count - q;
+      }
+      const int q_end = q + len;
       for (int qq = q + ((gr - q) & (kR1Groups - 1)); qq < q_end; qq += kR1Groups) {
         R1_PROF_BEGIN(e0);
         mbar_wait(&sfull[gr], (uint32_t)((qq >> 2) & 1));
@@ -584,42 +510,18 @@ __global__ void __launch_bounds__(kR1Threads, 1)
         }
         R1_PROF_END(1, e1);
       }
-    };
-    // segment end, first half: the group's row sums into red, all four groups synchronised;
-    // returns (for the group 0 threads) the fixed-order sum of the four
-    auto seg_sum = [&]() -> double {
+      R1_PROF_BEGIN(e2);
+      // ---- segment end: the four groups' row sums in a fixed order, then V or a partial slot
       fold();
       nblk = 0;
+      const bool whole = (st0 == 0) && (len == n_s);
+      const int64_t grow = tt * 128 + row;
       const double wsc = logw ? (double)__uint_as_float(args.wstat[0]) : 1.0;
       red[gr * 128 + row] = ((double)vhi + (double)vlo) * wsc;
       vhi = vlo = 0.f;
       named_bar_sync(1, 32 * kR1EpiWarps);
-      return ((red[row] + red[128 + row]) + red[256 + row]) + red[384 + row];
-    };
-    // segments (runs of units of one target tile) computed once each, so the unit loop keeps
-    // only q and the segment end live
-    int q = 0;
-    while (q < count) {
-      int64_t tt;
-      int st0, len;
-      if (q < sc.qw) {
-        tt = b + (int64_t)(q / n_s) * sc.G;
-        st0 = 0;
-        len = n_s;
-      } else {
-        const int64_t v = sc.v0 + (q - sc.qw);
-        tt = sc.rem_t0 + v / n_s;
-        st0 = (int)(v % n_s);
-        len = n_s - st0 < count - q ? n_s - st0 : count - q;
-      }
-      const int q_end = q + len;
-      run_units(q, q_end);
-      R1_PROF_BEGIN(e2);
-      // ---- segment end: the four groups' row sums in a fixed order, then V or a partial slot
-      const bool whole = (st0 == 0) && (len == n_s);
-      const int64_t grow = tt * 128 + row;
-      const double v = seg_sum();
       if (gr == 0) {
+        const double v = ((red[row] + red[128 + row]) + red[256 + row]) + red[384 + row];
         if (whole) {
           if (grow < args.N) args.V[grow] = (float)v;
         } else {
@@ -653,38 +555,6 @@ __global__ void __launch_bounds__(kR1Threads, 1)
       R1_PROF_END(2, e2);
       q = q_end;
     }
-    if (dyn) {
-      // dynamic tail: each published chunk is a segment of dyn_c units; every group writes its
-      // row sums of the chunk to its own slot and moves on -- no barrier, fence or atomic on the
-      // way (a cross-group sync per chunk measured +10% cycles) -- and r1_dyn_finish_kernel sums
-      // a tile's slots in (chunk, group) order after the launch.  Units keep the CTA's running
-      // index q: every CTA enters the tail at q = (static units) with the same q % 4 and chunks
-      // are multiples of 4 units, so unit u of a chunk always lands in group (q0 + u) % 4 -- the
-      // slots do not depend on which CTA ran the chunk (bitwise reproducible V).
-      const double wsc = logw ? (double)__uint_as_float(args.wstat[0]) : 1.0;
-      int r = 0;
-      uint32_t rph = 0;
-      for (;;) {
-        mbar_wait(&cfull[r], rph);
-        const long long id = ring[r];
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&cempty[r]);
-        if (++r == kR1CRing) {
-          r = 0;
-          rph ^= 1u;
-        }
-        if (id < 0) break;
-        const int64_t tl = id % n_dyn;  // tile dyn_t0 + tl
-        const int ch = (int)(id / n_dyn);
-        run_units(q, q + dyn_c);
-        q += dyn_c;
-        fold();
-        nblk = 0;
-        args.cslots[((tl * args.dyn_nc + ch) * kR1Groups + gr) * 128 + row] =
-            (float)(((double)vhi + (double)vlo) * wsc);
-        vhi = vlo = 0.f;
-      }
-    }
   }
 
 #if KS_PROF
@@ -695,44 +565,13 @@ __global__ void __launch_bounds__(kR1Threads, 1)
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  pdl_trigger();  // the dynamic tail's finish kernel may launch (it waits for this grid to complete)
   if (warp == 2) tmem_dealloc(tbase, 512);
-  // dynamic tail: the last CTA to leave (every CTA has made its final claim) zeroes the counter,
-  // so any launch order, CUDA-graph replay included, finds them at zero
-  if (dyn && tid == 0 && atomicAdd(args.claim + 1, 1ull) == (unsigned long long)(args.sk.grid - 1)) {
-    args.claim[0] = 0ull;
-    args.claim[1] = 0ull;
-  }
   if (ct != nullptr && tid == 0) {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     ct[4 * b + 2] = t;
     ct[4 * b + 3] = (unsigned long long)clock64();
   }
-}
-
-// Dynamic tail, after the fused launch: V rows of the dynamically scheduled tiles = the sum of
-// their (chunk, group) slots, FP64: 8 lanes per row each sum every 8th slot in order, then a
-// fixed xor tree (the same bits whatever the schedule).  One block of 1,024 threads per tile.
-__global__ void __launch_bounds__(1024) r1_dyn_finish_kernel(const float* __restrict__ cslots, int nc, int64_t dyn_t0,
-                                                             int64_t N, float* __restrict__ V) {
-  pdl_wait();  // every chunk slot of the fused launch is written
-  const int64_t tl = blockIdx.x;
-  const int row = threadIdx.x >> 3, l = threadIdx.x & 7;
-  const float* p = cslots + tl * nc * kR1Groups * 128 + row;
-  double sum = 0.0;
-#pragma unroll 4
-  for (int k = l; k < nc * kR1Groups; k += 8) sum += (double)__ldcg(p + k * 128);
-#pragma unroll
-  for (int o = 4; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
-  const int64_t grow = (dyn_t0 + tl) * 128 + row;
-  if (l == 0 && grow < N) V[grow] = (float)sum;
-}
-
-cudaError_t launch_r1_dyn_finish(const R1Args& a, cudaStream_t st) {
-  const int64_t n_dyn = a.sk.n_t - a.dyn_t0;
-  return launch_pdl(r1_dyn_finish_kernel, (unsigned)n_dyn, 1024, 0, st, (const float*)a.cslots, a.dyn_nc, a.dyn_t0,
-                    a.N, a.V);
 }
 
 // exponential pairs of 16 on the FMA pipe (KS_OPT_EXP_POLY tuning option; default measured)
@@ -745,7 +584,8 @@ static cudaError_t launch_r1_t(const CUtensorMap* m, const R1Args& a, cudaStream
   cudaError_t e = smem_optin_once(attr_done, reinterpret_cast<const void*>(ks_fused_r1_kernel<NPOLY, CLAMP>),
                                   (int)kR1Smem);
   if (e != cudaSuccess) return e;
-  return launch_pdl(ks_fused_r1_kernel<NPOLY, CLAMP>, a.sk.grid, kR1Threads, kR1Smem, st, m[0], m[1], m[2], m[3], a);
+  return launch_pdl(ks_fused_r1_kernel<NPOLY, CLAMP>, a.sk.grid, kR1Threads, kR1Smem, st, m[0], m[1], m[2], m[3], m[4],
+                    m[5], a);
 }
 
 cudaError_t launch_fused_r1(const CUtensorMap* maps, const R1Args& a, int npoly, cudaStream_t st) {
@@ -768,10 +608,10 @@ cudaError_t launch_fused_r1(const CUtensorMap* maps, const R1Args& a, int npoly,
   }
 }
 
-int fused_r1_stages(int K) {
+int fused_r1_stages(int K, bool fold_narrow) {
   const int n_kc = K + 6 <= 32 ? 1 : 2;
   const int P = 2 + (n_kc == 2 ? (K > 32 ? 2 : 1) : 0);
-  const uint32_t tb = (uint32_t)P * (K + 6 <= 16 ? kR1Plane / 2 : kR1Plane);
+  const uint32_t tb = fold_narrow ? 2 * kR1Plane + kR1Plane / 2 : (uint32_t)P * (K + 6 <= 16 ? kR1Plane / 2 : kR1Plane);
   int d = (int)((kR1Region - 2 * tb) / tb);
   return d > kR1MaxStages ? kR1MaxStages : d;
 }

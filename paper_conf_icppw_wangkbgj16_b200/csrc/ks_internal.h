@@ -174,20 +174,13 @@ struct R1Args {
   unsigned long long* cta_times;  // debug: [grid][4] globaltimer, clock64 at CTA start; the same at the end
                                   // (KS_PROF builds: then [grid][20 warps][4] per-warp phase clocks)
   int dbg;                // KS_DEBUG builds only (KS_R1_DEBUG): 1 no epilogue math, 2 no MMAs, 3 neither, 4 + no source loads
-  // dynamic tail (dyn = 1): target tiles [dyn_t0, n_t) are split into chunks of dyn_c units (a
-  // multiple of 4 dividing n_s; dyn_nc chunks per tile) that CTAs claim from a global counter, so
-  // SMs at a higher clock take more of them; sk.n_t tiles before dyn_t0 (a multiple of the grid)
-  // stay static whole-tile waves.  Chunk partials go to cslots and the last chunk of a tile to
-  // arrive ... (see below): each epilogue group writes its row sums of a chunk to its own slot;
-  // launch_r1_dyn_finish sums a tile's slots in (chunk, group) order after the fused launch
-  // (bitwise deterministic whatever CTA ran which chunk).
-  int dyn, dyn_c, dyn_nc;
-  int64_t dyn_t0;
-  unsigned long long* claim;  // [2] {chunks claimed, CTAs departed}: zero on entry, left zero
-  float* cslots;              // [(n_t - dyn_t0) * dyn_nc][4 groups][128]
+  int fold_narrow;        // the second chunk holds only the folded norm pieces (K <= 32, K + 6 <= 48):
+                          // it is loaded as ONE 16-column plane with 32-byte rows (maps 4, 5,
+                          // SWIZZLE_32B) instead of a 64-byte chunk -- a sixth fewer operand bytes
 };
+// maps: A_hi, A_lo (targets), B_hi, B_lo (sources), A_fold, B_fold (the hi planes' columns 32..47
+// as 32-byte boxes; read only with fold_narrow)
 cudaError_t launch_fused_r1(const CUtensorMap* maps, const R1Args& a, int npoly, cudaStream_t st);
-cudaError_t launch_r1_dyn_finish(const R1Args& a, cudaStream_t st);
 
 // ---------------------------------------------------------------- R > 1 folded kernel (ks_fused_rv.cu)
 // Split-FP16, K + 6 <= 64, weights as the FP16 V-MMA's wcat (launch_prep_wcat); r_c = 16 or 32
@@ -207,7 +200,7 @@ struct RvArgs {
 };
 cudaError_t launch_fused_rv(const CUtensorMap* maps, const RvArgs& a, cudaStream_t st);
 int rv_poly_for(int opt_value);
-int fused_r1_stages(int K);
+int fused_r1_stages(int K, bool fold_narrow);
 int r1_poly();
 int r1_poly_for(int opt_value);  // the NPOLY the R = 1 kernel runs for a KS_OPT_EXP_POLY value
 

@@ -288,49 +288,16 @@ def test_cooperative_prep_graph_replay():
                 assert torch.equal(V, ref)
 
 
-@pytest.mark.parametrize("M,N,wkind", [(4096, 40077, "pos"), (10240, 65536, "pos"), (5000, 38000, "signed"),
-                                       (2048, 75000, "signed")])
-def test_dynamic_tail(oracle_mod, M, N, wkind):
-    """The R = 1 kernel's dynamic tail (option dyn_tail, off by default): with >= 2 whole waves of
-    target tiles, the last wave and the remainder are claimed in chunks by the CTAs.  Chunk
-    partials are summed per tile in chunk order, so the result is bitwise reproducible whatever
-    CTA ran which chunk; it matches the static stream-K schedule to rounding and meets the bar.
-    Shapes: 2 chunks of 16 units per tile, 5 chunks, chunks of 20 units (n_s = 40), and the
-    weight mode (signed W: the weight ring also follows the claimed chunks)."""
-    a, W, b, h = workloads.custom(M, N, 32, 1, 1.0, dist="gm", sigma=0.1, wkind=wkind, seed=M + N)
-    Vd = run(a, W, b, h, dyn_tail=1)
-    Vd2 = run(a, W, b, h, dyn_tail=1)
-    Vs = run(a, W, b, h, dyn_tail=0)
-    assert np.array_equal(Vd, Vd2)
-    assert np.max(np.abs(Vd - Vs)) / np.abs(W).sum() <= 1e-6
-    J = workloads.sample_targets(N, 300, seed=11)
-    Vr = oracle_mod.oracle_eval(a, W, b, float(h), J=J)
-    assert e_norm(Vd[J], Vr, W) <= TOL_3XTF32
-
-
-def test_dynamic_tail_graph_replay():
-    """The chunk-claim counter resets itself at the end of every launch: an eval captured in a
-    CUDA graph after ks_reserve replays correctly any number of times, between live evals."""
-    a, W, b, h = workloads.custom(4096, 40077, 32, 1, 1.0, dist="gm", sigma=0.1, wkind="pos", seed=3)
-    ta, tw, tb = (torch.from_numpy(x).cuda() for x in (a, W, b))
-    with ks.KernelSum(a.shape[1], float(h), "auto", options={"dyn_tail": 1}) as plan:
-        s = torch.cuda.Stream()
-        with torch.cuda.stream(s):
-            plan.set_sources(ta, tw)
-            ks.ks_reserve(plan.ctx, b.shape[0])
-            V = torch.empty((b.shape[0], 1), device="cuda")
-            plan.eval(tb, out=V)
-            s.synchronize()
-            ref = V.clone()
-            g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g, stream=s):
-                plan.eval(tb, out=V)
-            for _ in range(3):
-                V.zero_()
-                g.replay()
-                g.replay()
-                s.synchronize()
-                assert torch.equal(V, ref)
-                V2 = plan.eval(tb)
-                s.synchronize()
-                assert torch.equal(V2, ref)
+@pytest.mark.parametrize("K", [26, 27, 30, 32, 33, 42])
+def test_fold_narrow_plane(oracle_mod, K):
+    """At 27 <= K <= 32 the second operand chunk holds only the six folded norm columns: the R = 1
+    kernel loads it as one 16-column plane of 32-byte rows (SWIZZLE_32B TMA box over the same
+    array, its own MMA descriptor layout) instead of a 64-byte chunk.  The MMAs multiply the same
+    values in the same order, so V is bitwise the 64-byte layout's (option fold_narrow = 0); the
+    neighbouring K (26: fold inside chunk 0; 33, 42: coordinates in chunk 1) are unaffected."""
+    a, W, b, h = workloads.custom(3000, 1500, K, 1, 1.0, dist="gm", sigma=0.1, wkind="pos", seed=K)
+    V1 = run(a, W, b, h)
+    V0 = run(a, W, b, h, fold_narrow=0)
+    assert np.array_equal(V1, V0)
+    Vr = oracle_mod.oracle_eval(a, W, b, float(h))
+    assert e_norm(V1, Vr, W) <= TOL_3XTF32
