@@ -1618,8 +1618,19 @@ struct FoldLanes {
   __device__ static int col(int g, int c, int k) { return V * g + 8 * V * c + k; }
 };
 
+// The lane's columns of mu (zero past K), loaded once per thread (mu: global or shared memory).
 template <int CPL>
-__device__ __forceinline__ void fold_load_row(const float* __restrict__ row, const float* __restrict__ mu, int K,
+__device__ __forceinline__ void fold_lane_mu(const float* mu, int K, int g, float (&m)[CPL]) {
+  using L = FoldLanes<CPL>;
+#pragma unroll
+  for (int q = 0; q < CPL; ++q) {
+    const int d = L::col(g, q / L::V, q % L::V);
+    m[q] = d < K ? mu[d] : 0.f;
+  }
+}
+
+template <int CPL>
+__device__ __forceinline__ void fold_load_row(const float* __restrict__ row, const float (&m)[CPL], int K,
                                               bool live, int g, float (&x)[CPL]) {
   using L = FoldLanes<CPL>;
 #pragma unroll
@@ -1634,27 +1645,47 @@ __device__ __forceinline__ void fold_load_row(const float* __restrict__ row, con
         x[2 * c] = v.x, x[2 * c + 1] = v.y;
       }
 #pragma unroll
-      for (int k = 0; k < L::V; ++k) x[L::V * c + k] -= mu[d + k];  // FP32 centring, both sides alike
+      for (int k = 0; k < L::V; ++k) x[L::V * c + k] -= m[L::V * c + k];  // FP32 centring, both sides alike
     } else {
 #pragma unroll
-      for (int k = 0; k < L::V; ++k) x[L::V * c + k] = (live && d + k < K) ? row[d + k] - mu[d + k] : 0.f;
+      for (int k = 0; k < L::V; ++k) x[L::V * c + k] = (live && d + k < K) ? row[d + k] - m[L::V * c + k] : 0.f;
     }
   }
 }
 
-template <int CPL>
-__device__ __forceinline__ void fold_store_row(void* base, int64_t row_halves, int g, const __half (&h)[CPL]) {
+// x (the lane's columns, scaled, zero past K) -> hi / lo planes of one row: hi = RN_f16(x),
+// lo = RN_f16(x - hi) (x - hi is exact in FP32), two columns per packed conversion (the same
+// bits as split_f16 per element); columns d >= K take hi = fold_hi(d) (folded norm pieces,
+// their unit columns, zero padding) and lo = 0.  One vector store per chunk and plane.
+template <int CPL, typename FoldHi>
+__device__ __forceinline__ void fold_split_store(const float (&x)[CPL], int K, int g, void* __restrict__ hi_base,
+                                                 void* __restrict__ lo_base, int64_t row_halves, FoldHi fold_hi) {
   using L = FoldLanes<CPL>;
+  __half2 hi[CPL / 2], lo[CPL / 2];
+#pragma unroll
+  for (int p = 0; p < CPL / 2; ++p) {
+    hi[p] = __floats2half2_rn(x[2 * p], x[2 * p + 1]);
+    const float2 hf = __half22float2(hi[p]);
+    lo[p] = __floats2half2_rn(x[2 * p] - hf.x, x[2 * p + 1] - hf.y);
+    const int d0 = L::col(g, (2 * p) / L::V, (2 * p) % L::V);  // columns d0, d0 + 1 (V is even)
+    if (d0 + 1 >= K) {
+      if (d0 >= K) hi[p].x = fold_hi(d0);
+      hi[p].y = fold_hi(d0 + 1);
+    }
+  }
 #pragma unroll
   for (int c = 0; c < L::NCH; ++c) {
-    __half* dst = static_cast<__half*>(base) + row_halves + L::col(g, c, 0);
-    const __half2 v0 = __halves2half2(h[L::V * c], h[L::V * c + 1]);
+    const int64_t off = row_halves + L::col(g, c, 0);
+    __half* dh = static_cast<__half*>(hi_base) + off;
+    __half* dl = static_cast<__half*>(lo_base) + off;
     if constexpr (L::V == 4) {
-      const __half2 v1 = __halves2half2(h[L::V * c + 2], h[L::V * c + 3]);
-      *reinterpret_cast<uint2*>(dst) =
-          make_uint2(*reinterpret_cast<const uint32_t*>(&v0), *reinterpret_cast<const uint32_t*>(&v1));
+      *reinterpret_cast<uint2*>(dh) = make_uint2(*reinterpret_cast<const uint32_t*>(&hi[2 * c]),
+                                                 *reinterpret_cast<const uint32_t*>(&hi[2 * c + 1]));
+      *reinterpret_cast<uint2*>(dl) = make_uint2(*reinterpret_cast<const uint32_t*>(&lo[2 * c]),
+                                                 *reinterpret_cast<const uint32_t*>(&lo[2 * c + 1]));
     } else {
-      *reinterpret_cast<uint32_t*>(dst) = *reinterpret_cast<const uint32_t*>(&v0);
+      *reinterpret_cast<uint32_t*>(dh) = *reinterpret_cast<const uint32_t*>(&hi[c]);
+      *reinterpret_cast<uint32_t*>(dl) = *reinterpret_cast<const uint32_t*>(&lo[c]);
     }
   }
 }
@@ -1664,7 +1695,7 @@ __device__ __forceinline__ void fold_store_row(void* base, int64_t row_halves, i
 // shift fsh, scale exponent fexp, log2 max W) are evaluated once per block by the caller.
 template <int CPL>
 __device__ __forceinline__ void fold_source_row(const float* row, const float* wrow,
-                                                int64_t M, int K, int R, const float* mu, double c, bool logw,
+                                                int64_t M, int K, int R, const float (&m)[CPL], double c, bool logw,
                                                 int fsh, int fexp, double lwmax, int64_t i, int g,
                                                 void* __restrict__ src_hi, void* __restrict__ src_lo,
                                                 float* __restrict__ na, float* __restrict__ wv, int rv) {
@@ -1672,7 +1703,7 @@ __device__ __forceinline__ void fold_source_row(const float* row, const float* w
   constexpr int G = 8, KP = 8 * CPL;
   const bool live = i < M;
   float x[CPL];
-  fold_load_row<CPL>(row, mu, K, live, g, x);
+  fold_load_row<CPL>(row, m, K, live, g, x);
   double n = 0.0;
 #pragma unroll
   for (int k = 0; k < CPL; ++k) n += (double)x[k] * (double)x[k];
@@ -1694,19 +1725,12 @@ __device__ __forceinline__ void fold_source_row(const float* row, const float* w
     if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
     else split3_f16(nf, np);
   }
-  __half hi[CPL], lo[CPL];
+  float xs[CPL];
 #pragma unroll
-  for (int q = 0; q < CPL; ++q) {
-    const int d = L::col(g, q / L::V, q % L::V);
-    if (d < K) {
-      split_f16((float)(c2 * (double)x[q]) * sA, hi[q], lo[q]);  // exact power-of-2 scaling
-    } else {
-      hi[q] = d < K + 3 ? np[d - K] : d < K + 6 ? one : zero;  // folded norm columns: hi planes only
-      lo[q] = zero;
-    }
-  }
-  fold_store_row<CPL>(src_hi, i * KP, g, hi);
-  fold_store_row<CPL>(src_lo, i * KP, g, lo);
+  for (int q = 0; q < CPL; ++q) xs[q] = (float)(c2 * (double)x[q]) * sA;  // exact power-of-2 scaling; 0 past K
+  // folded norm columns: hi planes only
+  fold_split_store<CPL>(xs, K, g, src_hi, src_lo, i * KP,
+                        [&](int d) { return d < K + 3 ? np[d - K] : d < K + 6 ? one : zero; });
   if (g == 0) na[i] = 0.f;  // folded: the norm and log-weight ride in the contraction
   for (int r = g; r < rv; r += G) wv[i * rv + r] = logw ? (float)wl : (live && r < R) ? wrow[r] : 0.f;
 }
@@ -1731,7 +1755,9 @@ __global__ void __launch_bounds__(256) prep_fold_sources_kernel(
   const int64_t i = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
   if (i < m_pad) {
     const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && aug < 3;
-    fold_source_row<CPL>(alpha + i * K, W + i * R, M, K, R, mu, c, logw, s_fsh, s_fexp, s_lwmax, i, g, src_hi, src_lo, na, wv,
+    float m[CPL];
+    fold_lane_mu<CPL>(mu, K, g, m);
+    fold_source_row<CPL>(alpha + i * K, W + i * R, M, K, R, m, c, logw, s_fsh, s_fexp, s_lwmax, i, g, src_hi, src_lo, na, wv,
                          rv);
   }
   // PDL trigger last: a dependent fused kernel's CTA (640 threads, nearly all of an SM's registers)
@@ -1958,6 +1984,8 @@ __global__ void __launch_bounds__(kCoopThreads, 1) prep_fold_sources_coop_kernel
     const bool logw = s_logw;
     const double lwmax = s_lwmax;
     const int g = t & 7;
+    float m[CPL];
+    fold_lane_mu<CPL>(s_mu, K, g, m);
     // warp-uniform row base (the warp index through a shuffle: the compiler then knows the warp
     // is converged at group_sum's shuffles and emits plain SHFL, not WARPSYNC.COLLECTIVE loops)
     const int64_t wb = r0 + 4 * __shfl_sync(0xffffffffu, t >> 5, 0);
@@ -1965,7 +1993,7 @@ __global__ void __launch_bounds__(kCoopThreads, 1) prep_fold_sources_coop_kernel
       const int64_t i = base + ((t & 31) >> 3);
       const float* row = staged ? s_a + (i - r0) * K : alpha + i * K;
       const float* wrow = (staged && R == 1) ? s_wr + (i - r0) : W + i * R;
-      fold_source_row<CPL>(row, wrow, M, K, R, s_mu, c, logw, fsh, fexp, lwmax, i, g, src_hi, src_lo, na, wv, rv);
+      fold_source_row<CPL>(row, wrow, M, K, R, m, c, logw, fsh, fexp, lwmax, i, g, src_hi, src_lo, na, wv, rv);
     }
   }
   coop_grid_depart(bar, nb);
@@ -1988,48 +2016,65 @@ __global__ void __launch_bounds__(256) prep_fold_targets_kernel(const float* __r
   }
   __syncthreads();
   const int lane = threadIdx.x & 31, g = lane & (G - 1);
-  const int64_t j = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
-  if (j >= n_pad) return;
-  const bool live = j < N;
-  float x[CPL];
-  fold_load_row<CPL>(beta + j * K, mu, K, live, g, x);
-  double n = 0.0;
-#pragma unroll
-  for (int k = 0; k < CPL; ++k) n += (double)x[k] * (double)x[k];
-  n = group_sum<G>(n);
+  float m[CPL];
+  fold_lane_mu<CPL>(mu, K, g, m);  // once per thread; the warp then walks rows 4 at a time
   const int fsh = s_fsh;
   const float sB = ldexpf(1.f, -s_fexp);
   const __half one = __float2half(ldexpf(1.f, fsh)), zero = __float2half(0.f);
-  const bool far = c * n > ldexp(kFoldFar, fsh);  // row beyond every source: kernel row 0
+  const double far_lim = ldexp(kFoldFar, fsh);
   bool mine = false;  // this lane stores a folded norm piece (columns K + 3 .. K + 5)
 #pragma unroll
   for (int q = 0; q < CPL; ++q) {
     const int d = L::col(g, q / L::V, q % L::V);
     mine |= d >= K + 3 && d < K + 6;
   }
-  __half mp[3] = {zero, zero, zero};
-  if (far) mp[0] = __float2half(kFoldNegInf);
-  else if (mine) split3_f16(ldexp(-c * n, -fsh), mp);
-  __half hi[CPL], lo[CPL];
+  // warp-uniform row base (n_pad is a multiple of 128: a warp's four rows are all in range)
+  const int64_t w0 = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(0xffffffffu, threadIdx.x >> 5, 0);
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t base = 4 * w0; base < n_pad; base += 4 * nw) {
+    const int64_t j = base + lane / G;
+    const bool live = j < N;
+    float x[CPL];
+    fold_load_row<CPL>(beta + j * K, m, K, live, g, x);
+    double n = 0.0;
 #pragma unroll
-  for (int q = 0; q < CPL; ++q) {
-    const int d = L::col(g, q / L::V, q % L::V);
-    if (d < K) {
-      split_f16((far ? 0.f : x[q]) * sB, hi[q], lo[q]);
-    } else {
-      hi[q] = d < K + 3 ? one : d < K + 6 ? mp[d - K - 3] : zero;
-      lo[q] = zero;
+    for (int k = 0; k < CPL; ++k) n += (double)x[k] * (double)x[k];
+    n = group_sum<G>(n);
+    const bool far = c * n > far_lim;  // row beyond every source: kernel row 0
+    __half mp[3] = {zero, zero, zero};
+    if (far) mp[0] = __float2half(kFoldNegInf);
+    else if (mine) split3_f16(ldexp(-c * n, -fsh), mp);
+    float xs[CPL];
+#pragma unroll
+    for (int q = 0; q < CPL; ++q) xs[q] = far ? 0.f : x[q] * sB;  // 0 past K
+    fold_split_store<CPL>(xs, K, g, tgt_hi, tgt_lo, j * KP,
+                          [&](int d) { return d < K + 3 ? one : d < K + 6 ? mp[d - K - 3] : zero; });
+    if (g == 0) {
+      nb[j] = 0.f;
+      tsc[j] = 1.f;
     }
-  }
-  fold_store_row<CPL>(tgt_hi, j * KP, g, hi);
-  fold_store_row<CPL>(tgt_lo, j * KP, g, lo);
-  if (g == 0) {
-    nb[j] = 0.f;
-    tsc[j] = 1.f;
   }
   // PDL trigger last: a dependent fused kernel's CTA (640 threads, nearly all of an SM's registers)
   // launched early would hold its SM while waiting and starve this grid's remaining blocks
   pdl_trigger();
+}
+
+// SMs of the current device (cached per device ordinal; prep grids are sized by it)
+static int num_sms_current() {
+  static int cache[64] = {};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0) return 148;
+  if (dev >= 64) {
+    int v = 148;
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
+    return v;
+  }
+  if (cache[dev] == 0) {
+    int v = 148;
+    if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v <= 0) v = 148;
+    cache[dev] = v;
+  }
+  return cache[dev];
 }
 
 template <bool F16>
@@ -2073,7 +2118,11 @@ static cudaError_t launch_prep_targets(const float* beta, int64_t N, int64_t n_p
   const int bs = 256;
   if (F16 && aug >= 2 && K + 6 <= k_pad && (k_pad == 16 || k_pad == 32 || k_pad == 64) &&
       opt(KS_OPT_PREP_LANES, 0) == 0) {
-    const unsigned grid = (unsigned)((n_pad * 8 + bs - 1) / bs);
+    // warp-strided rows (mu and the fold constants loaded once per thread), at most 8 blocks per
+    // SM (measured at cfg3: 4 or 8 per SM let the fused kernel start 1.6 us earlier than one row
+    // quad per warp or 16 per SM)
+    unsigned grid = (unsigned)((n_pad * 8 + bs - 1) / bs);
+    if (grid > (unsigned)(8 * num_sms_current())) grid = (unsigned)(8 * num_sms_current());
 #define KS_PREP_F(cpl)                                                                                             \
   return launch_pdl(prep_fold_targets_kernel<cpl>, grid, bs, 0, st, beta, N, n_pad, K, mu, c, amax, tgt_hi, tgt_lo, nb, \
                     tsc)
