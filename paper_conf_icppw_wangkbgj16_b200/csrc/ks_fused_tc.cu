@@ -1,7 +1,9 @@
 // ks_fused_tc.cu -- the general fused tensor-core (tcgen05 / TMEM) kernel-summation kernel:
 // every (K, R) the dedicated R = 1 kernel (ks_fused_r1.cu: R = 1, split-FP16, K <= 58) does not
 // serve -- R > 1, K > 58, the TF32 modes, and R = 1 with KS_OPT_R1_KERNEL = 0 (scope rows a2-a7).
-// Also the prep kernels of the tensor-core path (a1 sources, a2 targets, FP16 weight split).
+// Also the prep kernels of the tensor-core path (a1 sources, a2 targets, FP16 weight split),
+// among them, for the folded layouts of the R = 1 and multi-column kernels, the statistics and
+// source prep in one cooperative launch (prep_fold_sources_coop_kernel).
 //
 // What it computes (PAPER.md SS III-C, Alg.2; Eq.3):
 //   S_ji = sum_d bh_jd * a_id           (a = 2c alpha_hat, bh = beta_hat; split operands)
