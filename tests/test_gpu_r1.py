@@ -288,14 +288,15 @@ def test_cooperative_prep_graph_replay():
                 assert torch.equal(V, ref)
 
 
+@pytest.mark.parametrize("wkind", ["pos", "signed"])
 @pytest.mark.parametrize("K", [26, 27, 30, 32, 33, 42])
-def test_fold_narrow_plane(oracle_mod, K):
+def test_fold_narrow_plane(oracle_mod, K, wkind):
     """At 27 <= K <= 32 the second operand chunk holds only the six folded norm columns: the R = 1
     kernel loads it as one 16-column plane of 32-byte rows (SWIZZLE_32B TMA box over the same
     array, its own MMA descriptor layout) instead of a 64-byte chunk.  The MMAs multiply the same
     values in the same order, so V is bitwise the 64-byte layout's (option fold_narrow = 0); the
     neighbouring K (26: fold inside chunk 0; 33, 42: coordinates in chunk 1) are unaffected."""
-    a, W, b, h = workloads.custom(3000, 1500, K, 1, 1.0, dist="gm", sigma=0.1, wkind="pos", seed=K)
+    a, W, b, h = workloads.custom(3000, 1500, K, 1, 1.0, dist="gm", sigma=0.1, wkind=wkind, seed=K)
     V1 = run(a, W, b, h)
     V0 = run(a, W, b, h, fold_narrow=0)
     assert np.array_equal(V1, V0)
