@@ -1334,23 +1334,19 @@ int prep_group(int K) {
 }
 
 template <bool F16, int G>
-__global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const float* __restrict__ W, int64_t M,
+__global__ void __launch_bounds__(256) prep_tc_sources_kernel(const float* __restrict__ alpha, const float* __restrict__ W, int64_t M,
                                        int64_t m_pad, int K, int k_pad, int R, int r_pad,
                                        const float* __restrict__ mu, double c, int aug,
                                        const unsigned* __restrict__ amax, void* __restrict__ src_hi,
                                        void* __restrict__ src_lo, float* __restrict__ na,
                                        float* __restrict__ wt_hi, float* __restrict__ wt_lo,
                                        float* __restrict__ wv, int rv, const unsigned* __restrict__ wstat) {
-  pdl_wait();  // the source statistics are complete (the trigger for the next grid is at the end)
-  // uniform values, once per block (FP64 log2 per thread made the kernel issue-bound)
-  __shared__ int s_fsh, s_fexp;
-  __shared__ double s_lwmax;
-  if (threadIdx.x == 0) {
-    s_fsh = (F16 && aug >= 2) ? f16_fold_shift(amax, c, K) : 0;
-    s_fexp = F16 ? f16_fold_exp(c) : 0;
-    s_lwmax = (wstat != nullptr && wstat[0] != 0u) ? log2((double)__uint_as_float(wstat[0])) : 0.0;
-  }
-  __syncthreads();
+  // the next kernel may launch early (a target / weight prep: small CTAs), and the per-thread
+  // uniform values (FP64 log2) overlap the row loads -- measured 15-17% faster than one
+  // computation per block behind a __syncthreads, or per warp (general-kernel shapes K = 64 ..
+  // 256, M = 262,144 .. 524,288; bitwise the same output)
+  pdl_trigger();
+  pdl_wait();  // the source statistics are complete
   const int lane = threadIdx.x & 31, gl = lane & (G - 1);
   const int64_t i = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
   if (i >= m_pad) return;
@@ -1365,35 +1361,27 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
   const float nai = live ? (float)(-c * n) : 0.f;
   const double c2 = 2.0 * c;
   // aug (FP16): 1 folded layout when f16_fold_ok, 2 always folded (fold shift), 3 the same
-  // without log-weights (the R = 1 kernel's weight mode and the multi-column kernel)
-  const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && !(F16 && aug >= 3);
-  // log2(W_i / Wmax) (R = 1, W >= 0; -inf for W_i = 0 and padding); FP64 log2, so only the
-  // lanes that store it evaluate it
-  auto wl_of = [&]() -> double { return !logw ? 0.0 : live ? log2((double)W[i]) - s_lwmax : -INFINITY; };
+  // without log-weights (the R = 1 kernel's weight mode)
+  const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && !(F16 && aug == 3);
+  // log2(W_i / Wmax) (R = 1, W >= 0; -inf for W_i = 0 and padding)
+  const double wl = !logw ? 0.0 : live ? log2((double)W[i]) - log2((double)__uint_as_float(wstat[0])) : -INFINITY;
   float sA = 1.f;
   bool fa = false;  // folded layout active
-  int fsh = 0;
   __half np[3] = {__float2half(0.f), __float2half(0.f), __float2half(0.f)};
-  bool np_ready = false;
   __half one = __float2half(1.f);  // unit columns (times the target's norm pieces): 2^s
   if constexpr (F16) {
     fa = aug >= 2 || (aug == 1 && f16_fold_ok(amax, c, K));
     if (fa) {
-      fsh = s_fsh;
+      const int fsh = aug >= 2 ? f16_fold_shift(amax, c, K) : 0;
       one = __float2half(ldexpf(1.f, fsh));
-      sA = ldexpf(1.f, s_fexp);
+      sA = ldexpf(1.f, f16_fold_exp(c));
+      const double nf = ldexp(-c * n + wl, -fsh);  // finite unless W_i = 0: then the FP16 stand-in for -inf
+      if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
+      else split3_f16(nf, np);
     } else {
       sA = ldexpf(1.f, f16_scale_exp((float)(c2 * (double)__uint_as_float(*amax))));
     }
   }
-  // the folded norm pieces, for the lanes that store columns K .. K + 2
-  auto need_np = [&]() {
-    if (np_ready) return;
-    np_ready = true;
-    const double nf = ldexp(-c * n + wl_of(), -fsh);  // finite unless W_i = 0: then the FP16 stand-in for -inf
-    if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
-    else split3_f16(nf, np);
-  };
   auto coord = [&](int d) -> float {
     if (d < K) {
       const float x = live ? alpha[i * K + d] - mu[d] : 0.f;
@@ -1409,7 +1397,6 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
       __half h0, l0, h1, l1;
       split_f16(a0 * sA, h0, l0);  // exact power-of-2 scaling
       split_f16(a1 * sA, h1, l1);
-      if (fa && d + 1 >= K && d < K + 3) need_np();
       if (fa && d >= K && d < K + 6) {  // folded norm columns: hi planes only
         h0 = d < K + 3 ? np[d - K] : one;
         l0 = __float2half(0.f);
@@ -1426,7 +1413,6 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
       static_cast<float2*>(src_lo)[(i * k_pad + d) >> 1] = make_float2(to_tf32(a0 - ah0), to_tf32(a1 - ah1));
     }
   }
-  const double wl = (gl == 0 && logw && !fa) || (gl == 0 && logw && rv > 0) ? wl_of() : 0.0;
   if (gl == 0) {
     if (fa) {
       na[i] = 0.f;  // folded: the norm and log-weight ride in the contraction
@@ -1449,27 +1435,19 @@ __global__ void prep_tc_sources_kernel(const float* __restrict__ alpha, const fl
     wt_hi[(int64_t)r * m_pad + i] = wh;
     wt_lo[(int64_t)r * m_pad + i] = to_tf32(w - wh);
   }
-  // PDL trigger last: a dependent fused kernel's CTA (640 threads, nearly all of an SM's registers)
-  // launched early would hold its SM while waiting and starve this grid's remaining blocks
-  pdl_trigger();
 }
 
 template <bool F16, int G>
-__global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N, int64_t n_pad, int K, int k_pad,
+__global__ void __launch_bounds__(256) prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N, int64_t n_pad, int K, int k_pad,
                                        const float* __restrict__ mu, double c, int aug,
                                        const unsigned* __restrict__ amax, void* __restrict__ tgt_hi,
                                        void* __restrict__ tgt_lo, float* __restrict__ nb,
                                        float* __restrict__ tsc) {
-  pdl_wait();  // the source statistics (mu, amax) are complete (trigger at the end)
-  __shared__ int s_fsh, s_fexp;  // uniform, once per block (FP64 log2)
-  if (threadIdx.x == 0) {
-    s_fsh = (F16 && aug >= 2) ? f16_fold_shift(amax, c, K) : 0;
-    s_fexp = F16 ? f16_fold_exp(c) : 0;
-  }
-  __syncthreads();
+  pdl_trigger();  // the fused kernel's CTAs may start their prologue (measured: earlier than at the end)
+  pdl_wait();     // the source statistics (mu, amax) are complete
   const int lane = threadIdx.x & 31, gl = lane & (G - 1);
   const int64_t j = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / G) + lane / G;
-  if (j >= n_pad) return;
+  if (j >= n_pad) return;  // whole warps (n_pad is a multiple of 128)
   const bool live = j < N;
   double n = 0.0;
   float bmax = 0.f;
@@ -1487,10 +1465,16 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
   __half one = __float2half(1.f);  // unit columns (times the source's norm pieces): 2^s
   if constexpr (F16) {
     fa = aug >= 2 || (aug == 1 && f16_fold_ok(amax, c, K));
-    if (fa) {
-      const int fsh = s_fsh;
+    if (fa) {  // warp-uniform; the FP64 log2 of the uniform values by lane 0 (see the source prep)
+      int fsh = 0, fexp = 0;
+      if (lane == 0) {
+        fsh = aug >= 2 ? f16_fold_shift(amax, c, K) : 0;
+        fexp = f16_fold_exp(c);
+      }
+      fsh = __shfl_sync(0xffffffffu, fsh, 0);
+      fexp = __shfl_sync(0xffffffffu, fexp, 0);
       one = __float2half(ldexpf(1.f, fsh));
-      sB = ldexpf(1.f, -s_fexp);
+      sB = ldexpf(1.f, -fexp);
       far = c * n > ldexp(kFoldFar, fsh);
       // the folded norm pieces, for the lanes that store columns K + 3 .. K + 5
       bool mine = false;
@@ -1538,9 +1522,6 @@ __global__ void prep_tc_targets_kernel(const float* __restrict__ beta, int64_t N
     nb[j] = (fa || (!F16 && aug)) ? 0.f : nbj;
     tsc[j] = rj;
   }
-  // PDL trigger last: a dependent fused kernel's CTA (640 threads, nearly all of an SM's registers)
-  // launched early would hold its SM while waiting and starve this grid's remaining blocks
-  pdl_trigger();
 }
 
 // FP16 V-MMA weights (reading Q27): per-column max |W_ir| (block partials, fixed-order

@@ -26,5 +26,14 @@ for K in (1, 4, 8, 10, 16, 26, 27, 32, 40, 58):
                 V = plan.eval(torch.from_numpy(b).cuda())
                 torch.cuda.synchronize()
                 out[f"K{K}_R{R}_{wk}_coop{coop}"] = V.cpu().numpy()
+# the general kernel's prep paths (K > 58; R = 1 log-weights, signed W, R = 16; TF32 modes)
+for K, R, wk, prec in ((64, 1, "pos", "auto"), (100, 1, "signed", "auto"), (128, 16, "signed", "auto"),
+                       (40, 1, "pos", "3xtf32"), (300, 2, "signed", "auto")):
+    a, W, b, h = workloads.custom(2500, 1700, K, R, 2.0, dist="uniform", wkind=wk, seed=K + R)
+    with ks.KernelSum(K, float(h), prec) as plan:
+        plan.set_sources(torch.from_numpy(a).cuda(), torch.from_numpy(W).cuda())
+        V = plan.eval(torch.from_numpy(b).cuda())
+        torch.cuda.synchronize()
+        out[f"gen_K{K}_R{R}_{wk}_{prec}"] = V.cpu().numpy()
 np.savez(sys.argv[2], **out)
 print("saved", len(out))

@@ -2,7 +2,7 @@
 activity trace (torch.profiler / CUPTI): each kernel's start offset from the step's first kernel
 and its duration, so the gaps between launches and the time outside the fused kernel show.
 A measurement tool, not the bench contract (numbers under a tracer are never bench values).
-Usage: tools/step_timeline.py [CFG] [STEPS]"""
+Usage: tools/step_timeline.py [CFG] [STEPS]  |  tools/step_timeline.py custom M N K h [STEPS]"""
 import sys
 
 import torch
@@ -12,9 +12,14 @@ sys.path.insert(0, ".")
 import workloads  # noqa: E402
 import paper_conf_icppw_wangkbgj16_b200 as ks  # noqa: E402
 
-cfg = int(sys.argv[1]) if len(sys.argv) > 1 else 3
-steps = int(sys.argv[2]) if len(sys.argv) > 2 else 3
-a, W, b, h = workloads.make(cfg, wkind="pos")
+if len(sys.argv) > 1 and sys.argv[1] == "custom":  # custom M N K h [steps]: uniform points, W ~ U[0,1]
+    M, N, K, hh = int(sys.argv[2]), int(sys.argv[3]), int(sys.argv[4]), float(sys.argv[5])
+    steps = int(sys.argv[6]) if len(sys.argv) > 6 else 3
+    a, W, b, h = workloads.custom(M, N, K, 1, hh, seed=K)
+else:
+    cfg = int(sys.argv[1]) if len(sys.argv) > 1 else 3
+    steps = int(sys.argv[2]) if len(sys.argv) > 2 else 3
+    a, W, b, h = workloads.make(cfg, wkind="pos")
 plan = ks.KernelSum(a.shape[1], float(h))
 da, dw, db = (torch.from_numpy(x).cuda() for x in (a, W, b))
 V = torch.empty((b.shape[0], W.shape[1]), device="cuda")
