@@ -514,8 +514,8 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   const bool want_wstat = use_wstat || r1;  // the R = 1 kernel decides its epilogue from wstat
   // folded layouts (the R = 1 and multi-column kernels): statistics and source prep in one
   // cooperative launch (KS_OPT_COOP_PREP = 0: the separate statistics and prep kernels)
-  const bool coop = f16 && fold >= 2 && K + 6 <= k_pad && (k_pad == 16 || k_pad == 32 || k_pad == 64) &&
-                    ks::opt(KS_OPT_PREP_LANES, 0) == 0 && ks::opt(KS_OPT_COOP_PREP, 1) != 0;
+  bool coop = f16 && fold >= 2 && K + 6 <= k_pad && (k_pad == 16 || k_pad == 32 || k_pad == 64) &&
+              ks::opt(KS_OPT_PREP_LANES, 0) == 0 && ks::opt(KS_OPT_COOP_PREP, 1) != 0;
   if (coop) {
     const int grid = ks::coop_prep_grid(k_pad, m_pad, ctx->num_sms);
     KS_CUDA(ctx->mean_part.reserve((size_t)grid * K, st, false), "allocate statistics partials");
@@ -525,14 +525,18 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
     KS_CUDA(ctx->stats_counter.reserve(1, st, true), "allocate statistics counter");  // the W column prep
     KS_CUDA(ctx->amax.reserve(1, st, false), "allocate amax");
     if (want_wstat) KS_CUDA(ctx->wstat.reserve(2, st, false), "allocate weight statistics");
-    KS_CUDA(ks::launch_prep_fold_sources_coop(alpha, W, M, m_pad, K, k_pad, R, ctx->c, fold, grid,
-                                              ctx->mean_part.p, ctx->mean_pmm.p, ctx->mean_pw.p, ctx->coop_bar.p,
-                                              ctx->mu.p, ctx->amax.p, want_wstat ? ctx->wstat.p : nullptr,
-                                              ctx->src_hi.p, ctx->src_lo.p, ctx->na.p, ctx->wv.p, vcc, st),
-            "statistics + source prep (cooperative, folded)");
-  } else {
-    KS_CUDA(source_stats(ctx, alpha, W, want_wstat, M, k_pad, f16), "source statistics");
+    const cudaError_t ce = ks::launch_prep_fold_sources_coop(
+        alpha, W, M, m_pad, K, k_pad, R, ctx->c, fold, grid, ctx->mean_part.p, ctx->mean_pmm.p, ctx->mean_pw.p,
+        ctx->coop_bar.p, ctx->mu.p, ctx->amax.p, want_wstat ? ctx->wstat.p : nullptr, ctx->src_hi.p, ctx->src_lo.p,
+        ctx->na.p, ctx->wv.p, vcc, st);
+    if (ce == cudaErrorCooperativeLaunchTooLarge) {  // fewer SMs than the device reports (MPS, partitions):
+      (void)cudaGetLastError();                       // the separate statistics and prep kernels instead
+      coop = false;
+    } else {
+      KS_CUDA(ce, "statistics + source prep (cooperative, folded)");
+    }
   }
+  if (!coop) KS_CUDA(source_stats(ctx, alpha, W, want_wstat, M, k_pad, f16), "source statistics");
   const unsigned* wst = want_wstat ? ctx->wstat.p : nullptr;
   if (f16) {
     if (!coop) {
