@@ -184,9 +184,10 @@ typedef enum {
   KS_OPT_COOP_PREP = 18,      /* KS_COOP_PREP: folded layouts (R = 1 and multi-column kernels):
                                  1 (default) source statistics and prep in one cooperative
                                  launch, 0 the separate kernels [sources] */
-  KS_OPT_FOLD_NARROW = 19,    /* KS_FOLD_NARROW: R = 1 kernel, 27 <= K <= 32: 1 (default) the
-                                 folded norm pieces load as one 16-column plane of 32-byte rows,
-                                 0 as a second 64-byte chunk [eval] */
+  KS_OPT_NARROW_PLANES = 19,  /* KS_NARROW_PLANES: R = 1 kernel: 1 (default) operand planes with
+                                 only 16 used columns load as 32-byte rows -- the folded norm
+                                 pieces at 27 <= K <= 32, the lo plane at 11 <= K <= 16 -- 0 as
+                                 64-byte chunks [eval] */
   KS_OPT_COUNT_ = 20
 } ks_option;
 

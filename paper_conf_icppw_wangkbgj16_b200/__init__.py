@@ -40,7 +40,7 @@ OPTIONS = {"r1_kernel": 1, "r1_epilogue": 2, "exp_poly": 3, "weighted_sum": 4, "
            "aug": 7, "clamp": 8, "target_resident": 9, "stages": 10, "ar_stages": 11, "wslots": 12,
            "prep_lanes": 13, "eval_chunks": 14, "fp32_split": 15, "measure_clock": 16,
            "eval_chunk0": 17, "coop_prep": 18,
-           "fold_narrow": 19}
+           "narrow_planes": 19}
 
 
 class KsInfo(ctypes.Structure):

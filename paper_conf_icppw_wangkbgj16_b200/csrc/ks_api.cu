@@ -146,7 +146,8 @@ struct ks_ctx {
   int rv = 0;      // R > 1 folded kernel (ks_fused_rv.cu)
   int r1_clamp = 0;
   CUtensorMap tmB_hi, tmB_lo;
-  CUtensorMap tmB_f;  // R = 1 fold_narrow: columns 32..47 of the source hi plane, 32-byte boxes
+  CUtensorMap tmB_f;  // R = 1 narrow planes: the source hi plane's columns 32..47 (fold_narrow) or the lo
+                      // plane's columns 0..15 (lo_narrow) as 32-byte boxes
   DBuf<float> mu;         // [k_pad]
   DBuf<double> mean_part; // [nparts][K]
   DBuf<float> mean_pmm;   // [nparts][K][2] column min/max
@@ -219,7 +220,7 @@ const OptSpec kOpt[KS_OPT_COUNT_] = {
     {"KS_MEASURE_CLOCK", 0, 0, 1},
     {"KS_EVAL_CHUNK0", 0, -1, 1 << 20},
     {"KS_COOP_PREP", 1, 0, 1},
-    {"KS_FOLD_NARROW", 1, 0, 1},
+    {"KS_NARROW_PLANES", 1, 0, 1},
 };
 
 void init_opts(ks_ctx* ctx) {
@@ -570,6 +571,9 @@ ks_status prepare_tc(ks_ctx* ctx, const float* alpha, const float* W, int64_t M,
   if (r1 && k_pad == 64) {  // the fold chunk as one 16-column plane (fold_narrow, eval_r1)
     s = encode_2d_sw64(&ctx->tmB_f, ctx->src_hi.p, k_pad, m_pad, box_s, true, true);
     if (s != KS_OK) return s;
+  } else if (r1 && k_pad == 32 && K <= 16) {  // the lo plane as 16 columns (lo_narrow, eval_r1)
+    s = encode_2d_sw64(&ctx->tmB_f, ctx->src_lo.p, k_pad, m_pad, box_s, true, true);
+    if (s != KS_OK) return s;
   }
   ctx->k_pad = k_pad;
   ctx->m_pad = m_pad;
@@ -602,7 +606,9 @@ ks_status eval_r1(ks_ctx* ctx, const CUtensorMap* maps, int64_t N, float* V) {
   ks::R1Args a;
   // the second operand chunk holds only the folded norm pieces: load it as one 16-column plane
   a.fold_narrow = (ctx->k_pad == 64 && ctx->tc_kdims <= 32 && ctx->tc_kcols <= 48 &&
-                   ctx->opts.v[KS_OPT_FOLD_NARROW] != 0) ? 1 : 0;
+                   ctx->opts.v[KS_OPT_NARROW_PLANES] != 0) ? 1 : 0;
+  // one chunk with coordinates only in its first 16 columns: the lo plane as 16 columns
+  a.lo_narrow = (ctx->k_pad == 32 && ctx->tc_kdims <= 16 && ctx->opts.v[KS_OPT_NARROW_PLANES] != 0) ? 1 : 0;
   a.N = N;
   a.narrow = ctx->k_pad == ks::kTcKC ? 1 : 0;
   a.n_kc = a.narrow ? 1 : ctx->k_pad / 32;
@@ -782,6 +788,10 @@ ks_status eval_tc(ks_ctx* ctx, const float* beta, int64_t N, float* V) {
     maps[5] = maps[2];
     if (k_pad == 64) {
       s = encode_2d_sw64(&maps[4], ctx->tgt_hi.p, k_pad, n_pad, ks::kTcTileT, true, true);
+      if (s != KS_OK) return s;
+      maps[5] = ctx->tmB_f;
+    } else if (k_pad == 32 && ctx->K <= 16) {
+      s = encode_2d_sw64(&maps[4], ctx->tgt_lo.p, k_pad, n_pad, ks::kTcTileT, true, true);
       if (s != KS_OK) return s;
       maps[5] = ctx->tmB_f;
     }
@@ -1249,8 +1259,7 @@ ks_status ks_get_info(const ks_ctx* ctx, ks_info* out) {
   out->tile_s = tc ? (ctx->r1 ? 128 : ctx->rv ? ks::kRvTileS : ks::fused_tc_tile_s(ctx->tc_vcc)) : ks::kTileS;
   out->num_ctas = ctx->last_grid;
   out->stages = !ctx->k_pad ? 0
-                : tc && ctx->r1 ? ks::fused_r1_stages(ctx->K, ctx->k_pad == 64 && ctx->K <= 32 &&
-                                                                 ctx->opts.v[KS_OPT_FOLD_NARROW] != 0)
+                : tc && ctx->r1 ? ks::fused_r1_stages(ctx->K, ctx->opts.v[KS_OPT_NARROW_PLANES] != 0)
                 : (tc ? ks::fused_tc_stages(ctx->tc_vcc, ctx->tc_f16 != 0, ctx->tc_f16 ? ctx->k_pad / 2 : ctx->k_pad,
                                             ctx->r_pad >= 32 ? 32 : 16)
                       : ks::fused_fp32_stages(ctx->k_pad));

@@ -218,7 +218,9 @@ __global__ void __launch_bounds__(kR1Threads, 1)
   // fold_narrow: the fold chunk is one 16-column plane of 32-byte rows (4 KB) after the two 8 KB
   // planes of chunk 0
   const bool fnar = args.fold_narrow != 0;
-  const uint32_t tile_bytes = fnar ? 2 * plane + kR1Plane / 2 : (uint32_t)P * plane;
+  // lo_narrow: one chunk, the lo plane as 16 columns of 32-byte rows (4 KB) after the 8 KB hi plane
+  const bool lnar = args.lo_narrow != 0;
+  const uint32_t tile_bytes = fnar ? 2 * plane + kR1Plane / 2 : lnar ? plane + kR1Plane / 2 : (uint32_t)P * plane;
   int D = (int)((kR1Region - 2 * tile_bytes) / tile_bytes);
   if (D > kR1MaxStages) D = kR1MaxStages;
   D &= ~1;  // even: the S-MMA warp of unit q (q & 1) also issues unit q + D, so it waits on every
@@ -295,7 +297,7 @@ __global__ void __launch_bounds__(kR1Threads, 1)
           const int y = (int)(cu.tt * 128);
           mbar_arrive_expect_tx(&afull[ab], tile_bytes);
           tma_load_2d(ap, &mA_hi, 0, y, &afull[ab]);
-          tma_load_2d(ap + plane, &mA_lo, 0, y, &afull[ab]);
+          tma_load_2d(ap + plane, lnar ? &mA_f : &mA_lo, 0, y, &afull[ab]);
           if (fnar) {
             tma_load_2d(ap + 2 * plane, &mA_f, 32, y, &afull[ab]);
           } else if (n_kc == 2) {
@@ -313,7 +315,7 @@ __global__ void __launch_bounds__(kR1Threads, 1)
         const int y = cu.st * kR1TS;
         mbar_arrive_expect_tx(&full[s], tile_bytes);
         tma_load_2d(sp, &mB_hi, 0, y, &full[s]);
-        tma_load_2d(sp + plane, &mB_lo, 0, y, &full[s]);
+        tma_load_2d(sp + plane, lnar ? &mB_f : &mB_lo, 0, y, &full[s]);
         if (fnar) {
           tma_load_2d(sp + 2 * plane, &mB_f, 32, y, &full[s]);
         } else if (n_kc == 2) {
@@ -346,6 +348,7 @@ __global__ void __launch_bounds__(kR1Threads, 1)
     // descriptors: low words (start address >> 4) advance within the same high word
     const uint32_t dhi = (uint32_t)((narrow ? sdesc_k_sw32(smem) : sdesc_k_sw64(smem)) >> 32);
     const uint32_t dhi1 = fnar ? (uint32_t)(sdesc_k_sw32(smem) >> 32) : dhi;  // chunk 1's layout
+    const uint32_t dhiL = lnar ? (uint32_t)(sdesc_k_sw32(smem) >> 32) : dhi;  // the lo plane's layout
     const uint32_t dA0 = (uint32_t)sdesc_k_sw64(smem + offA), dS0 = (uint32_t)sdesc_k_sw64(smem + offS);
     const uint32_t kP16 = plane >> 4;
     const uint32_t tile16 = tile_bytes >> 4;
@@ -392,8 +395,13 @@ __global__ void __launch_bounds__(kR1Threads, 1)
           const uint32_t acc0 = (kc > 0 || ks > 0) ? 1u : 0u;
           if (dbg_nomma) {
           } else if (np == 3u) {  // small terms first
-            mma_f16_lo(dS, aL + o, bH + o, dhi, idS, acc0, lead);
-            mma_f16_lo(dS, aH + o, bL + o, dhi, idS, 1u, lead);
+            if (lnar) {  // lo planes in the 32-byte-row layout (ks = 0 only: columns 0..15)
+              mma_f16_lo2(dS, aL, dhiL, bH, dhi, idS, acc0, lead);
+              mma_f16_lo2(dS, aH, dhi, bL, dhiL, idS, 1u, lead);
+            } else {
+              mma_f16_lo(dS, aL + o, bH + o, dhi, idS, acc0, lead);
+              mma_f16_lo(dS, aH + o, bL + o, dhi, idS, 1u, lead);
+            }
             mma_f16_lo(dS, aH + o, bH + o, dhi, idS, 1u, lead);
           } else if (np == 1u) {
             mma_f16_lo(dS, aH + o, bH + o, kc == 0 ? dhi : dhi1, idS, acc0, lead);
@@ -608,10 +616,13 @@ cudaError_t launch_fused_r1(const CUtensorMap* maps, const R1Args& a, int npoly,
   }
 }
 
-int fused_r1_stages(int K, bool fold_narrow) {
+int fused_r1_stages(int K, bool narrow_planes) {
   const int n_kc = K + 6 <= 32 ? 1 : 2;
   const int P = 2 + (n_kc == 2 ? (K > 32 ? 2 : 1) : 0);
-  const uint32_t tb = fold_narrow ? 2 * kR1Plane + kR1Plane / 2 : (uint32_t)P * (K + 6 <= 16 ? kR1Plane / 2 : kR1Plane);
+  const bool fnar = narrow_planes && K + 6 > 32 && K <= 32, lnar = narrow_planes && K + 6 > 16 && K <= 16;
+  const uint32_t tb = fnar ? 2 * kR1Plane + kR1Plane / 2
+                      : lnar ? kR1Plane + kR1Plane / 2
+                             : (uint32_t)P * (K + 6 <= 16 ? kR1Plane / 2 : kR1Plane);
   int d = (int)((kR1Region - 2 * tb) / tb);
   return d > kR1MaxStages ? kR1MaxStages : d;
 }

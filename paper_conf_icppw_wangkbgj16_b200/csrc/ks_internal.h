@@ -177,9 +177,12 @@ struct R1Args {
   int fold_narrow;        // the second chunk holds only the folded norm pieces (K <= 32, K + 6 <= 48):
                           // it is loaded as ONE 16-column plane with 32-byte rows (maps 4, 5,
                           // SWIZZLE_32B) instead of a 64-byte chunk -- a sixth fewer operand bytes
+  int lo_narrow;          // one chunk, K <= 16 < K + 6: the lo plane's columns 16..31 are never
+                          // multiplied -- it loads as a 16-column plane of 32-byte rows (maps 4, 5
+                          // over the lo arrays), a quarter fewer operand bytes
 };
-// maps: A_hi, A_lo (targets), B_hi, B_lo (sources), A_fold, B_fold (the hi planes' columns 32..47
-// as 32-byte boxes; read only with fold_narrow)
+// maps: A_hi, A_lo (targets), B_hi, B_lo (sources), then 32-byte-row boxes read only with
+// fold_narrow (the hi planes' columns 32..47) or lo_narrow (the lo planes' columns 0..15)
 cudaError_t launch_fused_r1(const CUtensorMap* maps, const R1Args& a, int npoly, cudaStream_t st);
 
 // ---------------------------------------------------------------- R > 1 folded kernel (ks_fused_rv.cu)
@@ -200,7 +203,7 @@ struct RvArgs {
 };
 cudaError_t launch_fused_rv(const CUtensorMap* maps, const RvArgs& a, cudaStream_t st);
 int rv_poly_for(int opt_value);
-int fused_r1_stages(int K, bool fold_narrow);
+int fused_r1_stages(int K, bool narrow_planes);
 int r1_poly();
 int r1_poly_for(int opt_value);  // the NPOLY the R = 1 kernel runs for a KS_OPT_EXP_POLY value
 

@@ -288,6 +288,19 @@ __device__ __forceinline__ void mma_f16_lo(uint32_t d_tmem, uint32_t a_lo, uint3
       "r"(a_lo), "r"(b_lo), "r"(idesc), "r"(accumulate), "r"(desc_hi), "r"(issue)
       : "memory");
 }
+// The same with separate descriptor high words for A and B (operands in different layouts).
+__device__ __forceinline__ void mma_f16_lo2(uint32_t d_tmem, uint32_t a_lo, uint32_t a_hi, uint32_t b_lo,
+                                            uint32_t b_hi, uint32_t idesc, uint32_t accumulate, uint32_t issue) {
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t.reg .b64 da, db;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "setp.ne.b32 q, %7, 0;\n\t"
+      "mov.b64 da, {%1, %5};\n\t"
+      "mov.b64 db, {%2, %6};\n\t"
+      "@q tcgen05.mma.cta_group::1.kind::f16 [%0], da, db, %3, p;\n\t}" ::"r"(d_tmem),
+      "r"(a_lo), "r"(b_lo), "r"(idesc), "r"(accumulate), "r"(a_hi), "r"(b_hi), "r"(issue)
+      : "memory");
+}
 __device__ __forceinline__ void tc_commit_if(uint64_t* bar, uint32_t issue) {
   asm volatile(
       "{\n\t.reg .pred q;\n\t"

@@ -289,16 +289,18 @@ def test_cooperative_prep_graph_replay():
 
 
 @pytest.mark.parametrize("wkind", ["pos", "signed"])
-@pytest.mark.parametrize("K", [26, 27, 30, 32, 33, 42])
-def test_fold_narrow_plane(oracle_mod, K, wkind):
-    """At 27 <= K <= 32 the second operand chunk holds only the six folded norm columns: the R = 1
-    kernel loads it as one 16-column plane of 32-byte rows (SWIZZLE_32B TMA box over the same
-    array, its own MMA descriptor layout) instead of a 64-byte chunk.  The MMAs multiply the same
-    values in the same order, so V is bitwise the 64-byte layout's (option fold_narrow = 0); the
-    neighbouring K (26: fold inside chunk 0; 33, 42: coordinates in chunk 1) are unaffected."""
+@pytest.mark.parametrize("K", [10, 11, 13, 16, 17, 26, 27, 30, 32, 33, 42])
+def test_narrow_planes(oracle_mod, K, wkind):
+    """Operand planes with only 16 used columns load as 32-byte rows (SWIZZLE_32B TMA box over the
+    same array, their own MMA descriptor layout) instead of 64-byte chunks: at 27 <= K <= 32 the
+    second chunk (the six folded norm columns), at 11 <= K <= 16 the lo plane (coordinates in its
+    first 16 columns only; the lo.hi / hi.lo MMAs then mix the two layouts).  The MMAs multiply
+    the same values in the same order, so V is bitwise the 64-byte layout's (option
+    narrow_planes = 0); the neighbouring K (10: 32-byte rows throughout; 17, 26: fold inside chunk
+    0; 33, 42: coordinates in chunk 1) are unaffected."""
     a, W, b, h = workloads.custom(3000, 1500, K, 1, 1.0, dist="gm", sigma=0.1, wkind=wkind, seed=K)
     V1 = run(a, W, b, h)
-    V0 = run(a, W, b, h, fold_narrow=0)
+    V0 = run(a, W, b, h, narrow_planes=0)
     assert np.array_equal(V1, V0)
     Vr = oracle_mod.oracle_eval(a, W, b, float(h))
     assert e_norm(V1, Vr, W) <= TOL_3XTF32
