@@ -138,9 +138,14 @@ KS_API ks_status ks_eval(ks_ctx *ctx, const float *beta, int64_t N, float *V);
  * returns once alpha and W have been copied (the caller may reuse them); the
  * source preparation then runs on the context's stream.  ks_eval_host uploads
  * beta on a library copy stream (overlapping that preparation) in up to 4 chunks
- * for large N, evaluating chunk c while chunk c + 1 uploads and downloading its V
- * while chunk c + 1 evaluates, and returns after V is in host memory.  Pinned host memory gives the fastest
- * copies; pageable memory works. */
+ * for large N -- by default, for N >= 2 waves of 128-target tiles, a first chunk
+ * of exactly one wave and the rest in one (KS_OPT_EVAL_CHUNK0 / _CHUNKS) --
+ * evaluating chunk c while chunk c + 1 uploads and downloading its V while
+ * chunk c + 1 evaluates, and returns after V is in host memory.  Pinned host
+ * memory gives the fastest copies; pageable memory works.
+ * ks_set_sources (device or host variant) may launch its statistics and
+ * preparation as one cooperative kernel (KS_OPT_COOP_PREP); when the grid does
+ * not fit the SMs available it falls back to separate kernels by itself. */
 KS_API ks_status ks_set_sources_host(ks_ctx *ctx, const float *alpha, const float *W,
                               int64_t M, int R);
 KS_API ks_status ks_eval_host(ks_ctx *ctx, const float *beta, int64_t N, float *V);
