@@ -235,15 +235,16 @@ def _run_any(alpha, W, beta, h, **opts):
 
 @pytest.mark.parametrize("K", [1, 4, 10, 16, 26, 32, 58])
 @pytest.mark.parametrize("M,R,wkind", [(1, 1, "pos"), (777, 1, "signed"), (70001, 1, "pos"), (5000, 3, "signed"),
-                                       (3000, 1, "zero")])
+                                       (3000, 1, "zero"), (150001, 1, "pos")])
 def test_cooperative_source_prep(oracle_mod, K, M, R, wkind):
     """Source statistics + folded source prep in one cooperative launch (option coop_prep, the
     default for the R = 1 and multi-column kernels; a grid barrier between the partial and the
     final statistics) against the separate statistics and prep kernels: the same layout and
     scales, so V agrees to the rounding of mu's FP64 column sums (a different fixed order); the
     result meets the bar and is bitwise reproducible.  Covers one source, ragged counts, more
-    rows than one block's share (70,001), R > 1 (multi-column kernel, no weight statistics),
-    negative weights (the weight mode) and all-zero weights."""
+    rows than one block's share (70,001), blocks whose rows do not fit shared memory at once
+    (150,001 at K >= 39: phase 1 in sub-chunks, phase 3 re-reads L2), R > 1 (multi-column kernel,
+    no weight statistics), negative weights (the weight mode) and all-zero weights."""
     if wkind == "zero":
         a, W, b, h = workloads.custom(M, 300, K, R, 1.0, dist="gm", sigma=0.1, wkind="pos", seed=K + M)
         W = np.zeros_like(W)
