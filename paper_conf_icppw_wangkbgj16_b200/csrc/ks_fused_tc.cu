@@ -1677,7 +1677,7 @@ __device__ __forceinline__ void fold_split_store(const float (&x)[CPL], int K, i
 // or all out: full-mask shuffles).  mu may be global or shared memory; the uniform values (fold
 // shift fsh, scale exponent fexp, log2 max W) are evaluated once per block by the caller.
 template <int CPL>
-__device__ __forceinline__ void fold_source_row(const float* row, const float* wrow,
+__device__ __forceinline__ void fold_source_row(const float* row, const float* wrow, const double* l2w,
                                                 int64_t M, int K, int R, const float (&m)[CPL], double c, bool logw,
                                                 int fsh, int fexp, double lwmax, int64_t i, int g,
                                                 void* __restrict__ src_hi, void* __restrict__ src_lo,
@@ -1702,7 +1702,9 @@ __device__ __forceinline__ void fold_source_row(const float* row, const float* w
     has_np |= d >= K && d < K + 3;
   }
   double wl = 0.0;
-  if (has_np || (g == 0 && logw && rv > 0)) wl = !logw ? 0.0 : live ? log2((double)wrow[0]) - lwmax : -INFINITY;
+  // log2(W_i) (FP64) precomputed by the caller (l2w) or here
+  if (has_np || (g == 0 && logw && rv > 0))
+    wl = !logw ? 0.0 : live ? (l2w != nullptr ? l2w[0] : log2((double)wrow[0])) - lwmax : -INFINITY;
   if (has_np) {
     const double nf = ldexp(-c * n + wl, -fsh);  // W_i = 0: the FP16 stand-in for -inf
     if (nf < -24576.0) np[0] = __float2half(kFoldNegInf);
@@ -1740,7 +1742,7 @@ __global__ void __launch_bounds__(256) prep_fold_sources_kernel(
     const bool logw = wstat != nullptr && wstat[1] == 0u && wstat[0] != 0u && aug < 3;
     float m[CPL];
     fold_lane_mu<CPL>(mu, K, g, m);
-    fold_source_row<CPL>(alpha + i * K, W + i * R, M, K, R, m, c, logw, s_fsh, s_fexp, s_lwmax, i, g, src_hi, src_lo, na, wv,
+    fold_source_row<CPL>(alpha + i * K, W + i * R, nullptr, M, K, R, m, c, logw, s_fsh, s_fexp, s_lwmax, i, g, src_hi, src_lo, na, wv,
                          rv);
   }
   // PDL trigger last: a dependent fused kernel's CTA (640 threads, nearly all of an SM's registers)
@@ -1798,8 +1800,9 @@ __global__ void __launch_bounds__(kCoopThreads, 1) prep_fold_sources_coop_kernel
     unsigned* __restrict__ wstat, void* __restrict__ src_hi, void* __restrict__ src_lo, float* __restrict__ na,
     float* __restrict__ wv, int rv, int dbg_stop) {
   constexpr int NT = kCoopThreads;
-  extern __shared__ __align__(16) float s_a[];  // [rows_cap][K], then (R = 1) [rows_cap] weights
+  extern __shared__ __align__(16) float s_a[];  // [rows_cap][K], (R = 1) [rows_cap] weights, their log2
   float* s_wr = s_a + (size_t)rows_cap * K;
+  double* s_l2w = reinterpret_cast<double*>(s_wr + rows_cap);  // rows_cap is a multiple of 64: aligned
   __shared__ double red[NT];
   __shared__ float rmn[NT], rmx[NT];
   __shared__ float s_mu[64];
@@ -1849,7 +1852,10 @@ __global__ void __launch_bounds__(kCoopThreads, 1) prep_fold_sources_coop_kernel
 #pragma unroll 4
       for (int64_t r = r0 + t; r < r1m; r += NT) {
         const float w = W[r];
-        if (staged) s_wr[r - r0] = w;  // phase 3 reads it from here
+        if (staged) {  // phase 3 reads them from here (the FP64 log2 here: one row per thread, no
+          s_wr[r - r0] = w;  // divergent lane-0 work in phase 3's 8-lane row groups)
+          s_l2w[r - r0] = log2((double)w);
+        }
         wm = fmaxf(wm, fabsf(w));
         neg |= (w < 0.f || w != w) ? 1u : 0u;  // NaN weights take the general path
       }
@@ -1976,7 +1982,8 @@ __global__ void __launch_bounds__(kCoopThreads, 1) prep_fold_sources_coop_kernel
       const int64_t i = base + ((t & 31) >> 3);
       const float* row = staged ? s_a + (i - r0) * K : alpha + i * K;
       const float* wrow = (staged && R == 1) ? s_wr + (i - r0) : W + i * R;
-      fold_source_row<CPL>(row, wrow, M, K, R, m, c, logw, fsh, fexp, lwmax, i, g, src_hi, src_lo, na, wv, rv);
+      const double* l2w = (staged && R == 1 && want_w) ? s_l2w + (i - r0) : nullptr;
+      fold_source_row<CPL>(row, wrow, l2w, M, K, R, m, c, logw, fsh, fexp, lwmax, i, g, src_hi, src_lo, na, wv, rv);
     }
   }
   coop_grid_depart(bar, nb);
@@ -2174,9 +2181,9 @@ cudaError_t launch_prep_fold_sources_coop(const float* alpha, const float* W, in
                                           void* src_hi, void* src_lo, float* na, float* wv, int rv, cudaStream_t st) {
   const int64_t per = (m_pad + grid - 1) / grid;
   const int64_t chunk = (per + 63) / 64 * 64;
-  int rows_cap = (kCoopSmem / (4 * (K + 1))) / 64 * 64;  // >= 64 rows for K <= 58
+  int rows_cap = (kCoopSmem / (4 * (K + 3))) / 64 * 64;  // >= 64 rows for K <= 58
   if (rows_cap > chunk) rows_cap = (int)chunk;
-  const size_t smem = (size_t)4 * (K + 1) * rows_cap;
+  const size_t smem = (size_t)4 * (K + 3) * rows_cap;  // coordinates, weight, FP64 log2 of the weight
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
   cfg.blockDim = dim3(kCoopThreads);
