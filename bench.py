@@ -83,6 +83,15 @@ def workload_desc(c: workloads.Config) -> str:
             f"W~U[0,1], seeds 2016{c.cfg}+(0,1,2,3)")
 
 
+def effective_gflops(pairs_per_s: float, K: int, R: int) -> dict:
+    """north_star's 'effective GFLOP/s': the pair rate times a fixed per-pair count of the method's
+    arithmetic in its Alg.1 form -- 2K for the -2 alpha^T beta contraction, 2 norm
+    adds, 1 scale by -1/2h^2, 1 exponential, 2R for the weighted sum -- whatever the kernel does."""
+    fpp = 2 * K + 4 + 2 * R
+    return {"value": pairs_per_s * fpp / 1e9, "unit": "GFLOP/s", "flop_per_pair": fpp,
+            "convention": "2K (contraction) + 2 (norm adds) + 1 (scale) + 1 (exp) + 2R (weighted sum)"}
+
+
 def per_pair_ops(K: int, R: int):
     """Algorithmic per-pair work charged to the pipe the FP32 design uses
     (SS7): K FFMA (dot) + 1 FADD (norm init) + R FFMA (weight) on the
@@ -238,7 +247,8 @@ def run_reference(args):
            "config": {"workload": workload_desc(c), "step": f"all {c.M:,} sources x {n} sampled targets"},
            "cpu_baseline": {"value": value, "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
                             "sample": f"per step: all {c.M:,} sources x {n} seeded targets"},
-           "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+           "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+           "effective_gflops": effective_gflops(value, c.K, c.R)}
     print(json.dumps(out), flush=True)
 
 
@@ -605,6 +615,7 @@ def run_ours(args):
                                 info1["r1_epilogue"] == 0 else
                                 {1: "on", 2: "on (|d^2|)", 3: "off"}.get(info1["r1_epilogue"], "on"))},
            "roofline": roof, "e2e": e2e, "clocks": clk_sum, "gpu_launches": launches,
+           "effective_gflops": effective_gflops(value, K, R),
            "gpu": torch.cuda.get_device_name(dev)}
     if energy is not None:
         out["energy"] = energy
@@ -689,7 +700,8 @@ def run_unfused(args):
                       "l2": "flushed before every step"},
            "hbm_bytes_per_pair": bpp,
            "hbm_bound_ms": {k: v * pairs / (load_peaks().get("hbm_gbs", 6545.9) * 1e9) * 1e3 for k, v in bpp.items()},
-           "clocks": clk.summary(), "gpu": torch.cuda.get_device_name(dev)}
+           "clocks": clk.summary(), "gpu": torch.cuda.get_device_name(dev),
+           "effective_gflops": effective_gflops(pairs / (ms / 1e3), K, R)}
     if energy is not None:
         out["energy"] = energy
     if not args.no_cpu_baseline:
