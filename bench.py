@@ -175,6 +175,9 @@ def energy_per_step(step, dev_index: int, seconds: float, sync):
         e1 = pynvml.nvmlDeviceGetTotalEnergyConsumption(hdl)
         j = (e1 - e0) / 1e3
         out = {"j_per_step": j / n, "avg_power_w": j / dt, "steps": n, "seconds": dt,
+               # back-to-back steps for >= `seconds` (no L2 flush between them): the rate once the
+               # board has settled at its power cap, beside the short timed window's
+               "sustained_ms_per_step": 1e3 * dt / n,
                "source": "nvmlDeviceGetTotalEnergyConsumption (board, mJ), whole steps incl. L2 flush-free loop"}
         try:  # the board cap the steps ran against (SS6: the headline is power-bound)
             out["power_limit_w"] = pynvml.nvmlDeviceGetEnforcedPowerLimit(hdl) / 1e3
